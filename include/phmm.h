@@ -1,0 +1,171 @@
+/*
+ * phmm.h -- C ABI of the B200-native batched PairHMM forward library
+ * (libphmm.so, sm_100a). No C++ types, exceptions or torch types cross it.
+ *
+ * Operation (J. Wang, X. Xie, J. Cong, "Communication Optimization on GPU:
+ * A Case Study of Sequence Alignment Algorithms", IPDPS 2017, PAPER.md):
+ *   A task is "a pair of sequences" (L22@4659, §V-B); tasks are batched per
+ *   region, one batch per launch (L24@575). For every (read, haplotype) pair
+ *   the library evaluates the PairHMM forward recurrence of Eq. 6
+ *   (L18@541, §III-B):
+ *     M(i,j) = P(i,j) * (alpha*M(i-1,j-1) + beta*I(i-1,j-1) + gamma*D(i-1,j-1))
+ *     I(i,j) = delta*M(i-1,j) + eps*I(i-1,j)
+ *     D(i,j) = zeta*M(i,j-1) + mu*D(i,j-1)
+ *   read = rows i = 1..m, haplotype = columns j = 1..N, and returns "one
+ *   single number" per pair (L18@1062): log10 of the sum of the last row of
+ *   M and I (L20@2262, §IV-C.1; reading R1).
+ *   The Phred -> probability mapping of alpha..mu and P(i,j), and the initial
+ *   row D(0,j) = 1/N, follow GATK 3.6 (L22@4113; readings R2-R6):
+ *     e(Q) = 10^(-Q/10); alpha = 1 - min(1, e(qi)+e(qd)); beta = gamma = 1 - e(qg);
+ *     delta = e(qi); eps = mu = e(qg); zeta = e(qd);
+ *     P = 1 - e(q) if bases match or either is 'N', else e(q)/3.
+ *   Precision (reading R7): PHMM_PREC_FP32_RESCUE computes in FP32 with the
+ *   initial row scaled by 2^120 and re-runs, in FP64 scaled by 2^1020, every
+ *   pair whose scaled FP32 sum is < 1e-28 or not finite; PHMM_PREC_FP64 runs
+ *   every pair in FP64.
+ *
+ * Ownership: the caller owns every input and output buffer. The library reads
+ * the inputs during the call (the host variant copies them to the device),
+ * keeps no pointer to them after return, and writes only out_log10 /
+ * out_status. Device workspace is owned by the context and reused across
+ * calls (grown on demand).
+ *
+ * Errors: every call validates its arguments and inputs before any output is
+ * written; on error it returns a negative status and leaves the outputs
+ * untouched. Input-content errors (bad base, quality > 127, empty sequence,
+ * pair index out of range) are detected on the device in the same pass that
+ * reads the data; the call then returns the error without writing outputs.
+ * CUDA failures return PHMM_E_CUDA. A context is bound to one device, is not
+ * thread-safe, and holds no global state: use one context per host thread.
+ */
+#ifndef PHMM_H_
+#define PHMM_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PHMM_ABI_VERSION 1
+
+typedef struct phmm_ctx phmm_ctx; /* opaque */
+
+typedef enum {
+  PHMM_OK = 0,
+  PHMM_E_INVALID_ARG = -1,  /* NULL pointer, negative count, bad offsets, bad config */
+  PHMM_E_INVALID_BASE = -2, /* a base outside 'A','C','G','T','N' (uppercase only) */
+  PHMM_E_INVALID_QUAL = -3, /* a quality > 127 */
+  PHMM_E_EMPTY_SEQ = -4,    /* a read or haplotype of length 0 used by a pair */
+  PHMM_E_INDEX = -5,        /* a pair's read or haplotype index out of range */
+  PHMM_E_CUDA = -6,         /* a CUDA runtime error */
+  PHMM_E_OOM = -7           /* device or pinned-host allocation failed */
+} phmm_status;
+
+typedef enum {
+  PHMM_PREC_FP64 = 0,        /* every pair in FP64 (scale 2^1020) */
+  PHMM_PREC_FP32_RESCUE = 1  /* FP32 (scale 2^120) + FP64 re-run of underflowing pairs */
+} phmm_precision;
+
+/* per-pair status byte written to out_status */
+enum { PHMM_PAIR_OK = 0, PHMM_PAIR_RESCUED = 1, PHMM_PAIR_FP64_UNDERFLOW = 2 };
+
+/* config flags */
+#define PHMM_FLAG_TIMING 1u /* record CUDA events around each phase; see phmm_get_timing */
+
+typedef struct {
+  int device;               /* CUDA device ordinal */
+  phmm_precision precision; /* default PHMM_PREC_FP32_RESCUE */
+  void* cuda_stream;        /* cudaStream_t to run on; NULL = a context-owned stream */
+  uint32_t flags;           /* PHMM_FLAG_* */
+  int32_t col_bucket;       /* haplotype-length bin width in columns (0 = default 4) */
+} phmm_config;
+
+/*
+ * A batch. Reads and their four quality arrays share one layout: read r is
+ * bytes [read_offsets[r], read_offsets[r+1]) of each array. Haplotype h is
+ * bytes [hap_offsets[h], hap_offsets[h+1]) of hap_bases. Offsets are int64,
+ * non-decreasing, start at 0. pairs[2p] = read index, pairs[2p+1] = haplotype
+ * index of pair p. Bases are ASCII 'A','C','G','T','N'; qualities are raw
+ * Phred integers 0..127 (NOT ASCII+33). For phmm_compute_batch every pointer
+ * is a host pointer; for phmm_compute_batch_dev every array pointer is a
+ * device pointer (the struct itself lives on the host).
+ */
+typedef struct {
+  const uint8_t* read_bases;
+  const uint8_t* base_quals; /* per read base: base quality q_i */
+  const uint8_t* ins_quals;  /* per read base: insertion (gap-open) quality qi_i */
+  const uint8_t* del_quals;  /* per read base: deletion (gap-open) quality qd_i */
+  const uint8_t* gcp_quals;  /* per read base: gap-continuation quality qg_i */
+  const int64_t* read_offsets; /* n_reads + 1 */
+  int64_t n_reads;
+  const uint8_t* hap_bases;
+  const int64_t* hap_offsets;  /* n_haps + 1 */
+  int64_t n_haps;
+  const int32_t* pairs;        /* 2 * n_pairs: (read_idx, hap_idx) */
+  int64_t n_pairs;
+  int64_t total_read_bases;    /* = read_offsets[n_reads] (required by the _dev variant) */
+  int64_t total_hap_bases;     /* = hap_offsets[n_haps]  (required by the _dev variant) */
+} phmm_batch;
+
+/* Create a context on cfg->device (cfg may be NULL: device 0, FP32+rescue). */
+phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg);
+
+/*
+ * Host-buffer variant. Copies the batch to the device (pinned staging,
+ * async H2D on the context stream), runs the whole path, copies the results
+ * back and returns when out_log10 (n_pairs doubles, caller-owned host memory)
+ * and, if non-NULL, out_status (n_pairs bytes) are written.
+ * out_log10[p] = log10 P(read | hap) of pair p; -inf when P underflows even
+ * the FP64 rescue or is exactly 0 (Q0 inputs).
+ */
+phmm_status phmm_compute_batch(phmm_ctx* ctx, const phmm_batch* b, double* out_log10,
+                               uint8_t* out_status);
+
+/*
+ * Device-buffer variant (for torch tensors): every array in *b, dev_out_log10
+ * and dev_out_status (optional) are device pointers on the context's device.
+ * Work is enqueued on the context stream; the call synchronises that stream
+ * once at the end to report input-content errors, so outputs are final when
+ * it returns PHMM_OK.
+ */
+phmm_status phmm_compute_batch_dev(phmm_ctx* ctx, const phmm_batch* b, double* dev_out_log10,
+                                   uint8_t* dev_out_status);
+
+/* Release the context and its device workspace. NULL-safe, idempotent per pointer. */
+void phmm_destroy(phmm_ctx* ctx);
+
+/* Static string for a status code. */
+const char* phmm_status_string(phmm_status s);
+
+/*
+ * Statistics of the last successful compute call on ctx.
+ * timing fields are filled only with PHMM_FLAG_TIMING (milliseconds, CUDA
+ * events on the context stream), else set to -1.
+ */
+typedef struct {
+  int64_t n_pairs;
+  int64_t cells;            /* sum of m*N over pairs (the paper's cell count, L22@1416) */
+  int64_t padded_cells;     /* cells the wavefront kernels actually computed (pad rows/cols) */
+  int64_t n_rescued;        /* pairs re-run in FP64 */
+  int64_t n_fp64_underflow; /* pairs whose FP64 sum was 0 or subnormal */
+  int32_t n_bins;           /* haplotype-length bins of the FP32 pass */
+  int32_t kernel_launches;  /* kernels launched by the call */
+  float ms_total;           /* whole call on the stream (device side) */
+  float ms_h2d;             /* host->device copies (host variant only) */
+  float ms_prep;            /* validation, per-read tables, binning */
+  float ms_wavefront;       /* main wavefront kernel (FP32 or FP64 mode) */
+  float ms_rescue;          /* FP64 rescue pass (prep + wavefront) */
+  float ms_finalize;        /* log10 + scatter */
+  float ms_d2h;             /* device->host copy (host variant only) */
+} phmm_stats;
+
+phmm_status phmm_get_stats(const phmm_ctx* ctx, phmm_stats* out);
+
+/* ABI version of the loaded library (PHMM_ABI_VERSION). */
+int phmm_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PHMM_H_ */

@@ -1,0 +1,636 @@
+// phmm_lib.cu -- host side of libphmm: the C ABI of include/phmm.h.
+//
+// PRODUCT PATH (no oracle code). Orchestrates, on one stream:
+//   validate + haplotype codes -> per pass: bin pairs by column count,
+//   per-read coefficient tables (the per-read precompute step),
+//   block allocation per bin (the length-binned scheduler, §8a-3), the
+//   wavefront kernel (§8a-4), finalize (§8a-5) and, for FP32, the FP64
+//   rescue of underflowing pairs (§8a-6). See DESIGN.md §3-§5.
+#include <cub/device/device_scan.cuh>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+
+#include "../../include/phmm.h"
+#include "phmm_device.cuh"
+
+using namespace phmm;
+
+namespace {
+
+enum BufId {
+  B_READ_BASES, B_BQ, B_IQ, B_DQ, B_GQ, B_ROFF, B_HAP, B_HOFF, B_PAIRS,  // host-variant inputs
+  B_HCODES, B_SCAL,                                                       // codes, scalars
+  B_PAIR_BIN, B_PAIR_NB, B_BINS, B_ITEM_NB, B_ITEM_OFF, B_SCAN_TMP,
+  B_TAB, B_BLK, B_OUT32, B_OUT64, B_RLIST, B_ITEM_READ, B_PAIR_ITEM,
+  B_OUT_LOG10, B_OUT_STATUS, B_COUNT
+};
+
+struct Buf {
+  void* p = nullptr;
+  size_t n = 0;
+};
+
+// device scalars written by the prep kernels, read back in one D2H copy
+struct Scalars {
+  uint32_t err;
+  int32_t max_ncols;
+  unsigned long long cells;
+  unsigned long long padded_cells;
+  unsigned long long total_blocks;
+  int64_t n_rescue;
+  unsigned long long n_underflow;
+  unsigned int item_counter;
+  unsigned int pad_;
+};
+
+constexpr int kEvents = 10;
+constexpr int kThreads = 256;
+constexpr int kWarpsPerBlock = 4;
+
+// haplotype code padding: columns past N read (finite, unused) codes
+constexpr int64_t kHapPad = 4224;
+
+}  // namespace
+
+struct phmm_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  phmm_precision prec = PHMM_PREC_FP32_RESCUE;
+  uint32_t flags = 0;
+  int bucket = 4;
+  int nsm = 148;
+  Buf buf[B_COUNT];
+  Scalars* host_scal = nullptr;  // pinned
+  cudaEvent_t ev[kEvents] = {};
+  phmm_stats st{};
+  int launches = 0;
+};
+
+namespace {
+
+void debug_cuda(cudaError_t e, const char* what, int line) {
+  if (std::getenv("PHMM_DEBUG"))
+    std::fprintf(stderr, "phmm: %s failed at line %d: %s\n", what, line, cudaGetErrorString(e));
+}
+
+#define CUDA_TRY(x)                   \
+  do {                                \
+    cudaError_t e_ = (x);             \
+    if (e_ != cudaSuccess) {          \
+      debug_cuda(e_, #x, __LINE__);   \
+      cudaGetLastError();             \
+      return PHMM_E_CUDA;             \
+    }                                 \
+  } while (0)
+
+#define ST_TRY(x)                     \
+  do {                                \
+    phmm_status s_ = (x);             \
+    if (s_ != PHMM_OK) return s_;     \
+  } while (0)
+
+#define LAUNCHED(c)                                   \
+  do {                                                \
+    ++(c)->launches;                                  \
+    cudaError_t e_ = cudaGetLastError();              \
+    if (e_ != cudaSuccess) {                          \
+      debug_cuda(e_, "kernel launch", __LINE__);      \
+      return PHMM_E_CUDA;                             \
+    }                                                 \
+  } while (0)
+
+template <class X>
+phmm_status ws(phmm_ctx* c, int id, size_t count, X** out) {
+  size_t bytes = count * sizeof(X);
+  if (bytes < 16) bytes = 16;
+  Buf& b = c->buf[id];
+  if (b.n < bytes) {
+    if (b.p) cudaFree(b.p);
+    b.p = nullptr;
+    b.n = 0;
+    size_t want = bytes + bytes / 8;  // headroom for the next, slightly larger batch
+    if (cudaMalloc(&b.p, want) != cudaSuccess) {
+      cudaGetLastError();
+      if (cudaMalloc(&b.p, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        b.p = nullptr;
+        return PHMM_E_OOM;
+      }
+      want = bytes;
+    }
+    b.n = want;
+  }
+  *out = reinterpret_cast<X*>(b.p);
+  return PHMM_OK;
+}
+
+int grid_for(const phmm_ctx* c, int64_t n) {
+  int64_t g = (n + kThreads - 1) / kThreads;
+  const int64_t cap = (int64_t)c->nsm * 16;
+  if (g > cap) g = cap;
+  if (g < 1) g = 1;
+  return (int)g;
+}
+
+phmm_status map_err(uint32_t e) {
+  if (e & ERR_INDEX) return PHMM_E_INDEX;
+  if (e & ERR_ARG) return PHMM_E_INVALID_ARG;
+  if (e & ERR_EMPTY) return PHMM_E_EMPTY_SEQ;
+  if (e & ERR_BASE) return PHMM_E_INVALID_BASE;
+  if (e & ERR_QUAL) return PHMM_E_INVALID_QUAL;
+  return PHMM_E_INVALID_ARG;
+}
+
+enum { EV_START, EV_H2D, EV_PREP, EV_WF0, EV_WF1, EV_RESC0, EV_RESC1, EV_FIN, EV_D2H, EV_END };
+
+void ev_record(phmm_ctx* c, int i) {
+  if (c->flags & PHMM_FLAG_TIMING) cudaEventRecord(c->ev[i], c->stream);
+}
+float ev_ms(phmm_ctx* c, int a, int b) {
+  if (!(c->flags & PHMM_FLAG_TIMING)) return -1.f;
+  float ms = -1.f;
+  if (cudaEventElapsedTime(&ms, c->ev[a], c->ev[b]) != cudaSuccess) {
+    cudaGetLastError();
+    return -1.f;
+  }
+  return ms;
+}
+
+// device view of a batch
+struct DevBatch {
+  const uint8_t *rb, *q, *qi, *qd, *qg, *hap;
+  const int64_t *roff, *hoff;
+  const int32_t* pairs;
+  int64_t n_reads, n_haps, n_pairs, n_rb, n_hb;
+};
+
+struct PassInfo {
+  unsigned long long cells = 0, padded_cells = 0, total_blocks = 0;
+  int max_ncols = 0;
+};
+
+// Validation of the whole batch + haplotype one-hot codes. Errors land in scal->err.
+phmm_status run_validate(phmm_ctx* c, const DevBatch& d, uint8_t** hcodes_out) {
+  cudaStream_t s = c->stream;
+  Scalars* scal;
+  uint8_t* hcodes;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  ST_TRY(ws(c, B_HCODES, (size_t)(d.n_hb + kHapPad), &hcodes));
+  CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
+  CUDA_TRY(cudaMemsetAsync(hcodes + d.n_hb, 0, kHapPad, s));
+  if (d.n_hb > 0) {
+    k_hap_codes<<<grid_for(c, d.n_hb), kThreads, 0, s>>>(d.hap, d.n_hb, hcodes, &scal->err);
+    LAUNCHED(c);
+  }
+  if (d.n_rb > 0) {
+    k_validate_reads<<<grid_for(c, d.n_rb), kThreads, 0, s>>>(d.rb, d.q, d.qi, d.qd, d.qg, d.n_rb, &scal->err);
+    LAUNCHED(c);
+  }
+  k_validate_offsets<<<grid_for(c, d.n_reads + 1), kThreads, 0, s>>>(d.roff, d.n_reads, d.n_rb, &scal->err);
+  LAUNCHED(c);
+  k_validate_offsets<<<grid_for(c, d.n_haps + 1), kThreads, 0, s>>>(d.hoff, d.n_haps, d.n_hb, &scal->err);
+  LAUNCHED(c);
+  *hcodes_out = hcodes;
+  return PHMM_OK;
+}
+
+// Part 1 of a pass: bin the pairs, size the table. Ends with one D2H + sync
+// (sizes for the allocations; input-content errors are reported here, before
+// any output is written).
+//   list == nullptr: all pairs, table items = reads, output slot = pair id
+//   list != nullptr: the n listed pairs, one table item per listed pair,
+//                    output slot = position in the list
+template <typename T, int K>
+phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_t n, PassInfo* pi,
+                         int64_t* total_tab_out) {
+  cudaStream_t s = c->stream;
+  Scalars* scal;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  const int nb1 = kMaxBins + 2;
+  unsigned long long* bins;  // [blocks | pairs | cursor | start | item_start], nb1 each
+  ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
+  int32_t *pair_bin, *pair_nb;
+  ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
+  ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
+  CUDA_TRY(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * 3 * nb1, s));
+  // per-pass scalars (err is kept: it accumulates validation errors)
+  CUDA_TRY(cudaMemsetAsync(&scal->max_ncols, 0, offsetof(Scalars, n_rescue) - offsetof(Scalars, max_ncols), s));
+  CUDA_TRY(cudaMemsetAsync(&scal->item_counter, 0, sizeof(unsigned int), s));
+
+  k_pair_bins<K><<<grid_for(c, n), kThreads, 0, s>>>(
+      d.pairs, list, nullptr, n, d.roff, d.n_reads, d.hoff, d.n_haps, c->bucket, pair_bin, pair_nb, bins,
+      bins + nb1, &scal->max_ncols, &scal->cells, &scal->padded_cells, &scal->total_blocks, &scal->err);
+  LAUNCHED(c);
+
+  // table items and their block offsets (exclusive scan over n_items + 1)
+  const int64_t n_items = list ? n : d.n_reads;
+  int32_t* item_read = nullptr;
+  if (list) {
+    int32_t* pair_item;
+    ST_TRY(ws(c, B_ITEM_READ, (size_t)n, &item_read));
+    ST_TRY(ws(c, B_PAIR_ITEM, (size_t)n, &pair_item));
+    k_rescue_items<<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, n, item_read, pair_item);
+    LAUNCHED(c);
+  }
+  int64_t *item_nb, *item_off;
+  ST_TRY(ws(c, B_ITEM_NB, (size_t)n_items + 1, &item_nb));
+  ST_TRY(ws(c, B_ITEM_OFF, (size_t)n_items + 1, &item_off));
+  k_item_nblocks<K><<<grid_for(c, n_items), kThreads, 0, s>>>(item_read, n_items, nullptr, d.roff, item_nb);
+  LAUNCHED(c);
+  size_t tmp_bytes = 0;
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, item_nb, item_off, (int64_t)(n_items + 1), s));
+  unsigned char* tmp;
+  ST_TRY(ws(c, B_SCAN_TMP, tmp_bytes, &tmp));
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, item_nb, item_off, (int64_t)(n_items + 1), s));
+  ++c->launches;
+
+  // one small D2H: sizes + error flag
+  CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+  int64_t total_tab = 0;
+  CUDA_TRY(cudaMemcpyAsync(&total_tab, item_off + n_items, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  if (c->host_scal->err) return map_err(c->host_scal->err);
+  pi->cells = c->host_scal->cells;
+  pi->padded_cells = c->host_scal->padded_cells;
+  pi->total_blocks = c->host_scal->total_blocks;
+  pi->max_ncols = c->host_scal->max_ncols;
+  *total_tab_out = total_tab;
+  return PHMM_OK;
+}
+
+// Part 2 of a pass: tables, block sequence, wavefront. Writes out[slot] = scaled sum.
+template <typename T, int K>
+phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const uint8_t* hcodes, const int32_t* list, int64_t n,
+                     const PassInfo& pi, int64_t total_tab, T* out, int* nbins_used) {
+  cudaStream_t s = c->stream;
+  Scalars* scal;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  const int nb1 = kMaxBins + 2;
+  unsigned long long* bins;
+  ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
+  unsigned long long *bin_blocks = bins, *bin_cursor = bins + 2 * nb1, *bin_start = bins + 3 * nb1,
+                     *item_start = bins + 4 * nb1;
+  int32_t *pair_bin, *pair_nb, *item_read = nullptr, *pair_item = nullptr;
+  ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
+  ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
+  const int64_t n_items = list ? n : d.n_reads;
+  if (list) {
+    ST_TRY(ws(c, B_ITEM_READ, (size_t)n, &item_read));
+    ST_TRY(ws(c, B_PAIR_ITEM, (size_t)n, &pair_item));
+  }
+  int64_t* item_off;
+  ST_TRY(ws(c, B_ITEM_OFF, (size_t)n_items + 1, &item_off));
+  TabBlock<T, K>* tab;
+  BlkDesc* blk;
+  ST_TRY(ws(c, B_TAB, (size_t)total_tab, &tab));
+  ST_TRY(ws(c, B_BLK, (size_t)pi.total_blocks, &blk));
+
+  // per-read (or per-rescued-pair) coefficient tables
+  if (total_tab > 0) {
+    k_build_table<T, K><<<grid_for(c, total_tab * K), kThreads, 0, s>>>(
+        item_read, nullptr, n_items, item_off, item_off + n_items, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
+    LAUNCHED(c);
+  }
+
+  // warps and work-item size
+  const size_t ring_bytes = (size_t)pi.max_ncols * sizeof(RingEnt<T>);
+  const size_t smem = ring_bytes * kWarpsPerBlock;
+  CUDA_TRY(cudaFuncSetAttribute(k_wavefront<T, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int bps = 0;
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_wavefront<T, K>, kWarpsPerBlock * 32, smem));
+  if (bps < 1) return PHMM_E_INVALID_ARG;  // haplotype too long for the shared-memory ring
+  const int64_t nwarps = (int64_t)c->nsm * bps * kWarpsPerBlock;
+  int64_t chunk = (int64_t)(pi.total_blocks / (unsigned long long)(nwarps * 6));
+  if (chunk < 128) chunk = 128;
+  if (chunk > 16384) chunk = 16384;
+
+  const int nbins = kMaxBins + 1;
+  k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, chunk, bin_start, item_start);
+  LAUNCHED(c);
+  k_alloc_blocks<K><<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, nullptr, n, pair_bin, pair_nb, bin_start,
+                                                        bin_cursor, d.hoff, item_off, pair_item, list ? 1 : 0, blk);
+  LAUNCHED(c);
+
+  WfArgs<T> A;
+  A.blk = blk;
+  A.tab = tab;
+  A.hcodes = hcodes;
+  A.bin_start = bin_start;
+  A.item_start = item_start;
+  A.nbins = nbins;
+  A.bucket = c->bucket;
+  A.chunk_blocks = chunk;
+  A.item_counter = &scal->item_counter;
+  A.out = out;
+  A.ring_len = pi.max_ncols;
+  CUDA_TRY(cudaMemsetAsync(&scal->item_counter, 0, sizeof(unsigned int), s));
+  const bool timing_wf = (sizeof(T) == 4 || c->prec == PHMM_PREC_FP64);
+  if (timing_wf) ev_record(c, EV_WF0);
+  k_wavefront<T, K><<<(unsigned)(c->nsm * bps), kWarpsPerBlock * 32, smem, s>>>(A);
+  LAUNCHED(c);
+  if (timing_wf) ev_record(c, EV_WF1);
+  if (nbins_used) *nbins_used = 0;
+  return PHMM_OK;
+}
+
+constexpr int K32 = 8;  // rows per lane, FP32 pass
+constexpr int K64 = 4;  // rows per lane, FP64 pass
+
+// The whole path on device-resident inputs. Writes dev_out (+ dev_status).
+phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status) {
+  cudaStream_t s = c->stream;
+  c->st = phmm_stats{};
+  c->st.n_pairs = d.n_pairs;
+  if (d.n_pairs == 0) return PHMM_OK;
+  uint8_t* hcodes = nullptr;
+  ST_TRY(run_validate(c, d, &hcodes));
+  PassInfo pi;
+  int64_t total_tab = 0;
+  Scalars* scal;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  if (c->prec == PHMM_PREC_FP64) {
+    ST_TRY((pass_prepare<double, K64>(c, d, nullptr, d.n_pairs, &pi, &total_tab)));
+    double* out64;
+    ST_TRY(ws(c, B_OUT64, (size_t)d.n_pairs, &out64));
+    ev_record(c, EV_PREP);
+    ST_TRY((pass_run<double, K64>(c, d, hcodes, nullptr, d.n_pairs, pi, total_tab, out64, nullptr)));
+    CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
+    k_finalize_fp64<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out64, nullptr, nullptr, d.n_pairs, d.pairs,
+                                                                  d.hoff, c->bucket, dev_out,
+                                                                  dev_status, dev_status != nullptr, 0,
+                                                                  &scal->n_underflow);
+    LAUNCHED(c);
+    ev_record(c, EV_FIN);
+    CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
+  } else {
+    ST_TRY((pass_prepare<float, K32>(c, d, nullptr, d.n_pairs, &pi, &total_tab)));
+    float* out32;
+    ST_TRY(ws(c, B_OUT32, (size_t)d.n_pairs, &out32));
+    ev_record(c, EV_PREP);
+    ST_TRY((pass_run<float, K32>(c, d, hcodes, nullptr, d.n_pairs, pi, total_tab, out32, nullptr)));
+    int32_t* rlist;
+    ST_TRY(ws(c, B_RLIST, (size_t)d.n_pairs, &rlist));
+    CUDA_TRY(cudaMemsetAsync(&scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
+    k_finalize_fp32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out32, d.n_pairs, d.pairs, d.hoff, c->bucket,
+                                                                  dev_out, dev_status, rlist,
+                                                                  &scal->n_rescue, dev_status != nullptr);
+    LAUNCHED(c);
+    ev_record(c, EV_RESC0);
+    CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    const int64_t nr = c->host_scal->n_rescue;
+    c->st.n_rescued = nr;
+    if (nr > 0) {
+      PassInfo pr;
+      int64_t tab_r = 0;
+      ST_TRY((pass_prepare<double, K64>(c, d, rlist, nr, &pr, &tab_r)));
+      double* out64;
+      ST_TRY(ws(c, B_OUT64, (size_t)nr, &out64));
+      ST_TRY((pass_run<double, K64>(c, d, hcodes, rlist, nr, pr, tab_r, out64, nullptr)));
+      CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
+      k_finalize_fp64<<<grid_for(c, nr), kThreads, 0, s>>>(out64, rlist, nullptr, nr, d.pairs, d.hoff, c->bucket,
+                                                           dev_out, dev_status,
+                                                           dev_status != nullptr, 1, &scal->n_underflow);
+      LAUNCHED(c);
+      c->st.padded_cells += (int64_t)pr.padded_cells;
+    }
+    ev_record(c, EV_RESC1);
+    if (nr > 0) {
+      CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+      CUDA_TRY(cudaStreamSynchronize(s));
+      c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
+    }
+  }
+  c->st.cells = (int64_t)pi.cells;
+  c->st.padded_cells += (int64_t)pi.padded_cells;
+  return PHMM_OK;
+}
+
+phmm_status check_batch_args(const phmm_batch* b) {
+  if (!b) return PHMM_E_INVALID_ARG;
+  if (b->n_reads < 0 || b->n_haps < 0 || b->n_pairs < 0) return PHMM_E_INVALID_ARG;
+  if (b->n_pairs > 0x7fffffffLL || b->n_reads > 0x7fffffffLL || b->n_haps > 0x7fffffffLL) return PHMM_E_INVALID_ARG;
+  if (b->n_pairs == 0) return PHMM_OK;
+  if (!b->pairs || !b->read_offsets || !b->hap_offsets) return PHMM_E_INVALID_ARG;
+  if (b->total_read_bases < 0 || b->total_hap_bases < 0) return PHMM_E_INVALID_ARG;
+  if (b->total_hap_bases >= 0xffffffffLL - kHapPad) return PHMM_E_INVALID_ARG;
+  if (b->total_read_bases > 0 &&
+      (!b->read_bases || !b->base_quals || !b->ins_quals || !b->del_quals || !b->gcp_quals))
+    return PHMM_E_INVALID_ARG;
+  if (b->total_hap_bases > 0 && !b->hap_bases) return PHMM_E_INVALID_ARG;
+  return PHMM_OK;
+}
+
+void finish_stats(phmm_ctx* c) {
+  c->st.kernel_launches = c->launches;
+  if (c->flags & PHMM_FLAG_TIMING) {
+    cudaEventSynchronize(c->ev[EV_END]);
+    c->st.ms_total = ev_ms(c, EV_START, EV_END);
+    c->st.ms_wavefront = ev_ms(c, EV_WF0, EV_WF1);
+    if (c->prec == PHMM_PREC_FP64) {
+      c->st.ms_prep = ev_ms(c, EV_H2D, EV_PREP);
+      c->st.ms_finalize = ev_ms(c, EV_WF1, EV_FIN);
+      c->st.ms_rescue = 0.f;
+    } else {
+      c->st.ms_prep = ev_ms(c, EV_H2D, EV_PREP);
+      c->st.ms_finalize = ev_ms(c, EV_WF1, EV_RESC0);
+      c->st.ms_rescue = ev_ms(c, EV_RESC0, EV_RESC1);
+    }
+  } else {
+    c->st.ms_total = c->st.ms_h2d = c->st.ms_prep = c->st.ms_wavefront = -1.f;
+    c->st.ms_rescue = c->st.ms_finalize = c->st.ms_d2h = -1.f;
+  }
+}
+
+}  // namespace
+
+extern "C" {
+
+int phmm_abi_version(void) { return PHMM_ABI_VERSION; }
+
+const char* phmm_status_string(phmm_status s) {
+  switch (s) {
+    case PHMM_OK: return "ok";
+    case PHMM_E_INVALID_ARG: return "invalid argument";
+    case PHMM_E_INVALID_BASE: return "invalid base (expected A, C, G, T or N)";
+    case PHMM_E_INVALID_QUAL: return "invalid quality (> 127)";
+    case PHMM_E_EMPTY_SEQ: return "empty read or haplotype";
+    case PHMM_E_INDEX: return "pair index out of range";
+    case PHMM_E_CUDA: return "CUDA error";
+    case PHMM_E_OOM: return "out of memory";
+  }
+  return "unknown status";
+}
+
+phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
+  if (!out) return PHMM_E_INVALID_ARG;
+  *out = nullptr;
+  phmm_config def{};
+  def.device = 0;
+  def.precision = PHMM_PREC_FP32_RESCUE;
+  def.cuda_stream = nullptr;
+  def.flags = 0;
+  def.col_bucket = 0;
+  if (!cfg) cfg = &def;
+  if (cfg->precision != PHMM_PREC_FP64 && cfg->precision != PHMM_PREC_FP32_RESCUE) return PHMM_E_INVALID_ARG;
+  if (cfg->col_bucket < 0 || cfg->col_bucket > 64) return PHMM_E_INVALID_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) return PHMM_E_INVALID_ARG;
+  phmm_ctx* c = new (std::nothrow) phmm_ctx();
+  if (!c) return PHMM_E_OOM;
+  c->device = cfg->device;
+  c->prec = cfg->precision;
+  c->flags = cfg->flags;
+  c->bucket = cfg->col_bucket > 0 ? cfg->col_bucket : 4;
+  auto fail = [&](phmm_status s) {
+    phmm_destroy(c);
+    return s;
+  };
+  if (cudaSetDevice(c->device) != cudaSuccess) return fail(PHMM_E_CUDA);
+  if (cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess)
+    return fail(PHMM_E_CUDA);
+  if (cfg->cuda_stream) {
+    c->stream = reinterpret_cast<cudaStream_t>(cfg->cuda_stream);
+  } else {
+    if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) return fail(PHMM_E_CUDA);
+    c->own_stream = true;
+  }
+  if (cudaMallocHost(&c->host_scal, sizeof(Scalars)) != cudaSuccess) {
+    c->host_scal = nullptr;
+    return fail(PHMM_E_OOM);
+  }
+  for (int i = 0; i < kEvents; ++i)
+    if (cudaEventCreate(&c->ev[i]) != cudaSuccess) return fail(PHMM_E_CUDA);
+  *out = c;
+  return PHMM_OK;
+}
+
+void phmm_destroy(phmm_ctx* c) {
+  if (!c) return;
+  cudaSetDevice(c->device);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  for (int i = 0; i < B_COUNT; ++i)
+    if (c->buf[i].p) cudaFree(c->buf[i].p);
+  for (int i = 0; i < kEvents; ++i)
+    if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  if (c->host_scal) cudaFreeHost(c->host_scal);
+  if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+  cudaGetLastError();
+  delete c;
+}
+
+phmm_status phmm_get_stats(const phmm_ctx* c, phmm_stats* out) {
+  if (!c || !out) return PHMM_E_INVALID_ARG;
+  *out = c->st;
+  return PHMM_OK;
+}
+
+phmm_status phmm_compute_batch_dev(phmm_ctx* c, const phmm_batch* b, double* dev_out, uint8_t* dev_status) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  ST_TRY(check_batch_args(b));
+  if (b->n_pairs > 0 && !dev_out) return PHMM_E_INVALID_ARG;
+  if (cudaSetDevice(c->device) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  c->launches = 0;
+  DevBatch d{b->read_bases, b->base_quals, b->ins_quals, b->del_quals, b->gcp_quals, b->hap_bases,
+             b->read_offsets, b->hap_offsets, b->pairs, b->n_reads, b->n_haps, b->n_pairs,
+             b->total_read_bases, b->total_hap_bases};
+  ev_record(c, EV_START);
+  ev_record(c, EV_H2D);
+  phmm_status st = compute_dev(c, d, dev_out, dev_status);
+  if (st != PHMM_OK) {
+    cudaStreamSynchronize(c->stream);
+    cudaGetLastError();
+    return st;
+  }
+  ev_record(c, EV_END);
+  if (cudaStreamSynchronize(c->stream) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  finish_stats(c);
+  c->st.ms_h2d = 0.f;
+  c->st.ms_d2h = 0.f;
+  return PHMM_OK;
+}
+
+phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  ST_TRY(check_batch_args(b));
+  if (b->n_pairs > 0 && !out_log10) return PHMM_E_INVALID_ARG;
+  if (cudaSetDevice(c->device) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  c->launches = 0;
+  if (b->n_pairs == 0) {
+    c->st = phmm_stats{};
+    return PHMM_OK;
+  }
+  // host-side size checks that need the host offsets
+  if (b->read_offsets[b->n_reads] != b->total_read_bases || b->hap_offsets[b->n_haps] != b->total_hap_bases)
+    return PHMM_E_INVALID_ARG;
+  cudaStream_t s = c->stream;
+  uint8_t *rb, *q, *qi, *qd, *qg, *hap;
+  int64_t *roff, *hoff;
+  int32_t* pairs;
+  double* out;
+  uint8_t* status = nullptr;
+  const size_t nr = (size_t)b->total_read_bases, nh = (size_t)b->total_hap_bases;
+  ST_TRY(ws(c, B_READ_BASES, nr, &rb));
+  ST_TRY(ws(c, B_BQ, nr, &q));
+  ST_TRY(ws(c, B_IQ, nr, &qi));
+  ST_TRY(ws(c, B_DQ, nr, &qd));
+  ST_TRY(ws(c, B_GQ, nr, &qg));
+  ST_TRY(ws(c, B_HAP, nh, &hap));
+  ST_TRY(ws(c, B_ROFF, (size_t)b->n_reads + 1, &roff));
+  ST_TRY(ws(c, B_HOFF, (size_t)b->n_haps + 1, &hoff));
+  ST_TRY(ws(c, B_PAIRS, (size_t)b->n_pairs * 2, &pairs));
+  ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
+  if (out_status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
+  ev_record(c, EV_START);
+  if (nr) {
+    CUDA_TRY(cudaMemcpyAsync(rb, b->read_bases, nr, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaMemcpyAsync(q, b->base_quals, nr, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaMemcpyAsync(qi, b->ins_quals, nr, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaMemcpyAsync(qd, b->del_quals, nr, cudaMemcpyHostToDevice, s));
+    CUDA_TRY(cudaMemcpyAsync(qg, b->gcp_quals, nr, cudaMemcpyHostToDevice, s));
+  }
+  if (nh) CUDA_TRY(cudaMemcpyAsync(hap, b->hap_bases, nh, cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(roff, b->read_offsets, sizeof(int64_t) * (b->n_reads + 1), cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(hoff, b->hap_offsets, sizeof(int64_t) * (b->n_haps + 1), cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(pairs, b->pairs, sizeof(int32_t) * 2 * b->n_pairs, cudaMemcpyHostToDevice, s));
+  ev_record(c, EV_H2D);
+  DevBatch d{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs, (int64_t)nr, (int64_t)nh};
+  phmm_status st = compute_dev(c, d, out, status);
+  if (st != PHMM_OK) {
+    cudaStreamSynchronize(s);
+    cudaGetLastError();
+    return st;
+  }
+  ev_record(c, EV_D2H);
+  CUDA_TRY(cudaMemcpyAsync(out_log10, out, sizeof(double) * b->n_pairs, cudaMemcpyDeviceToHost, s));
+  if (out_status) CUDA_TRY(cudaMemcpyAsync(out_status, status, b->n_pairs, cudaMemcpyDeviceToHost, s));
+  ev_record(c, EV_END);
+  CUDA_TRY(cudaStreamSynchronize(s));
+  finish_stats(c);
+  c->st.ms_h2d = ev_ms(c, EV_START, EV_H2D);
+  c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
+  return PHMM_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,279 @@
+"""Thin Python binding of libphmm (include/phmm.h) -- argument marshalling only.
+
+Every step of the PairHMM path (validation, per-read tables, binning, the
+wavefront, the FP64 rescue, log10) runs inside libphmm.so on the GPU. This
+module never computes a likelihood itself and has no CPU fallback: if the
+library cannot be loaded it raises.
+
+Names follow the C ABI: ``phmm_create`` -> ``PairHMM(...)``,
+``phmm_compute_batch`` -> ``PairHMM.compute_batch`` (host buffers),
+``phmm_compute_batch_dev`` -> ``PairHMM.compute_batch_dev`` (torch CUDA
+tensors), ``phmm_destroy`` -> ``PairHMM.close``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+from typing import Optional
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libphmm.so")
+
+PHMM_OK = 0
+STATUS_NAMES = {
+    0: "PHMM_OK", -1: "PHMM_E_INVALID_ARG", -2: "PHMM_E_INVALID_BASE", -3: "PHMM_E_INVALID_QUAL",
+    -4: "PHMM_E_EMPTY_SEQ", -5: "PHMM_E_INDEX", -6: "PHMM_E_CUDA", -7: "PHMM_E_OOM",
+}
+PREC_FP64 = 0
+PREC_FP32_RESCUE = 1
+FLAG_TIMING = 1
+
+_u8p = ctypes.POINTER(ctypes.c_uint8)
+_i64p = ctypes.POINTER(ctypes.c_int64)
+_i32p = ctypes.POINTER(ctypes.c_int32)
+_f64p = ctypes.POINTER(ctypes.c_double)
+
+
+class PhmmError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        self.code = code
+        super().__init__(f"{what}: {STATUS_NAMES.get(code, code)} ({status_string(code)})")
+
+
+class _Config(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("precision", ctypes.c_int), ("cuda_stream", ctypes.c_void_p),
+                ("flags", ctypes.c_uint32), ("col_bucket", ctypes.c_int32)]
+
+
+class _Batch(ctypes.Structure):
+    _fields_ = [("read_bases", ctypes.c_void_p), ("base_quals", ctypes.c_void_p),
+                ("ins_quals", ctypes.c_void_p), ("del_quals", ctypes.c_void_p), ("gcp_quals", ctypes.c_void_p),
+                ("read_offsets", ctypes.c_void_p), ("n_reads", ctypes.c_int64),
+                ("hap_bases", ctypes.c_void_p), ("hap_offsets", ctypes.c_void_p), ("n_haps", ctypes.c_int64),
+                ("pairs", ctypes.c_void_p), ("n_pairs", ctypes.c_int64),
+                ("total_read_bases", ctypes.c_int64), ("total_hap_bases", ctypes.c_int64)]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [("n_pairs", ctypes.c_int64), ("cells", ctypes.c_int64), ("padded_cells", ctypes.c_int64),
+                ("n_rescued", ctypes.c_int64), ("n_fp64_underflow", ctypes.c_int64),
+                ("n_bins", ctypes.c_int32), ("kernel_launches", ctypes.c_int32),
+                ("ms_total", ctypes.c_float), ("ms_h2d", ctypes.c_float), ("ms_prep", ctypes.c_float),
+                ("ms_wavefront", ctypes.c_float), ("ms_rescue", ctypes.c_float),
+                ("ms_finalize", ctypes.c_float), ("ms_d2h", ctypes.c_float)]
+
+
+# every symbol include/phmm.h declares (checked by tests/test_abi.py)
+EXPORTED_SYMBOLS = ("phmm_create", "phmm_compute_batch", "phmm_compute_batch_dev", "phmm_destroy",
+                    "phmm_status_string", "phmm_get_stats", "phmm_abi_version")
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH):
+    """Load libphmm.so (raises if it is missing: there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise RuntimeError(f"libphmm.so not built ({path}); run `python -m paper_conf_ipps_wangxc17_b200.build` "
+                           "or __graft_entry__.build()")
+    L = ctypes.CDLL(path)
+    L.phmm_create.argtypes = [ctypes.POINTER(ctypes.c_void_p), ctypes.POINTER(_Config)]
+    L.phmm_create.restype = ctypes.c_int
+    L.phmm_compute_batch.argtypes = [ctypes.c_void_p, ctypes.POINTER(_Batch), _f64p, _u8p]
+    L.phmm_compute_batch.restype = ctypes.c_int
+    L.phmm_compute_batch_dev.argtypes = [ctypes.c_void_p, ctypes.POINTER(_Batch), ctypes.c_void_p, ctypes.c_void_p]
+    L.phmm_compute_batch_dev.restype = ctypes.c_int
+    L.phmm_destroy.argtypes = [ctypes.c_void_p]
+    L.phmm_destroy.restype = None
+    L.phmm_status_string.argtypes = [ctypes.c_int]
+    L.phmm_status_string.restype = ctypes.c_char_p
+    L.phmm_get_stats.argtypes = [ctypes.c_void_p, ctypes.POINTER(_Stats)]
+    L.phmm_get_stats.restype = ctypes.c_int
+    L.phmm_abi_version.argtypes = []
+    L.phmm_abi_version.restype = ctypes.c_int
+    _lib = L
+    return L
+
+
+def status_string(code: int) -> str:
+    try:
+        return load_library().phmm_status_string(int(code)).decode()
+    except Exception:  # noqa: BLE001 - only used for messages
+        return "?"
+
+
+def _ptr(a: np.ndarray) -> int:
+    return a.ctypes.data if a.size else 0
+
+
+def _host_struct(b) -> tuple:
+    """(struct, keepalive) for a host batch (synth.Batch-like, numpy arrays)."""
+    arrs = dict(
+        read_bases=np.ascontiguousarray(b.read_bases, dtype=np.uint8),
+        base_quals=np.ascontiguousarray(b.base_quals, dtype=np.uint8),
+        ins_quals=np.ascontiguousarray(b.ins_quals, dtype=np.uint8),
+        del_quals=np.ascontiguousarray(b.del_quals, dtype=np.uint8),
+        gcp_quals=np.ascontiguousarray(b.gcp_quals, dtype=np.uint8),
+        read_offsets=np.ascontiguousarray(b.read_offsets, dtype=np.int64),
+        hap_bases=np.ascontiguousarray(b.hap_bases, dtype=np.uint8),
+        hap_offsets=np.ascontiguousarray(b.hap_offsets, dtype=np.int64),
+        pairs=np.ascontiguousarray(b.pairs, dtype=np.int32).reshape(-1),
+    )
+    s = _Batch()
+    for k, v in arrs.items():
+        setattr(s, k, _ptr(v))
+    s.n_reads = arrs["read_offsets"].size - 1
+    s.n_haps = arrs["hap_offsets"].size - 1
+    s.n_pairs = arrs["pairs"].size // 2
+    s.total_read_bases = int(arrs["read_offsets"][-1]) if arrs["read_offsets"].size else 0
+    s.total_hap_bases = int(arrs["hap_offsets"][-1]) if arrs["hap_offsets"].size else 0
+    return s, arrs
+
+
+@dataclass
+class DeviceBatch:
+    """A batch resident on one CUDA device (torch tensors; torch is plumbing)."""
+
+    read_bases: "object"
+    base_quals: "object"
+    ins_quals: "object"
+    del_quals: "object"
+    gcp_quals: "object"
+    read_offsets: "object"
+    hap_bases: "object"
+    hap_offsets: "object"
+    pairs: "object"  # int32 (n_pairs, 2)
+    total_read_bases: int
+    total_hap_bases: int
+
+    @property
+    def n_pairs(self) -> int:
+        return int(self.pairs.shape[0])
+
+    @staticmethod
+    def from_host(b, device="cuda", pinned: bool = False, non_blocking: bool = False) -> "DeviceBatch":
+        import torch
+
+        def t(a, dt):
+            x = torch.from_numpy(np.ascontiguousarray(a, dtype=dt))
+            if pinned:
+                x = x.pin_memory()
+            return x.to(device, non_blocking=non_blocking)
+
+        return DeviceBatch(read_bases=t(b.read_bases, np.uint8), base_quals=t(b.base_quals, np.uint8),
+                           ins_quals=t(b.ins_quals, np.uint8), del_quals=t(b.del_quals, np.uint8),
+                           gcp_quals=t(b.gcp_quals, np.uint8), read_offsets=t(b.read_offsets, np.int64),
+                           hap_bases=t(b.hap_bases, np.uint8), hap_offsets=t(b.hap_offsets, np.int64),
+                           pairs=t(np.asarray(b.pairs, dtype=np.int32).reshape(-1, 2), np.int32),
+                           total_read_bases=int(b.read_offsets[-1]), total_hap_bases=int(b.hap_offsets[-1]))
+
+    def struct(self) -> _Batch:
+        s = _Batch()
+        for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets",
+                  "hap_bases", "hap_offsets", "pairs"):
+            x = getattr(self, k)
+            setattr(s, k, x.data_ptr() if x.numel() else 0)
+        s.n_reads = int(self.read_offsets.numel()) - 1
+        s.n_haps = int(self.hap_offsets.numel()) - 1
+        s.n_pairs = int(self.pairs.shape[0])
+        s.total_read_bases = int(self.total_read_bases)
+        s.total_hap_bases = int(self.total_hap_bases)
+        return s
+
+
+class PairHMM:
+    """One libphmm context (``phmm_create``) bound to one CUDA device."""
+
+    def __init__(self, device: int = 0, precision: str = "fp32", stream=None, timing: bool = False,
+                 col_bucket: int = 0):
+        L = load_library()
+        cfg = _Config()
+        cfg.device = int(device)
+        cfg.precision = {"fp64": PREC_FP64, "fp32": PREC_FP32_RESCUE, "fp32_rescue": PREC_FP32_RESCUE}[precision]
+        cfg.cuda_stream = int(stream) if stream is not None else None
+        cfg.flags = FLAG_TIMING if timing else 0
+        cfg.col_bucket = int(col_bucket)
+        h = ctypes.c_void_p()
+        rc = L.phmm_create(ctypes.byref(h), ctypes.byref(cfg))
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_create")
+        self._h = h
+        self._L = L
+        self.device = int(device)
+        self.precision = precision
+
+    # ------------------------------------------------------------ host API
+    def compute_batch(self, batch, out: Optional[np.ndarray] = None, status: Optional[np.ndarray] = None,
+                      want_status: bool = True):
+        """``phmm_compute_batch``: host buffers in, host log10 likelihoods out.
+        ``out``/``status`` may be pre-allocated (e.g. pinned) numpy arrays."""
+        s, keep = _host_struct(batch)
+        n = int(s.n_pairs)
+        if out is None:
+            out = np.empty(n, dtype=np.float64)
+        if status is None and want_status:
+            status = np.empty(n, dtype=np.uint8)
+        rc = self._L.phmm_compute_batch(self._h, ctypes.byref(s), out.ctypes.data_as(_f64p),
+                                        status.ctypes.data_as(_u8p) if status is not None else None)
+        del keep
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_compute_batch")
+        return out, status
+
+    def compute_batch_raw(self, s: _Batch, out_ptr: int, status_ptr: int = 0) -> int:
+        """Direct ``phmm_compute_batch`` with prepared pointers (bench e2e leg)."""
+        return int(self._L.phmm_compute_batch(self._h, ctypes.byref(s), ctypes.cast(out_ptr, _f64p),
+                                              ctypes.cast(status_ptr, _u8p) if status_ptr else None))
+
+    # ------------------------------------------------------------ device API
+    def compute_batch_dev(self, db: DeviceBatch, out=None, status=None, want_status: bool = True):
+        """``phmm_compute_batch_dev``: torch CUDA tensors in and out."""
+        import torch
+
+        n = db.n_pairs
+        dev = db.pairs.device
+        if out is None:
+            out = torch.empty(n, dtype=torch.float64, device=dev)
+        if status is None and want_status:
+            status = torch.empty(n, dtype=torch.uint8, device=dev)
+        s = db.struct()
+        rc = self._L.phmm_compute_batch_dev(self._h, ctypes.byref(s), out.data_ptr() if n else None,
+                                            status.data_ptr() if (status is not None and n) else None)
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_compute_batch_dev")
+        return out, status
+
+    def stats(self) -> dict:
+        st = _Stats()
+        rc = self._L.phmm_get_stats(self._h, ctypes.byref(st))
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_get_stats")
+        return {k: getattr(st, k) for k, _ in _Stats._fields_}
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            self._L.phmm_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+
+def compute(batch, precision: str = "fp32", device: int = 0):
+    """One-shot convenience: log10 P(read|hap) for every pair of a host batch."""
+    with PairHMM(device=device, precision=precision) as h:
+        return h.compute_batch(batch)

@@ -1,0 +1,221 @@
+"""GPU parity: libphmm (through the C ABI) against the CPU oracle, element by
+element on the same seeded inputs (BASELINE.json north_star tolerances):
+  * FP64 path: |d log10| <= 1e-9 * max(|ref|, 1e-3)   (relative, R15)
+  * FP32 + rescue path: |d log10| <= 1e-3 absolute
+Every pair the oracle computes is compared; -inf must match -inf.
+"""
+import math
+
+import numpy as np
+import pytest
+
+from oracle import core as oracle
+from paper_conf_ipps_wangxc17_b200 import phmm, synth
+
+pytestmark = pytest.mark.gpu
+
+TOL_FP64_REL = 1e-9
+TOL_FP32_ABS = 1e-3
+
+
+@pytest.fixture(scope="module")
+def ctx32():
+    h = phmm.PairHMM(precision="fp32")
+    yield h
+    h.close()
+
+
+@pytest.fixture(scope="module")
+def ctx64():
+    h = phmm.PairHMM(precision="fp64")
+    yield h
+    h.close()
+
+
+def _check(got, ref, mode):
+    got = np.asarray(got, dtype=np.float64)
+    ref = np.asarray(ref, dtype=np.float64)
+    assert got.shape == ref.shape
+    ninf_ref = np.isneginf(ref)
+    assert np.array_equal(np.isneginf(got), ninf_ref), "−inf mismatch"
+    ok = ~ninf_ref
+    assert np.all(np.isfinite(got[ok]))
+    d = np.abs(got[ok] - ref[ok])
+    if mode == "fp64":
+        bound = TOL_FP64_REL * np.maximum(np.abs(ref[ok]), 1e-3)
+    else:
+        bound = np.full_like(d, TOL_FP32_ABS)
+    bad = np.nonzero(d > bound)[0]
+    assert bad.size == 0, f"{bad.size} pairs out of tolerance; worst {d.max():.3e} at ref {ref[ok][np.argmax(d)]}"
+    return float(d.max()) if d.size else 0.0
+
+
+def test_c1_fp64(ctx64):
+    b = synth.config_batch("C1")
+    got, st = ctx64.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp64")
+    assert np.all(st == 0)
+
+
+def test_c1_fp32(ctx32):
+    b = synth.config_batch("C1")
+    got, st = ctx32.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp32")
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_random_edge_pairs_fp64(ctx64, seed):
+    """Ragged tiny pairs: m, N in 1..60, Q0..60, 'N' bases, m > N."""
+    b = synth.random_pairs_batch(seed, 400, m_range=(1, 60), n_range=(1, 60))
+    got, _ = ctx64.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp64")
+
+
+@pytest.mark.parametrize("seed", [4, 5, 6])
+def test_random_edge_pairs_fp32(ctx32, seed):
+    b = synth.random_pairs_batch(seed, 400, m_range=(1, 60), n_range=(1, 60))
+    got, st = ctx32.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp32")
+    assert set(np.unique(st)) <= {0, 1, 2}
+
+
+def test_single_cell_pairs(ctx32, ctx64):
+    b = synth.random_pairs_batch(9, 64, m_range=(1, 1), n_range=(1, 1))
+    ref = oracle.batch_log10(b)
+    _check(ctx64.compute_batch(b)[0], ref, "fp64")
+    _check(ctx32.compute_batch(b)[0], ref, "fp32")
+
+
+def test_c2_reduced_all_pairs(ctx32):
+    """C2 shape (101 x 300, 16 reads x 8 haplotypes per region, 2 % decoys)."""
+    b = synth.config_batch("C2", n_regions=48)
+    got, st = ctx32.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp32")
+    stats = ctx32.stats()
+    assert stats["n_rescued"] == int(np.sum(st == 1) + np.sum(st == 2))
+    assert stats["cells"] == b.cells()
+
+
+def test_c3_reduced_mixed_lengths(ctx32):
+    b = synth.config_batch("C3", n_regions=6)
+    got, _ = ctx32.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp32")
+
+
+def test_c4_reduced_long_reads(ctx32):
+    """1000 x 1500: 8 passes of 128 rows per lane stream, ring carry of 1502 columns."""
+    b = synth.config_batch("C4", n_regions=1)
+    got, st = ctx32.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp32")
+
+
+def test_forced_rescue_is_fp64_exact(ctx32):
+    """Random reads against random haplotypes: log10 P ~ -150, every pair
+    underflows FP32 and must come back through the FP64 rescue at FP64
+    accuracy."""
+    rng = np.random.default_rng(3)
+    b = synth.random_pairs_batch(21, 60, m_range=(150, 200), n_range=(200, 260), qual_range=(30, 40),
+                                 indel_qual_range=(40, 45), gcp_range=(10, 10), n_frac=0.0)
+    got, st = ctx32.compute_batch(b)
+    ref = oracle.batch_log10(b)
+    assert np.all(ref < -64.2)
+    assert np.all(st == 1)
+    _check(got, ref, "fp64")
+
+
+def test_fp64_underflow_gives_minus_inf(ctx32):
+    """Q60 mismatches everywhere: P < 1e-700, below even the FP64 scale."""
+    m = 400
+    b = synth.Batch(read_bases=np.frombuffer(b"A" * m, np.uint8).copy(),
+                    base_quals=np.full(m, 60, np.uint8), ins_quals=np.full(m, 60, np.uint8),
+                    del_quals=np.full(m, 60, np.uint8), gcp_quals=np.full(m, 60, np.uint8),
+                    read_offsets=np.array([0, m], np.int64),
+                    hap_bases=np.frombuffer(b"C" * 500, np.uint8).copy(), hap_offsets=np.array([0, 500], np.int64),
+                    pairs=np.array([[0, 0]], np.int32))
+    got, st = ctx32.compute_batch(b)
+    assert oracle.batch_log10(b)[0] < -2000
+    assert np.isneginf(got[0]) and st[0] == 2
+
+
+def test_order_and_batch_invariance_bitwise(ctx32):
+    """Each pair's result is bitwise identical whatever the batch order or
+    composition (a pair's rows never mix with its neighbours': Z/R pad rows)."""
+    b = synth.config_batch("C3", n_regions=3)
+    base, _ = ctx32.compute_batch(b)
+    perm = np.random.default_rng(0).permutation(b.n_pairs)
+    got, _ = ctx32.compute_batch(b.subset(perm))
+    assert np.array_equal(got, base[perm])
+    half = perm[: b.n_pairs // 2]
+    got2, _ = ctx32.compute_batch(b.subset(half))
+    assert np.array_equal(got2, base[half])
+    mixed = synth.concat_batches([synth.random_pairs_batch(77, 50), b])
+    got3, _ = ctx32.compute_batch(mixed)
+    assert np.array_equal(got3[50:], base)
+
+
+def test_host_and_device_variants_agree(ctx32):
+    import torch
+
+    b = synth.config_batch("C2", n_regions=6)
+    host, hst = ctx32.compute_batch(b)
+    db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+    dev, dst = ctx32.compute_batch_dev(db)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev.cpu().numpy(), host)
+    assert np.array_equal(dst.cpu().numpy(), hst)
+
+
+def _sentinel(n):
+    return np.full(n, 12345.0), np.full(n, 77, np.uint8)
+
+
+@pytest.mark.parametrize("kind,code", [("base", -2), ("qual", -3), ("empty", -4), ("index", -5)])
+def test_input_errors_leave_outputs_untouched(ctx32, kind, code):
+    b = synth.random_pairs_batch(2, 20)
+    if kind == "base":
+        b.read_bases[3] = ord("x")
+    elif kind == "qual":
+        b.ins_quals[5] = 200
+    elif kind == "empty":
+        ro = b.read_offsets.copy()
+        ro[4] = ro[3]  # read 3 becomes empty; read 4 absorbs its bases
+        b.read_offsets = ro
+    elif kind == "index":
+        b.pairs = b.pairs.copy()
+        b.pairs[7, 1] = 20
+    out, st = _sentinel(b.n_pairs)
+    with pytest.raises(phmm.PhmmError) as ei:
+        ctx32.compute_batch(b, out=out, status=st)
+    assert ei.value.code == code
+    assert np.all(out == 12345.0) and np.all(st == 77)
+    # the context stays usable
+    good = synth.random_pairs_batch(2, 5)
+    got, _ = ctx32.compute_batch(good)
+    _check(got, oracle.batch_log10(good), "fp32")
+
+
+def test_empty_batch(ctx32):
+    b = synth.random_pairs_batch(2, 3)
+    b.pairs = np.zeros((0, 2), np.int32)
+    got, st = ctx32.compute_batch(b)
+    assert got.size == 0
+
+
+def test_full_c2_sampled(ctx32):
+    """BASELINE configs[1] at full size (2^20 pairs), the launch bench.py times:
+    a seeded sample of pairs plus every rescued pair against the oracle."""
+    import torch
+
+    b = synth.config_batch("C2")
+    assert b.n_pairs == 1 << 20
+    db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+    out, st = ctx32.compute_batch_dev(db)
+    torch.cuda.synchronize()
+    out = out.cpu().numpy()
+    st = st.cpu().numpy()
+    rng = np.random.default_rng(123)
+    sample = np.unique(np.concatenate([rng.choice(b.n_pairs, 3000, replace=False), np.nonzero(st != 0)[0][:3000]]))
+    ref = oracle.batch_log10(b, pair_idx=sample)
+    _check(out[sample], ref, "fp32")
+    # decoy reads (2 %) make some pairs need the rescue
+    assert 0 < np.sum(st == 1) < b.n_pairs // 10
