@@ -1,0 +1,360 @@
+#!/usr/bin/env python3
+"""bench.py -- batched GATK PairHMM forward on B200: GCUPS per GPU and whole job.
+
+Contract (see the task statement / DESIGN.md §7):
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload C2] [--impl reference]
+  N > 1: launched by torch.distributed.run, one rank per GPU (NCCL).
+
+A "step" is one pass of the whole hot path (validate, per-read tables,
+length binning, FP32 wavefront, finalize, FP64 rescue) over one batch of
+synthetic input: ``phmm_compute_batch_dev`` on
+device-resident inputs for ``value``; ``phmm_compute_batch`` from pinned host
+buffers (H2D + compute + D2H of every result) for ``e2e``. For N > 1 each rank
+processes its own shard of regions (weak scaling, regions addressed by
+(seed, region id)) and the step ends with the NCCL all-gather of the results
+(the path's one exchange step).
+
+metric = GCUPS = sum over pairs of m*N / seconds / 1e9 (PAPER.md L22@1416:
+the three M/I/D updates of one cell count as one cell update).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+# FP32 pipe roofline: 8 FP32-pipe ops per cell (3 FFMA + 4 FMUL + 1 FADD),
+# 128 FP32 lanes per SM per clock.
+FP32_OPS_PER_CELL = 8
+FP32_LANES_PER_SM = 128
+FP64_LANES_PER_SM = 64
+SM_MAX_MHZ_FALLBACK = 1965.0
+
+WORKLOADS = {
+    "C2": "C2: 1M pairs (8192 regions x 16 reads x 8 haplotypes), 101 bp reads x 300 bp haplotypes, "
+          "2% decoy reads, FP32 + FP64 underflow rescue",
+    "C3": "C3: HaplotypeCaller-shaped regions, 250 bp reads x 4-8 haplotypes of 250-500 bp",
+    "C4": "C4: long-read stress, 1000 bp reads x 1500 bp haplotypes",
+    "C5": "C5-shaped shard: mixed 100-250 bp reads, N ~ U{m..2m}",
+}
+DEFAULT_REGIONS = {"C2": 8192, "C3": 4096, "C4": 256, "C5": 8192}
+
+
+def _measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except Exception:  # noqa: BLE001
+        return {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.path = None
+
+    def start(self):
+        fd, self.path = tempfile.mkstemp(prefix="clk_", suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:  # noqa: BLE001
+            self.proc = None
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:  # noqa: BLE001
+            self.proc.kill()
+        sm, smax, power, reasons = [], [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        with open(self.path) as f:
+            for line in f:
+                parts = [p.strip() for p in line.split(",")]
+                if len(parts) < 9:
+                    continue
+                try:
+                    sm.append(float(parts[1]))
+                    smax.append(float(parts[2]))
+                    power.append(float(parts[3]))
+                except ValueError:
+                    continue
+                for nm, v in zip(names, parts[5:9]):
+                    if v.lower().startswith("active"):
+                        reasons.add(nm)
+        os.unlink(self.path)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(smax), "power_w_max": max(power),
+                "samples": len(sm), "reasons": sorted(reasons)}
+
+
+def _dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def run_reference(args, ws, rank):
+    """--impl reference: the oracle (plain C, fp64, OpenMP) as it stands on the
+    host cores, on a bounded sample of the same workload each step."""
+    if rank != 0:
+        return 0
+    from oracle import core as oracle
+    from paper_conf_ipps_wangxc17_b200 import synth
+
+    n_regions = max(1, int(args.ref_regions))
+    cores = oracle.max_threads()
+    batches = [synth.config_batch(args.workload, n_regions=n_regions, region_start=i * n_regions)
+               for i in range(args.warmup + args.steps)]
+    for b in batches[:args.warmup]:
+        oracle.batch_log10(b)
+    t_total, cells = 0.0, 0
+    for b in batches[args.warmup:]:
+        t0 = time.perf_counter()
+        oracle.batch_log10(b)
+        t_total += time.perf_counter() - t0
+        cells += b.cells()
+    gcups = cells / t_total / 1e9
+    sample = f"{n_regions} regions ({batches[-1].n_pairs} pairs, {batches[-1].cells()} cells) of {args.workload} per step"
+    line = {"metric": "PairHMM GCUPS", "value": gcups, "unit": "GCUPS", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * t_total / max(1, args.steps), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "impl": "reference",
+            "config": {"workload": WORKLOADS[args.workload], "sample": sample},
+            "cpu_baseline": {"value": gcups, "unit": "GCUPS", "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": gcups, "unit": "GCUPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def cpu_baseline(args, batch):
+    """The oracle timed on this box's host cores on a bounded sample (~10-30 s)."""
+    from oracle import core as oracle
+
+    cores = oracle.max_threads()
+    rng = np.random.default_rng(7)
+    cells_per_pair = batch.pair_cells()
+    # size the sample: probe, then aim for ~args.cpu_seconds
+    probe = rng.choice(batch.n_pairs, size=min(batch.n_pairs, 64 * cores), replace=False)
+    t0 = time.perf_counter()
+    oracle.batch_log10(batch, pair_idx=probe)
+    dt = time.perf_counter() - t0
+    rate = cells_per_pair[probe].sum() / max(dt, 1e-6)
+    n_target = int(min(batch.n_pairs, max(len(probe), args.cpu_seconds * rate / cells_per_pair.mean())))
+    sample = np.sort(rng.choice(batch.n_pairs, size=n_target, replace=False))
+    t0 = time.perf_counter()
+    ref = oracle.batch_log10(batch, pair_idx=sample)
+    dt = time.perf_counter() - t0
+    cells = int(cells_per_pair[sample].sum())
+    return {"value": cells / dt / 1e9, "unit": "GCUPS", "cores": cores, "kind": "oracle",
+            "sample": f"{n_target} seeded-random pairs of the timed batch ({cells} cells, {dt:.1f} s)"}, sample, ref
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--workload", default="C2", choices=sorted(WORKLOADS))
+    ap.add_argument("--regions", type=int, default=None, help="regions per rank (default: the config's)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--ref-regions", type=int, default=16, help="regions per step for --impl reference")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--profile-steps", action="store_true", help="short run for ncu (no clocks/cpu)")
+    args = ap.parse_args()
+
+    ws, rank, local = _dist()
+    if args.impl == "reference":
+        return run_reference(args, ws, rank)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_wangxc17_b200 import phmm, synth
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    n_regions = args.regions or DEFAULT_REGIONS[args.workload]
+    batch = synth.config_batch(args.workload, n_regions=n_regions, region_start=rank * n_regions)
+    cells = batch.cells()
+    n_pairs = batch.n_pairs
+
+    stream = torch.cuda.Stream(device=dev)
+    ctx = phmm.PairHMM(device=local, precision="fp32", stream=stream.cuda_stream, timing=True)
+    with torch.cuda.stream(stream):
+        db = phmm.DeviceBatch.from_host(batch, device=dev)
+        out = torch.empty(n_pairs, dtype=torch.float64, device=dev)
+        status = torch.empty(n_pairs, dtype=torch.uint8, device=dev)
+        gathered = torch.empty(n_pairs * ws, dtype=torch.float64, device=dev) if ws > 1 else None
+        flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    torch.cuda.synchronize()
+
+    def step():
+        ctx.compute_batch_dev(db, out=out, status=status)
+        if ws > 1:
+            with torch.cuda.stream(stream):
+                dist.all_gather_into_tensor(gathered, out)
+
+    for _ in range(max(args.warmup, 0)):
+        step()
+    torch.cuda.synchronize()
+
+    clk = ClockSampler(local)
+    if not args.profile_steps:
+        clk.start()
+        time.sleep(0.3)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    wf_ms, launches, rescued = [], 0, 0
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(i & 0xff)  # L2 flush between timed steps (not timed)
+            ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+        st = ctx.stats()
+        wf_ms.append(st["ms_wavefront"])
+        launches += st["kernel_launches"]
+        rescued = st["n_rescued"]
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    clocks = clk.stop() if not args.profile_steps else {}
+    t_rank = sum(step_ms) / 1e3
+    if ws > 1:
+        tt = torch.tensor([t_rank], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_max = float(tt.item())
+        cc = torch.tensor([float(cells)], dtype=torch.float64, device=dev)
+        dist.all_reduce(cc, op=dist.ReduceOp.SUM)
+        cells_all = float(cc.item())
+    else:
+        t_max, cells_all = t_rank, float(cells)
+    value = cells_all * args.steps / t_max / 1e9
+
+    # ---- e2e: host API from pinned host buffers (H2D + compute + D2H each step)
+    e2e = None
+    if not args.no_e2e and not args.profile_steps:
+        pinned = {}
+        for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets", "hap_bases",
+                  "hap_offsets", "pairs"):
+            a = np.ascontiguousarray(getattr(batch, k))
+            t = torch.from_numpy(a).pin_memory()
+            pinned[k] = t
+        s = phmm._Batch()
+        for k, t in pinned.items():
+            setattr(s, k, t.data_ptr())
+        s.n_reads = batch.n_reads
+        s.n_haps = batch.n_haps
+        s.n_pairs = n_pairs
+        s.total_read_bases = int(batch.read_offsets[-1])
+        s.total_hap_bases = int(batch.hap_offsets[-1])
+        hout = torch.empty(n_pairs, dtype=torch.float64).pin_memory()
+        hst = torch.empty(n_pairs, dtype=torch.uint8).pin_memory()
+        h2d = int(sum(t.numel() * t.element_size() for t in pinned.values()))
+        d2h = n_pairs * (8 + 1)
+        for _ in range(max(1, args.warmup)):
+            rc = ctx.compute_batch_raw(s, hout.data_ptr(), hst.data_ptr())
+            assert rc == 0, rc
+        if ws > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e_ms = []
+        for i in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.fill_(i & 0xff)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            rc = ctx.compute_batch_raw(s, hout.data_ptr(), hst.data_ptr())
+            if ws > 1:
+                hg = torch.from_numpy(hout.numpy()).to(dev, non_blocking=False)
+                dist.all_gather_into_tensor(gathered, hg)
+                torch.cuda.synchronize()
+            e_ms.append((time.perf_counter() - t0) * 1e3)
+            assert rc == 0, rc
+        t_e = sum(e_ms) / 1e3
+        if ws > 1:
+            tt = torch.tensor([t_e], dtype=torch.float64, device=dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            t_e = float(tt.item())
+        e2e = {"value": cells_all * args.steps / t_e / 1e9, "unit": "GCUPS", "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "ms_per_step": 1e3 * t_e / args.steps,
+               "timing": "host wall clock around phmm_compute_batch (synchronous C-ABI call)"}
+
+    # ---- roofline of the dominant kernel (the FP32 wavefront), live CUDA events
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    peaks = _measured_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", SM_MAX_MHZ_FALLBACK))
+    peak_gcups = nsm * FP32_LANES_PER_SM * sm_max * 1e6 / FP32_OPS_PER_CELL / 1e9
+    wf = float(np.mean(wf_ms)) if wf_ms else float("nan")
+    achieved = cells / (wf / 1e3) / 1e9 if wf > 0 else None
+    sm_run = clocks.get("sm_mhz") if clocks else None
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak_gcups, "unit": "GCUPS",
+                "frac": (achieved / peak_gcups) if achieved else None, "traffic": None,
+                "kernel": "k_wavefront<float,8>",
+                "peak_basis": f"{nsm} SM x {FP32_LANES_PER_SM} FP32 lanes x {sm_max:.0f} MHz (MEASURED_PEAKS sm_max_mhz)"
+                              f" / {FP32_OPS_PER_CELL} FP32-pipe ops per cell (3 FFMA + 4 FMUL + 1 FADD)",
+                "frac_at_run_clock": (achieved / (peak_gcups * sm_run / sm_max)) if (achieved and sm_run) else None,
+                "wavefront_ms": wf, "wavefront_share_of_step": wf / (sum(step_ms) / len(step_ms))}
+
+    cpu = None
+    if rank == 0 and ws == 1 and not args.no_cpu_baseline and not args.profile_steps:
+        cpu, sample_idx, ref = cpu_baseline(args, batch)
+        got = out.cpu().numpy()[sample_idx]
+        fin = np.isfinite(ref)
+        cpu["parity_max_abs_log10"] = float(np.max(np.abs(got[fin] - ref[fin]))) if fin.any() else 0.0
+
+    if rank == 0:
+        line = {"metric": "PairHMM GCUPS", "value": value, "unit": "GCUPS", "n_gpus": ws, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": 1e3 * t_max / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": WORKLOADS[args.workload], "regions_per_rank": n_regions,
+                           "pairs_per_rank": n_pairs, "cells_per_rank": cells,
+                           "padded_cells_per_rank": ctx.stats()["padded_cells"],
+                           "rescued_pairs_per_rank": rescued,
+                           "l2": "flushed between timed steps (256 MiB write, untimed)",
+                           "parallelism": f"dp{ws} (independent pair shards, NCCL all-gather of results)"},
+                "gpu_launches": launches,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks}
+        print(json.dumps(line), flush=True)
+    ctx.close()
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -10,13 +10,18 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libphmm.so")
-SOURCES = [os.path.join(CSRC, "phmm_lib.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, "phmm_device.cuh"), os.path.join(ROOT, "include", "phmm.h")]
+SOURCES = [os.path.join(CSRC, "phmm_lib.cu"), os.path.join(CSRC, "wf32.cu")]
+# per-source extra flags: the FP32 wavefront kernel is built with ptxas -O1
+# (ptxas -O2/-O3 miscompiles it)
+SOURCE_FLAGS = {"wf32.cu": ["-Xptxas", "-O1"]}
+def _deps():
+    return SOURCES + [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith((".cuh", ".h"))] + \
+        [os.path.join(ROOT, "include", "phmm.h"), os.path.abspath(__file__)]
 
 NVCC_FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
     "-O3", "-lineinfo", "-std=c++17",
-    "-Xcompiler", "-fPIC", "-shared",
+    "-Xcompiler", "-fPIC",
     "-Xptxas", "-v",
 ]
 
@@ -32,24 +37,39 @@ def needs_build() -> bool:
     if not os.path.exists(LIB):
         return True
     t = os.path.getmtime(LIB)
-    return any(os.path.getmtime(p) > t for p in DEPS)
+    return any(os.path.getmtime(p) > t for p in _deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
+    """Build libphmm.so (or a variant at ``out`` with extra -D ``defines``, for A/B runs)."""
+    target = out or LIB
+    if not force and out is None and not needs_build():
         return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [nvcc()] + NVCC_FLAGS + ["-I", os.path.join(ROOT, "include"), "-o", tmp] + SOURCES
-    res = subprocess.run(cmd, capture_output=True, text=True)
+    tmp = target + f".tmp{os.getpid()}"
+    objs, log = [], []
+    for src in SOURCES:
+        obj = f"{tmp}.{os.path.basename(src)}.o"
+        cmd = ([nvcc()] + NVCC_FLAGS + SOURCE_FLAGS.get(os.path.basename(src), []) + [f"-D{d}" for d in defines]
+               + ["-I", os.path.join(ROOT, "include"), "-c", "-o", obj, src])
+        res = subprocess.run(cmd, capture_output=True, text=True)
+        if res.returncode != 0:
+            sys.stderr.write(res.stdout + res.stderr)
+            raise RuntimeError(f"nvcc failed building {os.path.basename(src)}")
+        log.append(res.stderr)
+        objs.append(obj)
+    res = subprocess.run([nvcc(), "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", tmp] + objs,
+                         capture_output=True, text=True)
+    for o in objs:
+        os.unlink(o)
     if res.returncode != 0:
         sys.stderr.write(res.stdout + res.stderr)
-        raise RuntimeError("nvcc failed building libphmm.so")
+        raise RuntimeError("nvcc failed linking libphmm.so")
     if verbose:
-        sys.stderr.write(res.stderr)
-    with open(os.path.join(PKG, "ptxas_info.txt"), "w") as f:
-        f.write(res.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+        sys.stderr.write("".join(log))
+    with open(target + ".ptxas.txt" if out else os.path.join(PKG, "ptxas_info.txt"), "w") as f:
+        f.write("".join(log))
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

@@ -1,0 +1,117 @@
+// phmm_common.cuh -- constants, descriptors and device helpers shared by the libphmm kernels (sm_100a).
+//
+// PRODUCT PATH. Shares no code with oracle/ (which is test infrastructure).
+//
+// What is computed: the PairHMM forward recurrence, Eq. 6 of PAPER.md
+// (L18@541, §III-B), for every (read, haplotype) pair, terminated by the sum
+// of the last row of M and I (L20@2262, §IV-C.1), with the GATK 3.6 Phred
+// mapping (L22@4113) -- see include/phmm.h and DESIGN.md §2.
+//
+// How (DESIGN.md §4 -- differs from the paper's one-warp-per-pair PH2):
+//  * "tall stream" layout: every pair is laid out as a whole number of K-row
+//    BLOCKS: [Z..Z][R][read rows 1..m][S1][S2] where the pad rows are plain
+//    rows of the same recurrence with special coefficients:
+//      Z  (zero)   : every coefficient 0            -> M = I = D = 0
+//      R  (reset)  : prior 0, delta=eps=zeta=0, mu=1, boundary D(.,0)=s/N
+//                    -> M = I = 0, D = s/N on every column: the virtual row 0
+//                       of Eq. 6 (D(0,j) = 1/N, scaled by s)
+//      S1 (sum)    : prior 0, delta=eps=1, zeta=0   -> I(j) = M(m,j) + I(m,j)
+//      S2 (scan)   : prior 1, alpha=0, beta=1, zeta=mu=1
+//                    -> M(j) = I_S1(j-1), D(j) = sum_{j'<j} M(j'),
+//                       so D_S2(N+2) = sum_{j=1..N} M(m,j) + I(m,j)
+//    The termination sum of L20@2262 therefore falls out of the recurrence
+//    itself, read as D of the S2 row at column N+2 (0-based c = N+1), and
+//    consecutive pairs can be stacked into one tall DP: a Z/R row ignores
+//    whatever (finite) values are above it. One warp streams through a long
+//    sequence of blocks of equal column count (a length bin) without
+//    draining between pairs.
+//  * lane l of a warp owns one K-row block per "pass" (blocks l, l+32, ...),
+//    processes one column per step (a K-row column tile), lags lane l-1 by
+//    one step, receives the (M,I,D) of the row above by __shfl_sync
+//    (the paper's Design B, Fig. 6b / Listing 2b, L20@44), and lane 31 hands
+//    its last row to lane 0 of the next pass through a per-warp shared-memory
+//    ring indexed by column (the stripe carry).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace phmm {
+
+// ---------------------------------------------------------------- constants
+constexpr int kMinCols = 40;        // ring delay needs ncols > 32
+constexpr int kMaxHapLen = 4094;    // FP32/FP64 ring in shared memory
+constexpr int kMaxBins = 4200;      // ncols / bucket <= kMaxBins
+
+// error flag bits (device) -> phmm_status
+enum : uint32_t {
+  ERR_BASE = 1u, ERR_QUAL = 2u, ERR_EMPTY = 4u, ERR_INDEX = 8u, ERR_ARG = 16u
+};
+
+// base -> one-hot code; N matches everything; 0xff = invalid
+__device__ __forceinline__ uint32_t base_code(uint8_t b) {
+  switch (b) {
+    case 'A': return 1u;
+    case 'C': return 2u;
+    case 'G': return 4u;
+    case 'T': return 8u;
+    case 'N': return 15u;
+    default: return 0xffu;
+  }
+}
+
+template <typename T> struct Prec;
+template <> struct Prec<float> { static constexpr int kScaleExp = 120; };
+template <> struct Prec<double> { static constexpr int kScaleExp = 1020; };
+
+// mask bits of a table row
+constexpr uint32_t MASK_BASE = 15u;
+constexpr uint32_t MASK_D0 = 16u;          // row boundary D(i,0) = s/N (the R row)
+constexpr uint32_t MASK_ABOVE_IS_R = 32u;  // (row 0 of a block) the row above is an R row
+
+// Per-block descriptor in the bin-sorted block sequence (16 bytes).
+struct BlkDesc {
+  uint32_t tab_blk;   // block index in the coefficient table
+  uint32_t hap_off;   // offset of the haplotype in the code array
+  int32_t out_idx;    // output slot of the pair (valid on its last block)
+  uint16_t n;         // haplotype length N
+  uint16_t flags;     // bit0: last block of its pair, bit1: first block of its pair
+};
+static_assert(sizeof(BlkDesc) == 16, "BlkDesc must be 16 bytes");
+constexpr uint16_t BLK_LAST = 1, BLK_FIRST = 2;
+
+// bytes of one table block: 8 coefficient fields x K values of T, then K masks
+template <typename T, int K>
+struct alignas(16) TabBlock {
+  T coef[8][K];  // alpha, beta, delta, eps, zeta, mu, pm, px
+  uint32_t mask[K];
+};
+
+template <typename T>
+struct alignas(16) RingEnt {
+  T m, i, d, pad;
+};
+
+__host__ __device__ constexpr int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
+
+__host__ __device__ inline int ncols_of(int n, int bucket) {
+  const int c = ((n + 2 + bucket - 1) / bucket) * bucket;
+  const int lo = ((kMinCols + bucket - 1) / bucket) * bucket;
+  return c < lo ? lo : c;
+}
+__host__ __device__ inline int bin_of_ncols(int ncols, int bucket) { return ncols / bucket; }
+template <int K>
+__host__ __device__ inline int nblocks_of(int m) { return (m + 3 + K - 1) / K; }
+
+// Phred -> error probability, 10^(-q/10), in the table's precision.
+template <typename T>
+__device__ __forceinline__ T qual_err(uint32_t q);
+template <>
+__device__ __forceinline__ float qual_err<float>(uint32_t q) {
+  return (float)exp10(-(double)q / 10.0);  // computed in double, rounded once
+}
+template <>
+__device__ __forceinline__ double qual_err<double>(uint32_t q) {
+  return exp10(-(double)q / 10.0);
+}
+
+}  // namespace phmm

@@ -17,6 +17,7 @@
 
 #include "../../include/phmm.h"
 #include "phmm_device.cuh"
+#include "f32_prep.cuh"
 
 using namespace phmm;
 
@@ -27,7 +28,7 @@ enum BufId {
   B_HCODES, B_SCAL,                                                       // codes, scalars
   B_PAIR_BIN, B_PAIR_NB, B_BINS, B_ITEM_NB, B_ITEM_OFF, B_SCAN_TMP,
   B_TAB, B_BLK, B_OUT32, B_OUT64, B_RLIST, B_ITEM_READ, B_PAIR_ITEM,
-  B_OUT_LOG10, B_OUT_STATUS, B_COUNT
+  B_OUT_LOG10, B_OUT_STATUS, B_HNC, B_HC_OFF, B_HCODES32, B_TAB32, B_COUNT
 };
 
 struct Buf {
@@ -208,7 +209,7 @@ phmm_status run_validate(phmm_ctx* c, const DevBatch& d, uint8_t** hcodes_out) {
 //                    output slot = position in the list
 template <typename T, int K>
 phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_t n, PassInfo* pi,
-                         int64_t* total_tab_out) {
+                         int64_t* total_tab_out, int64_t* total_hcodes_out = nullptr) {
   cudaStream_t s = c->stream;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
@@ -250,11 +251,28 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, item_nb, item_off, (int64_t)(n_items + 1), s));
   ++c->launches;
 
+  // FP32 kernel: per-haplotype padded code arrays (ncols codes each)
+  int64_t* hc_off = nullptr;
+  if (total_hcodes_out) {
+    int64_t* hnc;
+    ST_TRY(ws(c, B_HNC, (size_t)d.n_haps + 1, &hnc));
+    ST_TRY(ws(c, B_HC_OFF, (size_t)d.n_haps + 1, &hc_off));
+    k_hap_ncols<<<grid_for(c, d.n_haps), kThreads, 0, s>>>(d.hoff, d.n_haps, c->bucket, hnc);
+    LAUNCHED(c);
+    size_t tb2 = 0;
+    CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, hnc, hc_off, (int64_t)(d.n_haps + 1), s));
+    unsigned char* tmp2;
+    ST_TRY(ws(c, B_SCAN_TMP, std::max(tb2, tmp_bytes), &tmp2));
+    CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp2, tb2, hnc, hc_off, (int64_t)(d.n_haps + 1), s));
+    ++c->launches;
+  }
   // one small D2H: sizes + error flag
   CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
-  int64_t total_tab = 0;
+  int64_t total_tab = 0, total_hc = 0;
   CUDA_TRY(cudaMemcpyAsync(&total_tab, item_off + n_items, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  if (hc_off) CUDA_TRY(cudaMemcpyAsync(&total_hc, hc_off + d.n_haps, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaStreamSynchronize(s));
+  if (total_hcodes_out) *total_hcodes_out = total_hc;
   if (c->host_scal->err) return map_err(c->host_scal->err);
   pi->cells = c->host_scal->cells;
   pi->padded_cells = c->host_scal->padded_cells;
@@ -339,7 +357,76 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const uint8_t* hcodes, cons
   return PHMM_OK;
 }
 
-constexpr int K32 = 8;  // rows per lane, FP32 pass
+// FP32 pass over all pairs with k_wavefront_f32 (after pass_prepare<float, F32_K>).
+phmm_status pass_run_f32(phmm_ctx* c, const DevBatch& d, const PassInfo& pi, int64_t total_tab, int64_t total_hc,
+                         float* out) {
+  cudaStream_t s = c->stream;
+  Scalars* scal;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  const int nb1 = kMaxBins + 2;
+  unsigned long long* bins;
+  ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
+  unsigned long long *bin_blocks = bins, *bin_cursor = bins + 2 * nb1, *bin_start = bins + 3 * nb1,
+                     *item_start = bins + 4 * nb1;
+  int32_t *pair_bin, *pair_nb;
+  ST_TRY(ws(c, B_PAIR_BIN, (size_t)d.n_pairs, &pair_bin));
+  ST_TRY(ws(c, B_PAIR_NB, (size_t)d.n_pairs, &pair_nb));
+  int64_t *item_off, *hc_off;
+  ST_TRY(ws(c, B_ITEM_OFF, (size_t)d.n_reads + 1, &item_off));
+  ST_TRY(ws(c, B_HC_OFF, (size_t)d.n_haps + 1, &hc_off));
+  const int p_max = std::max(pi.max_ncols + F32_G, F32_MIN_P);
+  const int64_t pad_len = p_max + 256;
+  F32Block* tab;
+  BlkDesc* blk;
+  uint8_t* hc;
+  ST_TRY(ws(c, B_TAB32, (size_t)total_tab, &tab));
+  ST_TRY(ws(c, B_BLK, (size_t)pi.total_blocks, &blk));
+  ST_TRY(ws(c, B_HCODES32, (size_t)(total_hc + pad_len), &hc));
+  CUDA_TRY(cudaMemsetAsync(hc + total_hc, F32_PAD, (size_t)pad_len, s));
+  if (total_tab > 0) {
+    k_build_table_f32<<<grid_for(c, total_tab * F32_K), kThreads, 0, s>>>(
+        d.n_reads, item_off, item_off + d.n_reads, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
+    LAUNCHED(c);
+  }
+  k_hap_codes_f32<<<grid_for(c, d.n_haps * 32), kThreads, 0, s>>>(d.hap, d.hoff, d.n_haps, hc_off, c->bucket, hc);
+  LAUNCHED(c);
+
+  const int ring_len = p_max + 4;
+  const size_t smem = (size_t)F32_WARPS * (2 * F32_NCODE * 32 + ring_len) * sizeof(float4);
+  int bps = 0;
+  CUDA_TRY(wf32_occupancy(smem, &bps));
+  if (bps < 1) return PHMM_E_INVALID_ARG;
+  const int64_t nwarps = (int64_t)c->nsm * bps * F32_WARPS;
+  int64_t chunk = (int64_t)(pi.total_blocks / (unsigned long long)(nwarps * 4));
+  if (chunk < 512) chunk = 512;
+  if (chunk > 65536) chunk = 65536;
+  const int nbins = kMaxBins + 1;
+  k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, chunk, bin_start, item_start);
+  LAUNCHED(c);
+  k_alloc_blocks_f32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(d.pairs, d.n_pairs, pair_bin, pair_nb, bin_start,
+                                                                 bin_cursor, d.roff, d.hoff, hc_off, item_off, blk);
+  LAUNCHED(c);
+  F32Args A;
+  A.blk = blk;
+  A.tab = tab;
+  A.hcodes = hc;
+  A.pad_idx = (uint32_t)(total_hc + 16);
+  A.bin_start = bin_start;
+  A.item_start = item_start;
+  A.nbins = nbins;
+  A.bucket = c->bucket;
+  A.chunk_blocks = chunk;
+  A.item_counter = &scal->item_counter;
+  A.out = out;
+  A.ring_len = ring_len;
+  CUDA_TRY(cudaMemsetAsync(&scal->item_counter, 0, sizeof(unsigned int), s));
+  ev_record(c, EV_WF0);
+  CUDA_TRY(wf32_launch((unsigned)(c->nsm * bps), smem, s, A));
+  ++c->launches;
+  ev_record(c, EV_WF1);
+  return PHMM_OK;
+}
+
 constexpr int K64 = 4;  // rows per lane, FP64 pass
 
 // The whole path on device-resident inputs. Writes dev_out (+ dev_status).
@@ -371,11 +458,12 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     CUDA_TRY(cudaStreamSynchronize(s));
     c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
   } else {
-    ST_TRY((pass_prepare<float, K32>(c, d, nullptr, d.n_pairs, &pi, &total_tab)));
+    int64_t total_hc = 0;
+    ST_TRY((pass_prepare<float, F32_K>(c, d, nullptr, d.n_pairs, &pi, &total_tab, &total_hc)));
     float* out32;
     ST_TRY(ws(c, B_OUT32, (size_t)d.n_pairs, &out32));
     ev_record(c, EV_PREP);
-    ST_TRY((pass_run<float, K32>(c, d, hcodes, nullptr, d.n_pairs, pi, total_tab, out32, nullptr)));
+    ST_TRY(pass_run_f32(c, d, pi, total_tab, total_hc, out32));
     int32_t* rlist;
     ST_TRY(ws(c, B_RLIST, (size_t)d.n_pairs, &rlist));
     CUDA_TRY(cudaMemsetAsync(&scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
@@ -455,6 +543,8 @@ void finish_stats(phmm_ctx* c) {
 extern "C" {
 
 int phmm_abi_version(void) { return PHMM_ABI_VERSION; }
+
+
 
 const char* phmm_status_string(phmm_status s) {
   switch (s) {

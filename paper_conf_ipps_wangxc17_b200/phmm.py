@@ -20,7 +20,7 @@ from typing import Optional
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libphmm.so")
+LIB_PATH = os.environ.get("PHMM_LIB") or os.path.join(_PKG, "libphmm.so")
 
 PHMM_OK = 0
 STATUS_NAMES = {
