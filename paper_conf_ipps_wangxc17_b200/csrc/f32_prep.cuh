@@ -7,15 +7,17 @@ namespace phmm {
 
 // ---------------------------------------------------------------- prep for the FP32 kernel
 
-// Code slot of one haplotype: F32_HC_FRONT PAD codes, then columns
-// c < N: base code 0..4; c == N: 4 ('N', matches all); c > N: PAD, up to the
-// last column a lane can reach before its next switch event (its pass P).
-// BlkDesc.hap_off points at column 0.
-__host__ __device__ inline int f32_hc_slot(int n, int bucket) {
-  const int nc = ncols_of(n, bucket);
-  const int p = (nc + F32_G > F32_MIN_P) ? nc + F32_G : F32_MIN_P;
-  return (int)F32_HC_FRONT + p + 8;
+// Code region of one haplotype: 4 copies of f32_hc_copy_len(ncols) bytes; in copy k
+// column c sits at byte F32_HC_FRONT + k + c (so a lane picks the copy that makes its
+// code words 4-aligned). Byte = code * 2 with code A=0 C=1 G=2 T=3 N=4 PAD=5:
+// columns c < N carry the haplotype, c == N carries 'N' (matches every row), every
+// other byte is PAD (prior 0). BlkDesc.hap_off = region start + F32_HC_FRONT.
+// (Each byte holds code * 2: the kernel moves it into bits 8..15 -> code * 512 B,
+// the stride of a code's row in a lane's shared-memory prior table.)
+__host__ __device__ inline int64_t f32_hc_region(int n, int bucket) {
+  return 4 * (int64_t)f32_hc_copy_len(ncols_of(n, bucket));
 }
+
 __global__ void k_hap_codes_f32(const uint8_t* __restrict__ hap, const int64_t* __restrict__ hoff, int64_t n_haps,
                                 const int64_t* __restrict__ hc_off, int bucket, uint8_t* __restrict__ codes) {
   const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -25,9 +27,11 @@ __global__ void k_hap_codes_f32(const uint8_t* __restrict__ hap, const int64_t* 
     const int64_t h0 = hoff[h];
     const int n = (int)(hoff[h + 1] - h0);
     if (n < 1 || n > kMaxHapLen) continue;
-    const int slot = f32_hc_slot(n, bucket);
+    const int len = f32_hc_copy_len(ncols_of(n, bucket));
     uint8_t* dst = codes + hc_off[h];
-    for (int c = lane - (int)F32_HC_FRONT; c < slot - (int)F32_HC_FRONT; c += 32) {
+    for (int i = lane; i < 4 * len; i += 32) {
+      const int k = i / len;
+      const int c = (i % len) - (int)F32_HC_FRONT - k;  // column of this byte in copy k
       uint8_t v = F32_PAD;
       if (c >= 0 && c < n) {
         switch (hap[h0 + c]) {
@@ -40,7 +44,7 @@ __global__ void k_hap_codes_f32(const uint8_t* __restrict__ hap, const int64_t* 
       } else if (c == n) {
         v = 4;
       }
-      dst[c + F32_HC_FRONT] = v;
+      dst[i] = (uint8_t)(v * 2);
     }
   }
 }
@@ -48,7 +52,7 @@ __global__ void k_hap_codes_f32(const uint8_t* __restrict__ hap, const int64_t* 
 __global__ void k_hap_ncols(const int64_t* __restrict__ hoff, int64_t n_haps, int bucket, int64_t* __restrict__ nc) {
   for (int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; h < n_haps; h += (int64_t)gridDim.x * blockDim.x) {
     const int64_t n = hoff[h + 1] - hoff[h];
-    nc[h] = (n >= 1 && n <= kMaxHapLen) ? f32_hc_slot((int)n, bucket) : 0;
+    nc[h] = (n >= 1 && n <= kMaxHapLen) ? f32_hc_region((int)n, bucket) : 0;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) nc[n_haps] = 0;
 }
@@ -112,22 +116,39 @@ __global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ i
   }
 }
 
-// block descriptors for the FP32 pass (R row index in the flags, padded haplotype code offsets)
-__global__ void k_alloc_blocks_f32(const int32_t* __restrict__ pairs, int64_t n_pairs,
-                                   const int32_t* __restrict__ pair_bin, const int32_t* __restrict__ pair_nb,
-                                   const unsigned long long* __restrict__ bin_start,
-                                   unsigned long long* __restrict__ bin_cursor, const int64_t* __restrict__ roff,
+// Stable length binning: pairs are radix-sorted by bin (stable, so
+// read-major input order survives inside a bin and the pairs of one read stay
+// adjacent -- its coefficient table is reused from L2), then each sorted pair gets a
+// contiguous block range from an exclusive scan. Deterministic, no atomics.
+__global__ void k_iota_keys(const int32_t* __restrict__ pair_bin, int64_t n, uint32_t* __restrict__ keys,
+                            int32_t* __restrict__ vals) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    keys[i] = (uint32_t)pair_bin[i];
+    vals[i] = (int32_t)i;
+  }
+}
+
+__global__ void k_sorted_nb(const int32_t* __restrict__ sorted_pairs, const int32_t* __restrict__ pair_nb, int64_t n,
+                            int64_t* __restrict__ nb_sorted) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    nb_sorted[i] = pair_nb[sorted_pairs[i]];
+  if (blockIdx.x == 0 && threadIdx.x == 0) nb_sorted[n] = 0;
+}
+
+// block descriptors for the FP32 pass, one thread per sorted pair
+__global__ void k_alloc_blocks_f32(const int32_t* __restrict__ pairs, const int32_t* __restrict__ sorted_pairs,
+                                   int64_t n_pairs, const int32_t* __restrict__ pair_nb,
+                                   const int64_t* __restrict__ blk_off, const int64_t* __restrict__ roff,
                                    const int64_t* __restrict__ hoff, const int64_t* __restrict__ hc_off,
                                    const int64_t* __restrict__ item_tab_off, BlkDesc* __restrict__ blk) {
   constexpr int K = F32_K;
-  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n_pairs; p += (int64_t)gridDim.x * blockDim.x) {
-    const int bin = pair_bin[p];
-    if (bin < 0) continue;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_pairs; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t p = sorted_pairs[i];
     const int nb = pair_nb[p];
     const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
     const int m = (int)(roff[r + 1] - roff[r]);
     const int f = nb * K - (m + 3);  // R row index within the pair's rows
-    const unsigned long long g0 = bin_start[bin] + atomicAdd(&bin_cursor[bin], (unsigned long long)nb);
+    const int64_t g0 = blk_off[i];
     const uint32_t tab0 = (uint32_t)item_tab_off[r];
     const int nh = (int)(hoff[h + 1] - hoff[h]);
     for (int j = 0; j < nb; ++j) {

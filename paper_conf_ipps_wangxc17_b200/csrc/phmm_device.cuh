@@ -46,6 +46,9 @@ __global__ void k_validate_offsets(const int64_t* __restrict__ off, int64_t n, i
 
 // Per pair: validate indices/lengths, bin by column count, count blocks per bin.
 // pair_list == nullptr -> pairs 0..n-1, else the listed pair ids (rescue pass).
+// Counters are aggregated per warp (match_any + reduce) before one atomic per
+// distinct bin and per warp: with one length bin every pair would otherwise hit
+// the same address.
 template <int K>
 __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __restrict__ pair_list,
                             const int64_t* __restrict__ n_list_dev, int64_t n_pairs,
@@ -57,28 +60,62 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
                             unsigned long long* __restrict__ padded_cells, unsigned long long* __restrict__ total_blocks,
                             uint32_t* err) {
   const int64_t n = n_list_dev ? *n_list_dev : n_pairs;
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t p = pair_list ? pair_list[k] : k;
-    const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
-    if (r < 0 || r >= n_reads || h < 0 || h >= n_haps) {
-      atomicOr(err, ERR_INDEX);
-      pair_bin[k] = -1; pair_nb[k] = 0;
-      continue;
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  uint32_t e = 0;
+  unsigned long long my_cells = 0, my_padded = 0, my_blocks = 0;
+  int my_max = 0;
+  for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < n; base += stride) {
+    const int64_t k = base + lane;
+    int bin = -1, nb = 0;
+    if (k < n) {
+      const int64_t p = pair_list ? pair_list[k] : k;
+      const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
+      if (r < 0 || r >= n_reads || h < 0 || h >= n_haps) {
+        e |= ERR_INDEX;
+      } else {
+        const int64_t m = roff[r + 1] - roff[r], nh = hoff[h + 1] - hoff[h];
+        if (m < 1 || nh < 1) {
+          e |= ERR_EMPTY;
+        } else if (nh > kMaxHapLen || m > (1 << 20)) {
+          e |= ERR_ARG;
+        } else {
+          const int nc = ncols_of((int)nh, bucket);
+          bin = bin_of_ncols(nc, bucket);
+          nb = nblocks_of<K>((int)m);
+          my_max = max(my_max, nc);
+          my_cells += (unsigned long long)(m * nh);
+          my_padded += (unsigned long long)nb * K * nc;
+          my_blocks += (unsigned long long)nb;
+        }
+      }
+      pair_bin[k] = bin;
+      pair_nb[k] = nb;
     }
-    const int64_t m = roff[r + 1] - roff[r], nh = hoff[h + 1] - hoff[h];
-    if (m < 1 || nh < 1) { atomicOr(err, ERR_EMPTY); pair_bin[k] = -1; pair_nb[k] = 0; continue; }
-    if (nh > kMaxHapLen || m > (1 << 20)) { atomicOr(err, ERR_ARG); pair_bin[k] = -1; pair_nb[k] = 0; continue; }
-    const int nc = ncols_of((int)nh, bucket);
-    const int bin = bin_of_ncols(nc, bucket);
-    const int nb = nblocks_of<K>((int)m);
-    pair_bin[k] = bin;
-    pair_nb[k] = nb;
-    atomicAdd(&bin_blocks[bin], (unsigned long long)nb);
-    atomicAdd(&bin_pairs[bin], 1ull);
-    atomicMax(max_ncols, nc);
-    atomicAdd(cells, (unsigned long long)(m * nh));
-    atomicAdd(padded_cells, (unsigned long long)nb * K * nc);
-    atomicAdd(total_blocks, (unsigned long long)nb);
+    const unsigned act = __ballot_sync(0xffffffffu, bin >= 0);
+    if (bin >= 0) {
+      const unsigned peers = __match_any_sync(act, bin);
+      const unsigned sum_nb = __reduce_add_sync(peers, (unsigned)nb);
+      if (lane == __ffs(peers) - 1) {
+        atomicAdd(&bin_blocks[bin], (unsigned long long)sum_nb);
+        atomicAdd(&bin_pairs[bin], (unsigned long long)__popc(peers));
+      }
+    }
+  }
+  // one atomic per warp for the scalars
+  for (int o = 16; o > 0; o >>= 1) {
+    my_cells += __shfl_xor_sync(0xffffffffu, my_cells, o);
+    my_padded += __shfl_xor_sync(0xffffffffu, my_padded, o);
+    my_blocks += __shfl_xor_sync(0xffffffffu, my_blocks, o);
+    my_max = max(my_max, __shfl_xor_sync(0xffffffffu, my_max, o));
+    e |= __shfl_xor_sync(0xffffffffu, e, o);
+  }
+  if (lane == 0) {
+    if (my_cells) atomicAdd(cells, my_cells);
+    if (my_padded) atomicAdd(padded_cells, my_padded);
+    if (my_blocks) atomicAdd(total_blocks, my_blocks);
+    if (my_max) atomicMax(max_ncols, my_max);
+    if (e) atomicOr(err, e);
   }
 }
 

@@ -6,6 +6,7 @@
 //   block allocation per bin (the length-binned scheduler, §8a-3), the
 //   wavefront kernel (§8a-4), finalize (§8a-5) and, for FP32, the FP64
 //   rescue of underflowing pairs (§8a-6). See DESIGN.md §3-§5.
+#include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 
 #include <algorithm>
@@ -28,7 +29,8 @@ enum BufId {
   B_HCODES, B_SCAL,                                                       // codes, scalars
   B_PAIR_BIN, B_PAIR_NB, B_BINS, B_ITEM_NB, B_ITEM_OFF, B_SCAN_TMP,
   B_TAB, B_BLK, B_OUT32, B_OUT64, B_RLIST, B_ITEM_READ, B_PAIR_ITEM,
-  B_OUT_LOG10, B_OUT_STATUS, B_HNC, B_HC_OFF, B_HCODES32, B_TAB32, B_COUNT
+  B_OUT_LOG10, B_OUT_STATUS, B_HNC, B_HC_OFF, B_HCODES32, B_TAB32,
+  B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_COUNT
 };
 
 struct Buf {
@@ -382,7 +384,7 @@ phmm_status pass_run_f32(phmm_ctx* c, const DevBatch& d, const PassInfo& pi, int
   ST_TRY(ws(c, B_TAB32, (size_t)total_tab, &tab));
   ST_TRY(ws(c, B_BLK, (size_t)pi.total_blocks, &blk));
   ST_TRY(ws(c, B_HCODES32, (size_t)(total_hc + pad_len), &hc));
-  CUDA_TRY(cudaMemsetAsync(hc + total_hc, F32_PAD, (size_t)pad_len, s));
+  CUDA_TRY(cudaMemsetAsync(hc + total_hc, F32_PAD * 2, (size_t)pad_len, s));
   if (total_tab > 0) {
     k_build_table_f32<<<grid_for(c, total_tab * F32_K), kThreads, 0, s>>>(
         d.n_reads, item_off, item_off + d.n_reads, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
@@ -403,14 +405,40 @@ phmm_status pass_run_f32(phmm_ctx* c, const DevBatch& d, const PassInfo& pi, int
   const int nbins = kMaxBins + 1;
   k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, chunk, bin_start, item_start);
   LAUNCHED(c);
-  k_alloc_blocks_f32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(d.pairs, d.n_pairs, pair_bin, pair_nb, bin_start,
-                                                                 bin_cursor, d.roff, d.hoff, hc_off, item_off, blk);
-  LAUNCHED(c);
+  // stable sort of the pairs by bin, then contiguous block ranges by an exclusive scan
+  {
+    const int64_t n = d.n_pairs;
+    uint32_t* keys;
+    int32_t* vals;
+    int64_t *nbs, *blk_off;
+    ST_TRY(ws(c, B_SKEYS, (size_t)2 * n, &keys));
+    ST_TRY(ws(c, B_SVALS, (size_t)2 * n, &vals));
+    ST_TRY(ws(c, B_NBS, (size_t)n + 1, &nbs));
+    ST_TRY(ws(c, B_BLKOFF, (size_t)n + 1, &blk_off));
+    k_iota_keys<<<grid_for(c, n), kThreads, 0, s>>>(pair_bin, n, keys, vals);
+    LAUNCHED(c);
+    int end_bit = 1;
+    while ((1 << end_bit) <= kMaxBins + 1) ++end_bit;
+    size_t sort_bytes = 0, scan_bytes = 0;
+    CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+    CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, nbs, blk_off, n + 1, s));
+    unsigned char* tmp;
+    ST_TRY(ws(c, B_SORT_TMP, std::max(sort_bytes, scan_bytes), &tmp));
+    CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+    c->launches += 2;
+    k_sorted_nb<<<grid_for(c, n), kThreads, 0, s>>>(vals + n, pair_nb, n, nbs);
+    LAUNCHED(c);
+    CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, scan_bytes, nbs, blk_off, n + 1, s));
+    ++c->launches;
+    k_alloc_blocks_f32<<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, vals + n, n, pair_nb, blk_off, d.roff, d.hoff,
+                                                          hc_off, item_off, blk);
+    LAUNCHED(c);
+  }
   F32Args A;
   A.blk = blk;
   A.tab = tab;
   A.hcodes = hc;
-  A.pad_idx = (uint32_t)(total_hc + 16);
+  A.pad_idx = (uint32_t)total_hc;  // 4-aligned: every haplotype region is a multiple of 4
   A.bin_start = bin_start;
   A.item_start = item_start;
   A.nbins = nbins;

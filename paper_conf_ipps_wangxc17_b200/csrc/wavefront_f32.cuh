@@ -153,10 +153,34 @@ __device__ __forceinline__ void f32_column(F32Lane& L, const float4 pA, const fl
   }
 }
 
-// Load a block (or nothing) into half H of a lane.
+// ---- shared-memory ring accessors (inline PTX, "memory" clobber: the ring is read
+// and written through these only, so no compiler reordering or aliasing games)
+__device__ __forceinline__ void ring_put3(uint32_t saddr, float a, float b, float c) {
+  asm volatile("st.shared.f32 [%0], %1;\n\tst.shared.f32 [%0+4], %2;\n\tst.shared.f32 [%0+8], %3;"
+               :: "r"(saddr), "f"(a), "f"(b), "f"(c) : "memory");
+}
+__device__ __forceinline__ void ring_get3(uint32_t saddr, float& a, float& b, float& c) {
+  float d;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(a), "=f"(b), "=f"(c), "=f"(d) : "r"(saddr) : "memory");
+}
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// Haplotype code slots (4 shifted copies per haplotype so that every lane reads its
+// codes as aligned 32-bit words, 4 columns at a time). Byte = code * 32, the
+// float4 index of that code's entry in a lane's prior table.
+__host__ __device__ inline int f32_hc_copy_len(int ncols) {
+  const int p = (ncols + F32_G > F32_MIN_P) ? ncols + F32_G : F32_MIN_P;
+  return ((int)F32_HC_FRONT + p + 16 + 3) & ~3;
+}
+
+// Load a block (or nothing) into half H of a lane. Returns the 32-bit-aligned code
+// pointer for the lane's first step (column -1 - gi).
 template <int H>
-__device__ __forceinline__ void f32_load(const F32Args& A, F32Lane& L, float4* __restrict__ my_tab, bool have,
-                                         const BlkDesc& d, float d0, uint32_t& idx, int& out_idx, int gi) {
+__device__ __forceinline__ const uint32_t* f32_load(const F32Args& A, F32Lane& L, float4* __restrict__ my_tab,
+                                                    bool have, const BlkDesc& d, float d0, int& out_idx, int gi,
+                                                    int copy_len) {
   if (have) {
     const float4* __restrict__ s4 = reinterpret_cast<const float4*>(A.tab + d.tab_blk);
     float4 cw[6];
@@ -177,89 +201,88 @@ __device__ __forceinline__ void f32_load(const F32Args& A, F32Lane& L, float4* _
       L.M[u] = set_half<H>(L.M[u], 0.f); L.I[u] = set_half<H>(L.I[u], 0.f);
       L.D[u] = set_half<H>(L.D[u], rrow == u ? d0 : 0.f);
     }
-    idx = d.hap_off - (uint32_t)gi;  // = code index of column (-1 - gi) + 1
     out_idx = (d.flags & BLK_LAST) ? d.out_idx : -1;
-  } else {
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      L.al[u] = set_half<H>(L.al[u], 0.f); L.be[u] = set_half<H>(L.be[u], 0.f);
-      L.de[u] = set_half<H>(L.de[u], 0.f); L.ep[u] = set_half<H>(L.ep[u], 0.f);
-      L.ze[u] = set_half<H>(L.ze[u], 0.f); L.mu[u] = set_half<H>(L.mu[u], 0.f);
-      L.M[u] = set_half<H>(L.M[u], 0.f); L.I[u] = set_half<H>(L.I[u], 0.f);
-      L.D[u] = set_half<H>(L.D[u], 0.f);
-    }
-    idx = A.pad_idx;
-    out_idx = -1;
+    // copy k = (1 + gi) mod 4 has column 0 at hap_off + k*(copy_len + 1), so the byte
+    // of column (-1 - gi) is 4-aligned
+    const int k = (1 + gi) & 3;
+    const uint32_t col0 = d.hap_off + (uint32_t)(k * (copy_len + 1));
+    return reinterpret_cast<const uint32_t*>(A.hcodes + (col0 - 1u - (uint32_t)gi));
   }
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    L.al[u] = set_half<H>(L.al[u], 0.f); L.be[u] = set_half<H>(L.be[u], 0.f);
+    L.de[u] = set_half<H>(L.de[u], 0.f); L.ep[u] = set_half<H>(L.ep[u], 0.f);
+    L.ze[u] = set_half<H>(L.ze[u], 0.f); L.mu[u] = set_half<H>(L.mu[u], 0.f);
+    L.M[u] = set_half<H>(L.M[u], 0.f); L.I[u] = set_half<H>(L.I[u], 0.f);
+    L.D[u] = set_half<H>(L.D[u], 0.f);
+  }
+  out_idx = -1;
+  return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
 }
 
 // One warp streams through blocks [s, s+nblk) of one bin (ncols columns each).
+// Virtual lane v = 2*lane + h (h = 0: half A = low 32 bits, h = 1: half B = high 32 bits),
+// so half B's row above is its own lane's half A one step earlier (no shuffle) and
+// half A's row above is lane-1's half B (one shuffle per value).
 __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict__ ptab, float4* __restrict__ ring,
                                            int lane, int64_t s, int nblk, int ncols, bool trace = false) {
-  constexpr int G = F32_G;
-  constexpr int NGRP = 64 / G;  // switch events per pass
-  const int grp = lane / G, gi = lane % G;  // within a half
+  constexpr int G = F32_G;            // virtual lanes per switch group
+  constexpr int NGRP = 64 / G;        // switch events per pass
+  constexpr int LPG = G / 2;          // physical lanes per group
+  const int grp = lane / LPG;
+  const int giA = 2 * (lane % LPG), giB = giA + 1;  // position of each half inside its group
   const float d0 = ldexpf(1.0f, 120) / (float)ncols;  // virtual row 0
-  const int P = max(ncols + G, F32_MIN_P);
+  const int P = max(ncols + G, F32_MIN_P);           // multiple of 4 (ncols is)
   const int npass = (nblk + 63) >> 6;
-  const uint8_t* __restrict__ const hc = A.hcodes;
+  const int copy_len = f32_hc_copy_len(ncols);
   F32Lane L;
 #pragma unroll
   for (int u = 0; u < 4; ++u) {
     L.al[u] = L.be[u] = L.de[u] = L.ep[u] = L.ze[u] = L.mu[u] = 0ull;
     L.M[u] = L.I[u] = L.D[u] = 0ull;
   }
-  uint32_t idxA = A.pad_idx, idxB = A.pad_idx;  // code index of the next column
-  int codeA_nx = F32_PAD, codeB_nx = F32_PAD;
+  const uint32_t* pA = reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);  // next code word
+  const uint32_t* pB = pA;
+  constexpr uint32_t kPadW = 0x0a0a0a0au;  // four PAD codes (byte = code * 2)
+  uint32_t wA = kPadW, wB = kPadW, wA_nx = kPadW, wB_nx = kPadW;
   int outA = -1, outB = -1;
   v2 upM = 0ull, upI = 0ull, upD = 0ull, dgM = 0ull, dgI = 0ull, dgD = 0ull;
-  float4* const tabA = ptab + lane;                   // [code][lane], half A
-  float4* const tabB = ptab + F32_NCODE * 32 + lane;  // half B
+  const uint32_t tabA_s = smem_addr(ptab + lane);                   // [code][lane] float4, half A
+  const uint32_t tabB_s = smem_addr(ptab + F32_NCODE * 32 + lane);  // half B
+  const uint32_t ring_s = smem_addr(ring);
   const int src = (lane + 31) & 31;
   const bool is0 = lane == 0, is31 = lane == 31;
-  int c0 = -(1 << 20);    // (uniform) column of lane 0's half A
-  int c31B = -(1 << 20);  // (uniform) column of lane 31's half B
-  float* const ringf = reinterpret_cast<float*>(ring);
-  const int rmax = A.ring_len - 1;
+  int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
+  int c31B = -(1 << 20);  // (uniform) column of virtual lane 63 (lane 31, half B)
+  float rvM = 0.f, rvI = 0.f, rvD = 0.f;  // lane 31: ring slot for virtual lane 0's next column
 #ifdef PHMM_DBG_TRACE
   int tstep = 0;
 #endif
 
-  auto step = [&]() {
-#ifdef PHMM_DBG_SYNC
-    __syncwarp();
-#endif
-    // lane 31: the ring slot that virtual lane 0 needs next step (column c0 + 1)
-    // (the ring is only ever accessed as float: one access type, no aliasing games)
-    float rvM = 0.f, rvI = 0.f, rvD = 0.f;
-    if (is31) {
-      const float* r = ringf + 4 * min(c0 + 2, rmax);
-      rvM = r[0]; rvI = r[1]; rvD = r[2];
-    }
-    const int codeA = codeA_nx, codeB = codeB_nx;
-    codeA_nx = hc[idxA++];
-    codeB_nx = hc[idxB++];
-    const float4 pA = tabA[codeA * 32];
-    const float4 pB = tabB[codeB * 32];
-    f32_column(L, pA, pB, dgM, dgI, dgD, upM, upI);
-    // what lane 31 sends: half A stream <- ring (for virtual lane 0), half B stream <- its half A
+  auto step = [&](const int r) {
+    if (is31) ring_get3(ring_s + 16u * (uint32_t)(c0 + 2), rvM, rvI, rvD);
+    // code byte r (= code*2) placed in byte 1 -> code*512 = the code's row in the table
+    const uint32_t oA = __byte_perm(wA, 0, 0x4404 + (r << 4)), oB = __byte_perm(wB, 0, 0x4404 + (r << 4));
+    float4 prA, prB;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(prA.x), "=f"(prA.y), "=f"(prA.z), "=f"(prA.w)
+                 : "r"(tabA_s + oA));
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(prB.x), "=f"(prB.y), "=f"(prB.z), "=f"(prB.w)
+                 : "r"(tabB_s + oB));
+    f32_column(L, prA, prB, dgM, dgI, dgD, upM, upI);
     const float m3a = lo(L.M[3]), i3a = lo(L.I[3]), d3a = lo(L.D[3]);
     const float m3b = hi(L.M[3]), i3b = hi(L.I[3]), d3b = hi(L.D[3]);
-    const float sAM = is31 ? rvM : m3a;
-    const float sAI = is31 ? rvI : i3a;
-    const float sAD = is31 ? rvD : d3a;
-    const float sBM = is31 ? m3a : m3b;
-    const float sBI = is31 ? i3a : i3b;
-    const float sBD = is31 ? d3a : d3b;
-    if (is31 && (unsigned)(c31B + 1) <= (unsigned)ncols) {  // -1 <= c31B < ncols
-      float* e = ringf + 4 * (c31B + 1);
-      e[0] = m3b; e[1] = i3b; e[2] = d3b;
-    }
+    // half B of lane-1 -> half A of lane; lane 31 sends the ring slot instead (virtual 63 -> 0)
+    const float sM = is31 ? rvM : m3b;
+    const float sI = is31 ? rvI : i3b;
+    const float sD = is31 ? rvD : d3b;
+    if (is31 && (unsigned)(c31B + 1) <= (unsigned)ncols)  // -1 <= c31B < ncols
+      ring_put3(ring_s + 16u * (uint32_t)(c31B + 1), m3b, i3b, d3b);
     __syncwarp();
     dgM = upM; dgI = upI; dgD = upD;
-    upM = pk(__shfl_sync(0xffffffffu, sAM, src), __shfl_sync(0xffffffffu, sBM, src));
-    upI = pk(__shfl_sync(0xffffffffu, sAI, src), __shfl_sync(0xffffffffu, sBI, src));
-    upD = pk(__shfl_sync(0xffffffffu, sAD, src), __shfl_sync(0xffffffffu, sBD, src));
+    // next step: half A's row above = lane-1's half B; half B's row above = this lane's half A
+    upM = pk(__shfl_sync(0xffffffffu, sM, src), m3a);
+    upI = pk(__shfl_sync(0xffffffffu, sI, src), i3a);
+    upD = pk(__shfl_sync(0xffffffffu, sD, src), d3a);
 #ifdef PHMM_DBG_TRACE
     if (trace && tstep < 4096) {
       float* t = g_trace + ((size_t)tstep * 32 + lane) * 6;
@@ -272,44 +295,42 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
     ++c0;
     ++c31B;
   };
+  // 4 steps sharing one code word per half; the next words are prefetched
+  auto group4 = [&]() {
+    wA = wA_nx; wB = wB_nx;
+    wA_nx = __ldg(pA); wB_nx = __ldg(pB);
+    ++pA; ++pB;
+    step(0); step(1); step(2); step(3);
+  };
 
   for (int q = 0; q <= npass; ++q) {
 #pragma unroll 1
     for (int e = 0; e < NGRP; ++e) {
-      const int h = e / (NGRP / 2), g = e % (NGRP / 2);
-      if (e == 0) {  // lane 0 half A starts its pass: column -1 next
-        c0 = -1;
-      }
-      if (e == NGRP - 1) c31B = -1 - (G - 1);  // lane 31 half B
-      if (grp == g) {  // switch event of virtual group (h, g): SIMT over its G lanes
-        const int b = q * 64 + h * 32 + lane;
-        const bool have = (q < npass) && (b < nblk);
-        BlkDesc d;
-        d.tab_blk = 0; d.hap_off = 0; d.out_idx = -1; d.n = 1; d.flags = 0;
-        if (have) d = A.blk[s + b];
-        if (h == 0) {
-          if (outA >= 0) A.out[outA] = lo(L.D[3]);  // S2 row: the last-row M+I sum (L20@2262)
-          f32_load<0>(A, L, tabA, have, d, d0, idxA, outA, gi);
-          codeA_nx = F32_PAD;
-          if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
-            upM = set_half<0>(upM, ringf[0]); upI = set_half<0>(upI, ringf[1]); upD = set_half<0>(upD, ringf[2]);
-          }
-        } else {
-          if (outB >= 0) A.out[outB] = hi(L.D[3]);
-          f32_load<1>(A, L, tabB, have, d, d0, idxB, outB, gi);
-          codeB_nx = F32_PAD;
+      if (e == 0) c0 = -1;                      // virtual lane 0 starts its pass: column -1 next
+      if (e == NGRP - 1) c31B = -1 - (G - 1);  // virtual lane 63
+      if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
+        const int bA = q * 64 + 2 * lane, bB = bA + 1;
+        const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
+        BlkDesc dA, dB;
+        dA.tab_blk = 0; dA.hap_off = 0; dA.out_idx = -1; dA.n = 1; dA.flags = 0;
+        dB = dA;
+        if (hA) dA = A.blk[s + bA];
+        if (hB) dB = A.blk[s + bB];
+        if (outA >= 0) A.out[outA] = lo(L.D[3]);  // S2 row: the last-row M+I sum (L20@2262)
+        if (outB >= 0) A.out[outB] = hi(L.D[3]);
+        pA = f32_load<0>(A, L, ptab + lane, hA, dA, d0, outA, giA, copy_len);
+        pB = f32_load<1>(A, L, ptab + F32_NCODE * 32 + lane, hB, dB, d0, outB, giB, copy_len);
+        wA_nx = __ldg(pA); ++pA;
+        wB_nx = __ldg(pB); ++pB;
+        if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
+          float a, bb, c;
+          ring_get3(ring_s, a, bb, c);
+          upM = set_half<0>(upM, a); upI = set_half<0>(upI, bb); upD = set_half<0>(upD, c);
         }
       }
-      const int nsteps = (e < NGRP - 1) ? G : (q < npass ? P - (NGRP - 1) * G : 0);
-#ifndef PHMM_F32_UNROLL
-#define PHMM_F32_UNROLL 2
-#endif
-#if PHMM_F32_UNROLL == 1
+      const int ngroups = (e < NGRP - 1) ? G / 4 : (q < npass ? (P - (NGRP - 1) * G) / 4 : 0);
 #pragma unroll 1
-#else
-#pragma unroll 2
-#endif
-      for (int k = 0; k < nsteps; ++k) step();
+      for (int k = 0; k < ngroups; ++k) group4();
     }
   }
 }
@@ -323,7 +344,7 @@ cudaError_t wf32_launch(unsigned grid, size_t smem, cudaStream_t stream, const F
 
 #ifdef PHMM_DEFINE_WF32
 #ifndef PHMM_F32_MINB
-#define PHMM_F32_MINB 4  // CTAs (of 4 warps) per SM the register budget must allow
+#define PHMM_F32_MINB 3  // CTAs (of 4 warps) per SM the register budget must allow (168 regs)
 #endif
 __global__ void __launch_bounds__(F32_WARPS * 32, PHMM_F32_MINB) k_wavefront_f32(F32Args A) {
   extern __shared__ __align__(16) unsigned char smem_raw[];

@@ -1,0 +1,16 @@
+#!/bin/bash
+# compute-sanitizer passes on small inputs (each bounded by timeout)
+cat > /tmp/san_case.py <<'PY'
+import sys; sys.path.insert(0, '.')
+import numpy as np
+from paper_conf_ipps_wangxc17_b200 import phmm, synth
+b = synth.concat_batches([synth.config_batch("C2", n_regions=4), synth.random_pairs_batch(3, 100, m_range=(1, 60), n_range=(1, 80))])
+for prec in ("fp32", "fp64"):
+    with phmm.PairHMM(precision=prec) as h:
+        out, st = h.compute_batch(b)
+        print(prec, "ok", np.isfinite(out).sum(), "rescued", int((st == 1).sum()))
+PY
+for tool in memcheck racecheck synccheck; do
+  echo "== $tool"
+  timeout 600 compute-sanitizer --tool $tool --print-limit 5 python /tmp/san_case.py 2>&1 | grep -E "ERROR SUMMARY|hazard|ok|Invalid|RACECHECK" | head -8
+done
