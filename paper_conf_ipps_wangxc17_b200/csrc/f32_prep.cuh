@@ -57,17 +57,16 @@ __global__ void k_hap_ncols(const int64_t* __restrict__ hoff, int64_t n_haps, in
   if (blockIdx.x == 0 && threadIdx.x == 0) nc[n_haps] = 0;
 }
 
-// per-read FP32 tables: one thread per padded row (same row layout as k_build_table)
+// per-read FP32 tables: one thread per 4-row block (binary search of its read once
+// per block), the 176-byte block written as 11 float4 stores
 __global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ item_tab_off,
                                   const int64_t* __restrict__ total_tab_blocks_dev, const int64_t* __restrict__ roff,
                                   const uint8_t* __restrict__ rb, const uint8_t* __restrict__ q,
                                   const uint8_t* __restrict__ qi, const uint8_t* __restrict__ qd,
                                   const uint8_t* __restrict__ qg, F32Block* __restrict__ tab) {
   constexpr int K = F32_K;
-  const int64_t total_rows = (*total_tab_blocks_dev) * K;
-  for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < total_rows; g += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t b = g / K;
-    const int t = (int)(g % K);
+  const int64_t total = *total_tab_blocks_dev;
+  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < total; b += (int64_t)gridDim.x * blockDim.x) {
     int64_t lo = 0, hi = n_reads - 1;
     while (lo < hi) {
       const int64_t mid = (lo + hi + 1) >> 1;
@@ -78,41 +77,49 @@ __global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ i
     const int m = (int)(roff[r + 1] - r0);
     const int nb = nblocks_of<K>(m);
     const int f = nb * K - (m + 3);
-    const int row = (int)(b - item_tab_off[r]) * K + t;
-    float al = 0, be = 0, de = 0, ep = 0, ze = 0, mu = 0;
-    float pr[5] = {0, 0, 0, 0, 0};
-    if (row < f) {
-      // Z row: all zero
-    } else if (row == f) {  // R row: D = d0 on every column
-      mu = 1;
-    } else if (row <= f + m) {
-      const int64_t x = r0 + (row - f - 1);
-      const float ei = qual_err<float>(qi[x]), ed = qual_err<float>(qd[x]), eg = qual_err<float>(qg[x]),
-                  eb = qual_err<float>(q[x]);
-      const float sum = ei + ed;
-      al = 1.f - (sum < 1.f ? sum : 1.f);
-      be = 1.f - eg;
-      de = ei;
-      ep = eg;
-      ze = ed;
-      mu = eg;
-      const float pm = 1.f - eb, px = eb / 3.f;
-      const uint8_t base = rb[x];
-      const uint8_t codes[4] = {'A', 'C', 'G', 'T'};
+    float co[6][4], pr[5][4];
 #pragma unroll
-      for (int k = 0; k < 4; ++k) pr[k] = (base == codes[k] || base == 'N') ? pm : px;
-      pr[4] = pm;  // haplotype 'N' matches everything
-    } else if (row == f + m + 1) {  // S1: I = M(m,j) + I(m,j)
-      de = 1; ep = 1; mu = 1;
-    } else {  // S2: M = I_S1(j-1), D = running sum
-      be = 1; ze = 1; mu = 1;
-      pr[0] = pr[1] = pr[2] = pr[3] = pr[4] = 1;
+    for (int t = 0; t < K; ++t) {
+      const int row = (int)(b - item_tab_off[r]) * K + t;
+      float al = 0, be = 0, de = 0, ep = 0, ze = 0, mu = 0;
+      float p5[5] = {0, 0, 0, 0, 0};
+      if (row < f) {
+        // Z row: all zero
+      } else if (row == f) {  // R row: D = d0 on every column
+        mu = 1;
+      } else if (row <= f + m) {
+        const int64_t x = r0 + (row - f - 1);
+        const float ei = qual_err<float>(qi[x]), ed = qual_err<float>(qd[x]), eg = qual_err<float>(qg[x]),
+                    eb = qual_err<float>(q[x]);
+        const float sum = ei + ed;
+        al = 1.f - (sum < 1.f ? sum : 1.f);
+        be = 1.f - eg;
+        de = ei;
+        ep = eg;
+        ze = ed;
+        mu = eg;
+        const float pm = 1.f - eb, px = eb / 3.f;
+        const uint8_t base = rb[x];
+        p5[0] = (base == 'A' || base == 'N') ? pm : px;
+        p5[1] = (base == 'C' || base == 'N') ? pm : px;
+        p5[2] = (base == 'G' || base == 'N') ? pm : px;
+        p5[3] = (base == 'T' || base == 'N') ? pm : px;
+        p5[4] = pm;  // haplotype 'N' matches everything
+      } else if (row == f + m + 1) {  // S1: I = M(m,j) + I(m,j)
+        de = 1; ep = 1; mu = 1;
+      } else {  // S2: M = I_S1(j-1), D = running sum
+        be = 1; ze = 1; mu = 1;
+        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = 1;
+      }
+      co[0][t] = al; co[1][t] = be; co[2][t] = de; co[3][t] = ep; co[4][t] = ze; co[5][t] = mu;
+#pragma unroll
+      for (int k = 0; k < 5; ++k) pr[k][t] = p5[k];
     }
-    F32Block& B = tab[b];
-    B.coef[0][t] = al; B.coef[1][t] = be; B.coef[2][t] = de;
-    B.coef[3][t] = ep; B.coef[4][t] = ze; B.coef[5][t] = mu;
+    float4* dst = reinterpret_cast<float4*>(tab + b);
 #pragma unroll
-    for (int k = 0; k < 5; ++k) B.prior[k][t] = pr[k];
+    for (int k = 0; k < 6; ++k) dst[k] = make_float4(co[k][0], co[k][1], co[k][2], co[k][3]);
+#pragma unroll
+    for (int k = 0; k < 5; ++k) dst[6 + k] = make_float4(pr[k][0], pr[k][1], pr[k][2], pr[k][3]);
   }
 }
 
@@ -135,31 +142,52 @@ __global__ void k_sorted_nb(const int32_t* __restrict__ sorted_pairs, const int3
   if (blockIdx.x == 0 && threadIdx.x == 0) nb_sorted[n] = 0;
 }
 
-// block descriptors for the FP32 pass, one thread per sorted pair
+// block descriptors for the FP32 pass: one warp per 32 sorted pairs, the lanes of
+// the warp write one pair's descriptors together (coalesced 16-byte stores)
 __global__ void k_alloc_blocks_f32(const int32_t* __restrict__ pairs, const int32_t* __restrict__ sorted_pairs,
                                    int64_t n_pairs, const int32_t* __restrict__ pair_nb,
                                    const int64_t* __restrict__ blk_off, const int64_t* __restrict__ roff,
                                    const int64_t* __restrict__ hoff, const int64_t* __restrict__ hc_off,
                                    const int64_t* __restrict__ item_tab_off, BlkDesc* __restrict__ blk) {
   constexpr int K = F32_K;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n_pairs; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t p = sorted_pairs[i];
-    const int nb = pair_nb[p];
-    const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
-    const int m = (int)(roff[r + 1] - roff[r]);
-    const int f = nb * K - (m + 3);  // R row index within the pair's rows
-    const int64_t g0 = blk_off[i];
-    const uint32_t tab0 = (uint32_t)item_tab_off[r];
-    const int nh = (int)(hoff[h + 1] - hoff[h]);
-    for (int j = 0; j < nb; ++j) {
-      BlkDesc d;
-      d.tab_blk = tab0 + j;
-      d.hap_off = (uint32_t)(hc_off[h] + F32_HC_FRONT);
-      d.out_idx = (int32_t)p;
-      d.n = (uint16_t)nh;
-      const int rrow = (f / K == j) ? (f % K) : F32_RROW_NONE;
-      d.flags = (uint16_t)((j == nb - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) | (rrow << F32_RROW_SHIFT));
-      blk[g0 + j] = d;
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < n_pairs; base += stride) {
+    // per-lane pair data
+    const int64_t i = base + lane;
+    int nb = 0, m = 0, nh = 0;
+    int64_t g0 = 0, p = 0;
+    uint32_t tab0 = 0, hap = 0;
+    if (i < n_pairs) {
+      p = sorted_pairs[i];
+      nb = pair_nb[p];
+      const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
+      m = (int)(roff[r + 1] - roff[r]);
+      nh = (int)(hoff[h + 1] - hoff[h]);
+      g0 = blk_off[i];
+      tab0 = (uint32_t)item_tab_off[r];
+      hap = (uint32_t)(hc_off[h] + F32_HC_FRONT);
+    }
+    const int cnt = (int)min((int64_t)32, n_pairs - base);
+    for (int src = 0; src < cnt; ++src) {
+      const int nb_s = __shfl_sync(0xffffffffu, nb, src);
+      const int m_s = __shfl_sync(0xffffffffu, m, src);
+      const int nh_s = __shfl_sync(0xffffffffu, nh, src);
+      const int64_t g0_s = __shfl_sync(0xffffffffu, g0, src);
+      const int64_t p_s = __shfl_sync(0xffffffffu, p, src);
+      const uint32_t tab_s = __shfl_sync(0xffffffffu, tab0, src);
+      const uint32_t hap_s = __shfl_sync(0xffffffffu, hap, src);
+      const int f = nb_s * K - (m_s + 3);  // R row index within the pair's rows
+      for (int j = lane; j < nb_s; j += 32) {
+        BlkDesc d;
+        d.tab_blk = tab_s + j;
+        d.hap_off = hap_s;
+        d.out_idx = (int32_t)p_s;
+        d.n = (uint16_t)nh_s;
+        const int rrow = (f / K == j) ? (f % K) : F32_RROW_NONE;
+        d.flags = (uint16_t)((j == nb_s - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) | (rrow << F32_RROW_SHIFT));
+        blk[g0_s + j] = d;
+      }
     }
   }
 }

@@ -255,6 +255,9 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
   int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
   int c31B = -(1 << 20);  // (uniform) column of virtual lane 63 (lane 31, half B)
   float rvM = 0.f, rvI = 0.f, rvD = 0.f;  // lane 31: ring slot for virtual lane 0's next column
+  BlkDesc dnA, dnB;  // next pass's block descriptors (prefetched)
+  dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.n = 1; dnA.flags = 0;
+  dnB = dnA;
 #ifdef PHMM_DBG_TRACE
   int tstep = 0;
 #endif
@@ -311,17 +314,24 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
       if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
         const int bA = q * 64 + 2 * lane, bB = bA + 1;
         const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
-        BlkDesc dA, dB;
-        dA.tab_blk = 0; dA.hap_off = 0; dA.out_idx = -1; dA.n = 1; dA.flags = 0;
-        dB = dA;
-        if (hA) dA = A.blk[s + bA];
-        if (hB) dB = A.blk[s + bB];
+        // this pass's descriptors were prefetched one pass ago (pass 0: loaded now);
+        // prefetch the next pass's so their latency hides behind P steps
+        BlkDesc dA = dnA, dB = dnB;
+        if (q == 0) {
+          if (hA) dA = A.blk[s + bA];
+          if (hB) dB = A.blk[s + bB];
+        }
+
         if (outA >= 0) A.out[outA] = lo(L.D[3]);  // S2 row: the last-row M+I sum (L20@2262)
         if (outB >= 0) A.out[outB] = hi(L.D[3]);
         pA = f32_load<0>(A, L, ptab + lane, hA, dA, d0, outA, giA, copy_len);
         pB = f32_load<1>(A, L, ptab + F32_NCODE * 32 + lane, hB, dB, d0, outB, giB, copy_len);
         wA_nx = __ldg(pA); ++pA;
         wB_nx = __ldg(pB); ++pB;
+        // prefetch after this pass's loads are issued (a load issued before the
+        // consumers of the previous prefetch would share their scoreboard)
+        if (bA + 64 < nblk) dnA = A.blk[s + bA + 64];
+        if (bB + 64 < nblk) dnB = A.blk[s + bB + 64];
         if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
           float a, bb, c;
           ring_get3(ring_s, a, bb, c);
