@@ -44,7 +44,7 @@ __global__ void k_hap_codes_f32(const uint8_t* __restrict__ hap, const int64_t* 
       } else if (c == n) {
         v = 4;
       }
-      dst[i] = (uint8_t)(v * 2);
+      dst[i] = (uint8_t)(v * F32_CB);
     }
   }
 }
@@ -77,7 +77,7 @@ __global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ i
     const int m = (int)(roff[r + 1] - r0);
     const int nb = nblocks_of<K>(m);
     const int f = nb * K - (m + 3);
-    float co[6][4], pr[5][4];
+    float co[6][F32_K], pr[5][F32_K];
 #pragma unroll
     for (int t = 0; t < K; ++t) {
       const int row = (int)(b - item_tab_off[r]) * K + t;
@@ -117,9 +117,16 @@ __global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ i
     }
     float4* dst = reinterpret_cast<float4*>(tab + b);
 #pragma unroll
-    for (int k = 0; k < 6; ++k) dst[k] = make_float4(co[k][0], co[k][1], co[k][2], co[k][3]);
+    for (int k = 0; k < 6; ++k)
 #pragma unroll
-    for (int k = 0; k < 5; ++k) dst[6 + k] = make_float4(pr[k][0], pr[k][1], pr[k][2], pr[k][3]);
+      for (int ch = 0; ch < F32_KC; ++ch)
+        dst[k * F32_KC + ch] = make_float4(co[k][4 * ch], co[k][4 * ch + 1], co[k][4 * ch + 2], co[k][4 * ch + 3]);
+#pragma unroll
+    for (int k = 0; k < 5; ++k)
+#pragma unroll
+      for (int ch = 0; ch < F32_KC; ++ch)
+        dst[6 * F32_KC + k * F32_KC + ch] =
+            make_float4(pr[k][4 * ch], pr[k][4 * ch + 1], pr[k][4 * ch + 2], pr[k][4 * ch + 3]);
   }
 }
 

@@ -384,7 +384,7 @@ phmm_status pass_run_f32(phmm_ctx* c, const DevBatch& d, const PassInfo& pi, int
   ST_TRY(ws(c, B_TAB32, (size_t)total_tab, &tab));
   ST_TRY(ws(c, B_BLK, (size_t)pi.total_blocks, &blk));
   ST_TRY(ws(c, B_HCODES32, (size_t)(total_hc + pad_len), &hc));
-  CUDA_TRY(cudaMemsetAsync(hc + total_hc, F32_PAD * 2, (size_t)pad_len, s));
+  CUDA_TRY(cudaMemsetAsync(hc + total_hc, F32_PAD * F32_CB, (size_t)pad_len, s));
   if (total_tab > 0) {
     k_build_table_f32<<<grid_for(c, total_tab), kThreads, 0, s>>>(
         d.n_reads, item_off, item_off + d.n_reads, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
@@ -394,7 +394,7 @@ phmm_status pass_run_f32(phmm_ctx* c, const DevBatch& d, const PassInfo& pi, int
   LAUNCHED(c);
 
   const int ring_len = p_max + 4;
-  const size_t smem = (size_t)F32_WARPS * (2 * F32_NCODE * 32 + ring_len) * sizeof(float4);
+  const size_t smem = (size_t)F32_WARPS * (2 * F32_NCODE * F32_KC * 32 + ring_len) * sizeof(float4);
   int bps = 0;
   CUDA_TRY(wf32_occupancy(smem, &bps));
   if (bps < 1) return PHMM_E_INVALID_ARG;

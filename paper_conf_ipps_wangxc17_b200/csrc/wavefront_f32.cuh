@@ -47,7 +47,12 @@ __device__ float g_trace[4096 * 32 * 2 * 3];
 __device__ int g_trace_steps;
 #endif
 
-constexpr int F32_K = 4;      // rows per virtual lane (per half)
+#ifndef PHMM_F32_K
+#define PHMM_F32_K 8
+#endif
+constexpr int F32_K = PHMM_F32_K;  // rows per virtual lane (per half): 4 or 8
+static_assert(F32_K == 4 || F32_K == 8, "F32_K must be 4 or 8");
+constexpr int F32_KC = F32_K / 4;  // float4 chunks per row set
 constexpr int F32_G = 8;      // virtual lanes per switch group
 constexpr int F32_NCODE = 6;  // A C G T N PAD
 constexpr int F32_PAD = 5;
@@ -55,12 +60,15 @@ constexpr int F32_WARPS = 4;   // warps per CTA
 constexpr int F32_MIN_P = 72;  // ring delay: virtual lane 63 -> 0 needs P >= 72
 constexpr int64_t F32_HC_FRONT = 16;  // PAD codes before every haplotype's code array
 
-// per-block coefficient table: 6 transition fields + 5 prior codes, 4 rows each
+// per-block coefficient table: 6 transition fields + 5 prior codes, F32_K rows each
 struct alignas(16) F32Block {
-  float coef[6][4];   // alpha, beta, delta, eps, zeta, mu
-  float prior[5][4];  // P(row, code) for code = A, C, G, T, N
+  float coef[6][F32_K];   // alpha, beta, delta, eps, zeta, mu
+  float prior[5][F32_K];  // P(row, code) for code = A, C, G, T, N
 };
-static_assert(sizeof(F32Block) == 176, "F32Block layout");
+static_assert(sizeof(F32Block) == 44 * F32_K, "F32Block layout");
+// code byte in the haplotype code arrays: code * F32_CB; moved into bits 8..15 it is
+// code * F32_K * 128 bytes = the stride of one code's rows in a lane's prior table
+constexpr int F32_CB = F32_K / 2;
 
 // BlkDesc.flags for the FP32 kernel: bit0 last, bit1 first, bits 8-11 R row (15 = none)
 constexpr uint16_t F32_RROW_SHIFT = 8;
@@ -119,20 +127,18 @@ __device__ __forceinline__ v2 set_half(v2 r, float v) {
   return H == 0 ? pk(v, hi(r)) : pk(lo(r), v);
 }
 
-// lane state: lo = half A (virtual lane l), hi = half B (virtual lane l + 32); index = row 0..3
+// lane state: lo = half A, hi = half B; index = row 0..F32_K-1
 struct F32Lane {
-  v2 al[4], be[4], de[4], ep[4], ze[4], mu[4];
-  v2 M[4], I[4], D[4];
+  v2 al[F32_K], be[F32_K], de[F32_K], ep[F32_K], ze[F32_K], mu[F32_K];
+  v2 M[F32_K], I[F32_K], D[F32_K];
 };
 
 // One column for both halves, in place. dg* = row above at column x-1, up* = row above at column x.
-__device__ __forceinline__ void f32_column(F32Lane& L, const float4 pA, const float4 pB, const v2 dgM,
-                                           const v2 dgI, const v2 dgD, const v2 upM, const v2 upI) {
-  const float prA[4] = {pA.x, pA.y, pA.z, pA.w};
-  const float prB[4] = {pB.x, pB.y, pB.z, pB.w};
+__device__ __forceinline__ void f32_column(F32Lane& L, const float (&prA)[F32_K], const float (&prB)[F32_K],
+                                           const v2 dgM, const v2 dgI, const v2 dgD, const v2 upM, const v2 upI) {
   // M and D: rows descending so that row u-1's old values are intact when row u reads them
 #pragma unroll
-  for (int u = 3; u >= 0; --u) {
+  for (int u = F32_K - 1; u >= 0; --u) {
     const v2 md = (u == 0) ? dgM : L.M[u - 1];
     const v2 id = (u == 0) ? dgI : L.I[u - 1];
     const v2 dd = (u == 0) ? dgD : L.D[u - 1];
@@ -142,10 +148,10 @@ __device__ __forceinline__ void f32_column(F32Lane& L, const float4 pA, const fl
     const v2 x = fma2(L.al[u], md, mul2(L.be[u], add2(id, dd)));
     L.M[u] = pk(prA[u] * lo(x), prB[u] * hi(x));
   }
-  // I(i,j) = delta*M(i-1,j) + eps*I(i-1,j), rows ascending (a 4-deep FFMA2 chain)
+  // I(i,j) = delta*M(i-1,j) + eps*I(i-1,j), rows ascending (an F32_K-deep FFMA2 chain)
   v2 m_up = upM, i_up = upI;
 #pragma unroll
-  for (int u = 0; u < 4; ++u) {
+  for (int u = 0; u < F32_K; ++u) {
     const v2 ni = fma2(L.ep[u], i_up, mul2(L.de[u], m_up));
     m_up = L.M[u];
     i_up = ni;
@@ -183,17 +189,17 @@ __device__ __forceinline__ const uint32_t* f32_load(const F32Args& A, F32Lane& L
                                                     int copy_len) {
   if (have) {
     const float4* __restrict__ s4 = reinterpret_cast<const float4*>(A.tab + d.tab_blk);
-    float4 cw[6];
+    float4 cw[6 * F32_KC];
 #pragma unroll
-    for (int k = 0; k < 6; ++k) cw[k] = __ldg(s4 + k);
+    for (int k = 0; k < 6 * F32_KC; ++k) cw[k] = __ldg(s4 + k);
 #pragma unroll
-    for (int k = 0; k < 5; ++k) my_tab[k * 32] = __ldg(s4 + 6 + k);  // prior[code][row]
+    for (int k = 0; k < 5 * F32_KC; ++k) my_tab[k * 32] = __ldg(s4 + 6 * F32_KC + k);  // prior[code][chunk]
     const int rrow = (d.flags >> F32_RROW_SHIFT) & 15;
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
+    for (int u = 0; u < F32_K; ++u) {
       auto g = [&](int f) {
-        const float4 v = cw[f];
-        return u == 0 ? v.x : u == 1 ? v.y : u == 2 ? v.z : v.w;
+        const float4 v = cw[f * F32_KC + (u >> 2)];
+        return (u & 3) == 0 ? v.x : (u & 3) == 1 ? v.y : (u & 3) == 2 ? v.z : v.w;
       };
       L.al[u] = set_half<H>(L.al[u], g(0)); L.be[u] = set_half<H>(L.be[u], g(1));
       L.de[u] = set_half<H>(L.de[u], g(2)); L.ep[u] = set_half<H>(L.ep[u], g(3));
@@ -209,7 +215,7 @@ __device__ __forceinline__ const uint32_t* f32_load(const F32Args& A, F32Lane& L
     return reinterpret_cast<const uint32_t*>(A.hcodes + (col0 - 1u - (uint32_t)gi));
   }
 #pragma unroll
-  for (int u = 0; u < 4; ++u) {
+  for (int u = 0; u < F32_K; ++u) {
     L.al[u] = set_half<H>(L.al[u], 0.f); L.be[u] = set_half<H>(L.be[u], 0.f);
     L.de[u] = set_half<H>(L.de[u], 0.f); L.ep[u] = set_half<H>(L.ep[u], 0.f);
     L.ze[u] = set_half<H>(L.ze[u], 0.f); L.mu[u] = set_half<H>(L.mu[u], 0.f);
@@ -237,18 +243,18 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
   const int copy_len = f32_hc_copy_len(ncols);
   F32Lane L;
 #pragma unroll
-  for (int u = 0; u < 4; ++u) {
+  for (int u = 0; u < F32_K; ++u) {
     L.al[u] = L.be[u] = L.de[u] = L.ep[u] = L.ze[u] = L.mu[u] = 0ull;
     L.M[u] = L.I[u] = L.D[u] = 0ull;
   }
   const uint32_t* pA = reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);  // next code word
   const uint32_t* pB = pA;
-  constexpr uint32_t kPadW = 0x0a0a0a0au;  // four PAD codes (byte = code * 2)
+  constexpr uint32_t kPadW = (uint32_t)(F32_PAD * F32_CB) * 0x01010101u;  // four PAD codes
   uint32_t wA = kPadW, wB = kPadW, wA_nx = kPadW, wB_nx = kPadW;
   int outA = -1, outB = -1;
   v2 upM = 0ull, upI = 0ull, upD = 0ull, dgM = 0ull, dgI = 0ull, dgD = 0ull;
-  const uint32_t tabA_s = smem_addr(ptab + lane);                   // [code][lane] float4, half A
-  const uint32_t tabB_s = smem_addr(ptab + F32_NCODE * 32 + lane);  // half B
+  const uint32_t tabA_s = smem_addr(ptab + lane);                            // [code][chunk][lane] float4
+  const uint32_t tabB_s = smem_addr(ptab + F32_NCODE * F32_KC * 32 + lane);  // half B
   const uint32_t ring_s = smem_addr(ring);
   const int src = (lane + 31) & 31;
   const bool is0 = lane == 0, is31 = lane == 31;
@@ -264,16 +270,22 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
 
   auto step = [&](const int r) {
     if (is31) ring_get3(ring_s + 16u * (uint32_t)(c0 + 2), rvM, rvI, rvD);
-    // code byte r (= code*2) placed in byte 1 -> code*512 = the code's row in the table
+    // code byte r (= code*F32_CB) placed in byte 1 -> the code's rows in the table
     const uint32_t oA = __byte_perm(wA, 0, 0x4404 + (r << 4)), oB = __byte_perm(wB, 0, 0x4404 + (r << 4));
-    float4 prA, prB;
-    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(prA.x), "=f"(prA.y), "=f"(prA.z), "=f"(prA.w)
-                 : "r"(tabA_s + oA));
-    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(prB.x), "=f"(prB.y), "=f"(prB.z), "=f"(prB.w)
-                 : "r"(tabB_s + oB));
+    float prA[F32_K], prB[F32_K];
+#pragma unroll
+    for (int ch = 0; ch < F32_KC; ++ch) {
+      asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                   : "=f"(prA[4 * ch]), "=f"(prA[4 * ch + 1]), "=f"(prA[4 * ch + 2]), "=f"(prA[4 * ch + 3])
+                   : "r"(tabA_s + oA + 512u * ch));
+      asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                   : "=f"(prB[4 * ch]), "=f"(prB[4 * ch + 1]), "=f"(prB[4 * ch + 2]), "=f"(prB[4 * ch + 3])
+                   : "r"(tabB_s + oB + 512u * ch));
+    }
     f32_column(L, prA, prB, dgM, dgI, dgD, upM, upI);
-    const float m3a = lo(L.M[3]), i3a = lo(L.I[3]), d3a = lo(L.D[3]);
-    const float m3b = hi(L.M[3]), i3b = hi(L.I[3]), d3b = hi(L.D[3]);
+    constexpr int LR = F32_K - 1;  // last row of a block
+    const float m3a = lo(L.M[LR]), i3a = lo(L.I[LR]), d3a = lo(L.D[LR]);
+    const float m3b = hi(L.M[LR]), i3b = hi(L.I[LR]), d3b = hi(L.D[LR]);
     // half B of lane-1 -> half A of lane; lane 31 sends the ring slot instead (virtual 63 -> 0)
     const float sM = is31 ? rvM : m3b;
     const float sI = is31 ? rvI : i3b;
@@ -289,8 +301,8 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
 #ifdef PHMM_DBG_TRACE
     if (trace && tstep < 4096) {
       float* t = g_trace + ((size_t)tstep * 32 + lane) * 6;
-      t[0] = lo(L.M[3]); t[1] = lo(L.I[3]); t[2] = lo(L.D[3]);
-      t[3] = hi(L.M[3]); t[4] = hi(L.I[3]); t[5] = hi(L.D[3]);
+      t[0] = lo(L.M[F32_K - 1]); t[1] = lo(L.I[F32_K - 1]); t[2] = lo(L.D[F32_K - 1]);
+      t[3] = hi(L.M[F32_K - 1]); t[4] = hi(L.I[F32_K - 1]); t[5] = hi(L.D[F32_K - 1]);
       if (lane == 0) g_trace_steps = tstep + 1;
     }
     ++tstep;
@@ -322,10 +334,10 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
           if (hB) dB = A.blk[s + bB];
         }
 
-        if (outA >= 0) A.out[outA] = lo(L.D[3]);  // S2 row: the last-row M+I sum (L20@2262)
-        if (outB >= 0) A.out[outB] = hi(L.D[3]);
+        if (outA >= 0) A.out[outA] = lo(L.D[F32_K - 1]);  // S2 row: the last-row M+I sum (L20@2262)
+        if (outB >= 0) A.out[outB] = hi(L.D[F32_K - 1]);
         pA = f32_load<0>(A, L, ptab + lane, hA, dA, d0, outA, giA, copy_len);
-        pB = f32_load<1>(A, L, ptab + F32_NCODE * 32 + lane, hB, dB, d0, outB, giB, copy_len);
+        pB = f32_load<1>(A, L, ptab + F32_NCODE * F32_KC * 32 + lane, hB, dB, d0, outB, giB, copy_len);
         wA_nx = __ldg(pA); ++pA;
         wB_nx = __ldg(pB); ++pB;
         // prefetch after this pass's loads are issued (a load issued before the
@@ -354,17 +366,18 @@ cudaError_t wf32_launch(unsigned grid, size_t smem, cudaStream_t stream, const F
 
 #ifdef PHMM_DEFINE_WF32
 #ifndef PHMM_F32_MINB
-#define PHMM_F32_MINB 3  // CTAs (of 4 warps) per SM the register budget must allow (168 regs)
+#define PHMM_F32_MINB 2  // CTAs (of 4 warps) per SM the register budget must allow (255 regs)
 #endif
 __global__ void __launch_bounds__(F32_WARPS * 32, PHMM_F32_MINB) k_wavefront_f32(F32Args A) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
-  // per warp: prior tables [2 halves][6 codes][32 lanes] float4 (6 KB), then the ring
-  const int per_warp = 2 * F32_NCODE * 32 + A.ring_len;
+  // per warp: prior tables [2 halves][6 codes][F32_KC chunks][32 lanes] float4, then the ring
+  constexpr int kTab = 2 * F32_NCODE * F32_KC * 32;
+  const int per_warp = kTab + A.ring_len;
   float4* ptab = reinterpret_cast<float4*>(smem_raw) + (size_t)wib * per_warp;
-  float4* ring = ptab + 2 * F32_NCODE * 32;
-  for (int i = lane; i < 2 * F32_NCODE * 32; i += 32) ptab[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+  float4* ring = ptab + kTab;
+  for (int i = lane; i < kTab; i += 32) ptab[i] = make_float4(0.f, 0.f, 0.f, 0.f);
   for (int i = lane; i < 4 * A.ring_len; i += 32) reinterpret_cast<float*>(ring)[i] = 0.f;
   __syncwarp();
   const unsigned long long n_items = A.item_start[A.nbins];
