@@ -178,7 +178,7 @@ __device__ __forceinline__ uint32_t smem_addr(const void* p) {
 // float4 index of that code's entry in a lane's prior table.
 __host__ __device__ inline int f32_hc_copy_len(int ncols) {
   const int p = (ncols + F32_G > F32_MIN_P) ? ncols + F32_G : F32_MIN_P;
-  return ((int)F32_HC_FRONT + p + 16 + 3) & ~3;
+  return ((int)F32_HC_FRONT + p + 24 + 3) & ~3;  // + prefetch distance
 }
 
 // Load a block (or nothing) into half H of a lane. Returns the 32-bit-aligned code
@@ -250,7 +250,8 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
   const uint32_t* pA = reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);  // next code word
   const uint32_t* pB = pA;
   constexpr uint32_t kPadW = (uint32_t)(F32_PAD * F32_CB) * 0x01010101u;  // four PAD codes
-  uint32_t wA = kPadW, wB = kPadW, wA_nx = kPadW, wB_nx = kPadW;
+  // code words: current group, next group, the one after (prefetch distance 2 groups)
+  uint32_t wA = kPadW, wB = kPadW, wA_nx = kPadW, wB_nx = kPadW, wA_nx2 = kPadW, wB_nx2 = kPadW;
   int outA = -1, outB = -1;
   v2 upM = 0ull, upI = 0ull, upD = 0ull, dgM = 0ull, dgI = 0ull, dgD = 0ull;
   const uint32_t tabA_s = smem_addr(ptab + lane);                            // [code][chunk][lane] float4
@@ -313,7 +314,8 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
   // 4 steps sharing one code word per half; the next words are prefetched
   auto group4 = [&]() {
     wA = wA_nx; wB = wB_nx;
-    wA_nx = __ldg(pA); wB_nx = __ldg(pB);
+    wA_nx = wA_nx2; wB_nx = wB_nx2;
+    wA_nx2 = __ldg(pA); wB_nx2 = __ldg(pB);
     ++pA; ++pB;
     step(0); step(1); step(2); step(3);
   };
@@ -338,8 +340,8 @@ __device__ __forceinline__ void f32_stream(const F32Args& A, float4* __restrict_
         if (outB >= 0) A.out[outB] = hi(L.D[F32_K - 1]);
         pA = f32_load<0>(A, L, ptab + lane, hA, dA, d0, outA, giA, copy_len);
         pB = f32_load<1>(A, L, ptab + F32_NCODE * F32_KC * 32 + lane, hB, dB, d0, outB, giB, copy_len);
-        wA_nx = __ldg(pA); ++pA;
-        wB_nx = __ldg(pB); ++pB;
+        wA_nx = __ldg(pA); wA_nx2 = __ldg(pA + 1); pA += 2;
+        wB_nx = __ldg(pB); wB_nx2 = __ldg(pB + 1); pB += 2;
         // prefetch after this pass's loads are issued (a load issued before the
         // consumers of the previous prefetch would share their scoreboard)
         if (bA + 64 < nblk) dnA = A.blk[s + bA + 64];
