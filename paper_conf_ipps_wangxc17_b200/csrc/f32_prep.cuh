@@ -27,24 +27,31 @@ __global__ void k_hap_codes_f32(const uint8_t* __restrict__ hap, const int64_t* 
     const int64_t h0 = hoff[h];
     const int n = (int)(hoff[h + 1] - h0);
     if (n < 1 || n > kMaxHapLen) continue;
-    const int len = f32_hc_copy_len(ncols_of(n, bucket));
-    uint8_t* dst = codes + hc_off[h];
-    for (int i = lane; i < 4 * len; i += 32) {
-      const int k = i / len;
-      const int c = (i % len) - (int)F32_HC_FRONT - k;  // column of this byte in copy k
-      uint8_t v = F32_PAD;
-      if (c >= 0 && c < n) {
-        switch (hap[h0 + c]) {
-          case 'A': v = 0; break;
-          case 'C': v = 1; break;
-          case 'G': v = 2; break;
-          case 'T': v = 3; break;
-          default: v = 4; break;  // 'N' (invalid bytes were rejected by validation)
+    const int len = f32_hc_copy_len(ncols_of(n, bucket));  // multiple of 4, region start 4-aligned
+    uint32_t* dst = reinterpret_cast<uint32_t*>(codes + hc_off[h]);
+    const int wpc = len >> 2;  // words per copy
+    for (int k = 0; k < 4; ++k) {
+      for (int w = lane; w < wpc; w += 32) {
+        uint32_t word = 0;
+#pragma unroll
+        for (int by = 0; by < 4; ++by) {
+          const int c = 4 * w + by - (int)F32_HC_FRONT - k;  // column of this byte in copy k
+          uint32_t v = F32_PAD;
+          if (c >= 0 && c < n) {
+            switch (hap[h0 + c]) {
+              case 'A': v = 0; break;
+              case 'C': v = 1; break;
+              case 'G': v = 2; break;
+              case 'T': v = 3; break;
+              default: v = 4; break;  // 'N' (invalid bytes were rejected by validation)
+            }
+          } else if (c == n) {
+            v = 4;
+          }
+          word |= (v * F32_CB) << (8 * by);
         }
-      } else if (c == n) {
-        v = 4;
+        dst[k * wpc + w] = word;
       }
-      dst[i] = (uint8_t)(v * F32_CB);
     }
   }
 }
@@ -57,30 +64,30 @@ __global__ void k_hap_ncols(const int64_t* __restrict__ hoff, int64_t n_haps, in
   if (blockIdx.x == 0 && threadIdx.x == 0) nc[n_haps] = 0;
 }
 
-// per-read FP32 tables: one thread per 4-row block (binary search of its read once
-// per block), the 176-byte block written as 11 float4 stores
-__global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ item_tab_off,
-                                  const int64_t* __restrict__ total_tab_blocks_dev, const int64_t* __restrict__ roff,
-                                  const uint8_t* __restrict__ rb, const uint8_t* __restrict__ q,
-                                  const uint8_t* __restrict__ qi, const uint8_t* __restrict__ qd,
-                                  const uint8_t* __restrict__ qg, F32Block* __restrict__ tab) {
+// per-read FP32 tables: one warp per read, lanes over its padded rows; Phred -> error
+// probabilities from a 128-entry table built once per CUDA block (10^(-q/10) in double,
+// rounded to float -- the same values qual_err<float> gives)
+constexpr int kTabThreads = 256;
+__global__ void __launch_bounds__(kTabThreads) k_build_table_f32(
+    int64_t n_reads, const int64_t* __restrict__ item_tab_off, const int64_t* __restrict__ total_tab_blocks_dev,
+    const int64_t* __restrict__ roff, const uint8_t* __restrict__ rb, const uint8_t* __restrict__ q,
+    const uint8_t* __restrict__ qi, const uint8_t* __restrict__ qd, const uint8_t* __restrict__ qg,
+    F32Block* __restrict__ tab) {
   constexpr int K = F32_K;
-  const int64_t total = *total_tab_blocks_dev;
-  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < total; b += (int64_t)gridDim.x * blockDim.x) {
-    int64_t lo = 0, hi = n_reads - 1;
-    while (lo < hi) {
-      const int64_t mid = (lo + hi + 1) >> 1;
-      if (item_tab_off[mid] <= b) lo = mid; else hi = mid - 1;
-    }
-    const int64_t r = lo;
+  __shared__ float err[128];
+  for (int i = threadIdx.x; i < 128; i += blockDim.x) err[i] = qual_err<float>((uint32_t)i);
+  __syncthreads();
+  (void)total_tab_blocks_dev;
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; r < n_reads; r += nwarps) {
     const int64_t r0 = roff[r];
     const int m = (int)(roff[r + 1] - r0);
+    if (m < 1) continue;
     const int nb = nblocks_of<K>(m);
     const int f = nb * K - (m + 3);
-    float co[6][F32_K], pr[5][F32_K];
-#pragma unroll
-    for (int t = 0; t < K; ++t) {
-      const int row = (int)(b - item_tab_off[r]) * K + t;
+    F32Block* __restrict__ T = tab + item_tab_off[r];
+    for (int row = lane; row < nb * K; row += 32) {
       float al = 0, be = 0, de = 0, ep = 0, ze = 0, mu = 0;
       float p5[5] = {0, 0, 0, 0, 0};
       if (row < f) {
@@ -89,8 +96,7 @@ __global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ i
         mu = 1;
       } else if (row <= f + m) {
         const int64_t x = r0 + (row - f - 1);
-        const float ei = qual_err<float>(qi[x]), ed = qual_err<float>(qd[x]), eg = qual_err<float>(qg[x]),
-                    eb = qual_err<float>(q[x]);
+        const float ei = err[qi[x] & 127], ed = err[qd[x] & 127], eg = err[qg[x] & 127], eb = err[q[x] & 127];
         const float sum = ei + ed;
         al = 1.f - (sum < 1.f ? sum : 1.f);
         be = 1.f - eg;
@@ -111,22 +117,13 @@ __global__ void k_build_table_f32(int64_t n_reads, const int64_t* __restrict__ i
         be = 1; ze = 1; mu = 1;
         p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = 1;
       }
-      co[0][t] = al; co[1][t] = be; co[2][t] = de; co[3][t] = ep; co[4][t] = ze; co[5][t] = mu;
+      F32Block& B = T[row / K];
+      const int t = row % K;
+      B.coef[0][t] = al; B.coef[1][t] = be; B.coef[2][t] = de;
+      B.coef[3][t] = ep; B.coef[4][t] = ze; B.coef[5][t] = mu;
 #pragma unroll
-      for (int k = 0; k < 5; ++k) pr[k][t] = p5[k];
+      for (int k = 0; k < 5; ++k) B.prior[k][t] = p5[k];
     }
-    float4* dst = reinterpret_cast<float4*>(tab + b);
-#pragma unroll
-    for (int k = 0; k < 6; ++k)
-#pragma unroll
-      for (int ch = 0; ch < F32_KC; ++ch)
-        dst[k * F32_KC + ch] = make_float4(co[k][4 * ch], co[k][4 * ch + 1], co[k][4 * ch + 2], co[k][4 * ch + 3]);
-#pragma unroll
-    for (int k = 0; k < 5; ++k)
-#pragma unroll
-      for (int ch = 0; ch < F32_KC; ++ch)
-        dst[6 * F32_KC + k * F32_KC + ch] =
-            make_float4(pr[k][4 * ch], pr[k][4 * ch + 1], pr[k][4 * ch + 2], pr[k][4 * ch + 3]);
   }
 }
 

@@ -386,7 +386,7 @@ phmm_status pass_run_f32(phmm_ctx* c, const DevBatch& d, const PassInfo& pi, int
   ST_TRY(ws(c, B_HCODES32, (size_t)(total_hc + pad_len), &hc));
   CUDA_TRY(cudaMemsetAsync(hc + total_hc, F32_PAD * F32_CB, (size_t)pad_len, s));
   if (total_tab > 0) {
-    k_build_table_f32<<<grid_for(c, total_tab), kThreads, 0, s>>>(
+    k_build_table_f32<<<grid_for(c, d.n_reads * 32), kTabThreads, 0, s>>>(
         d.n_reads, item_off, item_off + d.n_reads, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
     LAUNCHED(c);
   }
