@@ -324,7 +324,7 @@ def main():
     sm_run = clocks.get("sm_mhz") if clocks else None
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak_gcups, "unit": "GCUPS",
                 "frac": (achieved / peak_gcups) if achieved else None, "traffic": None,
-                "kernel": "k_wavefront<float,8>",
+                "kernel": "k_wavefront<float>",
                 "peak_basis": f"{nsm} SM x {FP32_LANES_PER_SM} FP32 lanes x {sm_max:.0f} MHz (MEASURED_PEAKS sm_max_mhz)"
                               f" / {FP32_OPS_PER_CELL} FP32-pipe ops per cell (3 FFMA + 4 FMUL + 1 FADD)",
                 "frac_at_run_clock": (achieved / (peak_gcups * sm_run / sm_max)) if (achieved and sm_run) else None,

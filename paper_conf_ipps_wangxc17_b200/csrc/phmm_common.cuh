@@ -59,15 +59,6 @@ __device__ __forceinline__ uint32_t base_code(uint8_t b) {
   }
 }
 
-template <typename T> struct Prec;
-template <> struct Prec<float> { static constexpr int kScaleExp = 120; };
-template <> struct Prec<double> { static constexpr int kScaleExp = 1020; };
-
-// mask bits of a table row
-constexpr uint32_t MASK_BASE = 15u;
-constexpr uint32_t MASK_D0 = 16u;          // row boundary D(i,0) = s/N (the R row)
-constexpr uint32_t MASK_ABOVE_IS_R = 32u;  // (row 0 of a block) the row above is an R row
-
 // Per-block descriptor in the bin-sorted block sequence (16 bytes).
 struct BlkDesc {
   uint32_t tab_blk;   // block index in the coefficient table
@@ -78,18 +69,6 @@ struct BlkDesc {
 };
 static_assert(sizeof(BlkDesc) == 16, "BlkDesc must be 16 bytes");
 constexpr uint16_t BLK_LAST = 1, BLK_FIRST = 2;
-
-// bytes of one table block: 8 coefficient fields x K values of T, then K masks
-template <typename T, int K>
-struct alignas(16) TabBlock {
-  T coef[8][K];  // alpha, beta, delta, eps, zeta, mu, pm, px
-  uint32_t mask[K];
-};
-
-template <typename T>
-struct alignas(16) RingEnt {
-  T m, i, d, pad;
-};
 
 __host__ __device__ constexpr int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 

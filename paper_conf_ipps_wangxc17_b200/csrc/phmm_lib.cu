@@ -18,7 +18,7 @@
 
 #include "../../include/phmm.h"
 #include "phmm_device.cuh"
-#include "f32_prep.cuh"
+#include "stream_prep.cuh"
 
 using namespace phmm;
 
@@ -28,8 +28,8 @@ enum BufId {
   B_READ_BASES, B_BQ, B_IQ, B_DQ, B_GQ, B_ROFF, B_HAP, B_HOFF, B_PAIRS,  // host-variant inputs
   B_HCODES, B_SCAL,                                                       // codes, scalars
   B_PAIR_BIN, B_PAIR_NB, B_BINS, B_ITEM_NB, B_ITEM_OFF, B_SCAN_TMP,
-  B_TAB, B_BLK, B_OUT32, B_OUT64, B_RLIST, B_ITEM_READ, B_PAIR_ITEM,
-  B_OUT_LOG10, B_OUT_STATUS, B_HNC, B_HC_OFF, B_HCODES32, B_TAB32,
+  B_TAB32, B_TAB64, B_BLK, B_OUT32, B_OUT64, B_RLIST, B_ITEM_READ, B_PAIR_ITEM,
+  B_OUT_LOG10, B_OUT_STATUS, B_HNC, B_HC_OFF,
   B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_COUNT
 };
 
@@ -47,16 +47,11 @@ struct Scalars {
   unsigned long long total_blocks;
   int64_t n_rescue;
   unsigned long long n_underflow;
-  unsigned int item_counter;
-  unsigned int pad_;
+  unsigned int item_counter[2];  // work-item counters of the (at most 2) wavefront launches
 };
 
 constexpr int kEvents = 10;
 constexpr int kThreads = 256;
-constexpr int kWarpsPerBlock = 4;
-
-// haplotype code padding: columns past N read (finite, unused) codes
-constexpr int64_t kHapPad = 4224;
 
 }  // namespace
 
@@ -69,7 +64,9 @@ struct phmm_ctx {
   int bucket = 4;
   int nsm = 148;
   Buf buf[B_COUNT];
+  int smem_per_sm = 0, smem_reserved = 0, smem_optin = 0;  // bytes (device attributes)
   Scalars* host_scal = nullptr;  // pinned
+  int64_t* host_sizes = nullptr;  // pinned, 2 values
   cudaEvent_t ev[kEvents] = {};
   phmm_stats st{};
   int launches = 0;
@@ -178,17 +175,14 @@ struct PassInfo {
   int max_ncols = 0;
 };
 
-// Validation of the whole batch + haplotype one-hot codes. Errors land in scal->err.
-phmm_status run_validate(phmm_ctx* c, const DevBatch& d, uint8_t** hcodes_out) {
+// Validation of the whole batch. Errors land in scal->err (read back by pass_prepare).
+phmm_status run_validate(phmm_ctx* c, const DevBatch& d) {
   cudaStream_t s = c->stream;
   Scalars* scal;
-  uint8_t* hcodes;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
-  ST_TRY(ws(c, B_HCODES, (size_t)(d.n_hb + kHapPad), &hcodes));
   CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
-  CUDA_TRY(cudaMemsetAsync(hcodes + d.n_hb, 0, kHapPad, s));
   if (d.n_hb > 0) {
-    k_hap_codes<<<grid_for(c, d.n_hb), kThreads, 0, s>>>(d.hap, d.n_hb, hcodes, &scal->err);
+    k_validate_haps<<<grid_for(c, d.n_hb), kThreads, 0, s>>>(d.hap, d.n_hb, &scal->err);
     LAUNCHED(c);
   }
   if (d.n_rb > 0) {
@@ -199,24 +193,24 @@ phmm_status run_validate(phmm_ctx* c, const DevBatch& d, uint8_t** hcodes_out) {
   LAUNCHED(c);
   k_validate_offsets<<<grid_for(c, d.n_haps + 1), kThreads, 0, s>>>(d.hoff, d.n_haps, d.n_hb, &scal->err);
   LAUNCHED(c);
-  *hcodes_out = hcodes;
   return PHMM_OK;
 }
 
-// Part 1 of a pass: bin the pairs, size the table. Ends with one D2H + sync
-// (sizes for the allocations; input-content errors are reported here, before
-// any output is written).
+// Part 1 of a pass: bin the pairs, size the coefficient table (and, with
+// total_hcodes_out, the haplotype code regions). Ends with one D2H + sync (sizes for
+// the allocations; input-content errors are reported here, before any output is written).
 //   list == nullptr: all pairs, table items = reads, output slot = pair id
 //   list != nullptr: the n listed pairs, one table item per listed pair,
 //                    output slot = position in the list
-template <typename T, int K>
+template <typename T>
 phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_t n, PassInfo* pi,
                          int64_t* total_tab_out, int64_t* total_hcodes_out = nullptr) {
+  constexpr int K = WfT<T>::K;
   cudaStream_t s = c->stream;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   const int nb1 = kMaxBins + 2;
-  unsigned long long* bins;  // [blocks | pairs | cursor | start | item_start], nb1 each
+  unsigned long long* bins;  // [blocks | pairs | - | start | item_start], nb1 each
   ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
   int32_t *pair_bin, *pair_nb;
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
@@ -224,7 +218,6 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   CUDA_TRY(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * 3 * nb1, s));
   // per-pass scalars (err is kept: it accumulates validation errors)
   CUDA_TRY(cudaMemsetAsync(&scal->max_ncols, 0, offsetof(Scalars, n_rescue) - offsetof(Scalars, max_ncols), s));
-  CUDA_TRY(cudaMemsetAsync(&scal->item_counter, 0, sizeof(unsigned int), s));
 
   k_pair_bins<K><<<grid_for(c, n), kThreads, 0, s>>>(
       d.pairs, list, nullptr, n, d.roff, d.n_reads, d.hoff, d.n_haps, c->bucket, pair_bin, pair_nb, bins,
@@ -248,54 +241,74 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   LAUNCHED(c);
   size_t tmp_bytes = 0;
   CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, item_nb, item_off, (int64_t)(n_items + 1), s));
-  unsigned char* tmp;
-  ST_TRY(ws(c, B_SCAN_TMP, tmp_bytes, &tmp));
-  CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, item_nb, item_off, (int64_t)(n_items + 1), s));
-  ++c->launches;
-
-  // FP32 kernel: per-haplotype padded code arrays (ncols codes each)
-  int64_t* hc_off = nullptr;
+  size_t tb2 = 0;
+  int64_t *hnc = nullptr, *hc_off = nullptr;
   if (total_hcodes_out) {
-    int64_t* hnc;
     ST_TRY(ws(c, B_HNC, (size_t)d.n_haps + 1, &hnc));
     ST_TRY(ws(c, B_HC_OFF, (size_t)d.n_haps + 1, &hc_off));
+    CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, hnc, hc_off, (int64_t)(d.n_haps + 1), s));
+  }
+  unsigned char* tmp;
+  ST_TRY(ws(c, B_SCAN_TMP, std::max(tmp_bytes, tb2), &tmp));
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, item_nb, item_off, (int64_t)(n_items + 1), s));
+  ++c->launches;
+  // haplotype code regions (wf_hc_region bytes each)
+  if (total_hcodes_out) {
     k_hap_ncols<<<grid_for(c, d.n_haps), kThreads, 0, s>>>(d.hoff, d.n_haps, c->bucket, hnc);
     LAUNCHED(c);
-    size_t tb2 = 0;
-    CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, tb2, hnc, hc_off, (int64_t)(d.n_haps + 1), s));
-    unsigned char* tmp2;
-    ST_TRY(ws(c, B_SCAN_TMP, std::max(tb2, tmp_bytes), &tmp2));
-    CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp2, tb2, hnc, hc_off, (int64_t)(d.n_haps + 1), s));
+    CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, tb2, hnc, hc_off, (int64_t)(d.n_haps + 1), s));
     ++c->launches;
   }
   // one small D2H: sizes + error flag
   CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
-  int64_t total_tab = 0, total_hc = 0;
-  CUDA_TRY(cudaMemcpyAsync(&total_tab, item_off + n_items, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-  if (hc_off) CUDA_TRY(cudaMemcpyAsync(&total_hc, hc_off + d.n_haps, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  int64_t* hsz = c->host_sizes;
+  hsz[0] = hsz[1] = 0;
+  CUDA_TRY(cudaMemcpyAsync(&hsz[0], item_off + n_items, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  if (hc_off) CUDA_TRY(cudaMemcpyAsync(&hsz[1], hc_off + d.n_haps, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaStreamSynchronize(s));
-  if (total_hcodes_out) *total_hcodes_out = total_hc;
   if (c->host_scal->err) return map_err(c->host_scal->err);
+  if (total_hcodes_out) *total_hcodes_out = hsz[1];
   pi->cells = c->host_scal->cells;
   pi->padded_cells = c->host_scal->padded_cells;
   pi->total_blocks = c->host_scal->total_blocks;
   pi->max_ncols = c->host_scal->max_ncols;
-  *total_tab_out = total_tab;
+  // block descriptors address tables and code regions with 32-bit offsets
+  if (hsz[0] > 0xffffffffLL || pi->total_blocks > 0x7fffffffULL) return PHMM_E_INVALID_ARG;
+  *total_tab_out = hsz[0];
   return PHMM_OK;
 }
 
-// Part 2 of a pass: tables, block sequence, wavefront. Writes out[slot] = scaled sum.
-template <typename T, int K>
-phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const uint8_t* hcodes, const int32_t* list, int64_t n,
-                     const PassInfo& pi, int64_t total_tab, T* out, int* nbins_used) {
+// Haplotype code regions of the whole batch (after pass_prepare with total_hcodes_out),
+// followed by an all-PAD region for idle lanes. Returns the buffer and the PAD offset.
+phmm_status build_hap_codes(phmm_ctx* c, const DevBatch& d, int64_t total_hc, int max_ncols, uint8_t** hc_out) {
+  cudaStream_t s = c->stream;
+  const int64_t pad_len = wf_hc_copy_len(max_ncols) + 64;
+  if (total_hc + pad_len > 0xffffffffLL) return PHMM_E_INVALID_ARG;  // 32-bit code offsets
+  int64_t* hc_off;
+  uint8_t* hc;
+  ST_TRY(ws(c, B_HC_OFF, (size_t)d.n_haps + 1, &hc_off));
+  ST_TRY(ws(c, B_HCODES, (size_t)(total_hc + pad_len), &hc));
+  CUDA_TRY(cudaMemsetAsync(hc + total_hc, WF_PAD * WF_CB, (size_t)pad_len, s));
+  k_hap_codes_wf<<<grid_for(c, d.n_haps * 32), kThreads, 0, s>>>(d.hap, d.hoff, d.n_haps, hc_off, c->bucket, hc);
+  LAUNCHED(c);
+  *hc_out = hc;
+  return PHMM_OK;
+}
+
+// Part 2 of a pass: coefficient tables, stable bin sort, block descriptors, wavefront.
+// Writes out[slot] = scaled sum of the pair. The haplotype code regions
+// (hc, pad region at total_hc) were built by build_hap_codes.
+template <typename T>
+phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_t n, const PassInfo& pi,
+                     int64_t total_tab, const uint8_t* hc, int64_t total_hc, T* out, bool timed) {
+  constexpr int K = WfT<T>::K;
   cudaStream_t s = c->stream;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   const int nb1 = kMaxBins + 2;
   unsigned long long* bins;
   ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
-  unsigned long long *bin_blocks = bins, *bin_cursor = bins + 2 * nb1, *bin_start = bins + 3 * nb1,
-                     *item_start = bins + 4 * nb1;
+  unsigned long long *bin_blocks = bins, *bin_start = bins + 3 * nb1, *item_start = bins + 4 * nb1;
   int32_t *pair_bin, *pair_nb, *item_read = nullptr, *pair_item = nullptr;
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
   ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
@@ -304,158 +317,107 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const uint8_t* hcodes, cons
     ST_TRY(ws(c, B_ITEM_READ, (size_t)n, &item_read));
     ST_TRY(ws(c, B_PAIR_ITEM, (size_t)n, &pair_item));
   }
-  int64_t* item_off;
-  ST_TRY(ws(c, B_ITEM_OFF, (size_t)n_items + 1, &item_off));
-  TabBlock<T, K>* tab;
-  BlkDesc* blk;
-  ST_TRY(ws(c, B_TAB, (size_t)total_tab, &tab));
-  ST_TRY(ws(c, B_BLK, (size_t)pi.total_blocks, &blk));
-
-  // per-read (or per-rescued-pair) coefficient tables
-  if (total_tab > 0) {
-    k_build_table<T, K><<<grid_for(c, total_tab * K), kThreads, 0, s>>>(
-        item_read, nullptr, n_items, item_off, item_off + n_items, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
-    LAUNCHED(c);
-  }
-
-  // warps and work-item size
-  const size_t ring_bytes = (size_t)pi.max_ncols * sizeof(RingEnt<T>);
-  const size_t smem = ring_bytes * kWarpsPerBlock;
-  CUDA_TRY(cudaFuncSetAttribute(k_wavefront<T, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  int bps = 0;
-  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_wavefront<T, K>, kWarpsPerBlock * 32, smem));
-  if (bps < 1) return PHMM_E_INVALID_ARG;  // haplotype too long for the shared-memory ring
-  const int64_t nwarps = (int64_t)c->nsm * bps * kWarpsPerBlock;
-  int64_t chunk = (int64_t)(pi.total_blocks / (unsigned long long)(nwarps * 6));
-  if (chunk < 128) chunk = 128;
-  if (chunk > 16384) chunk = 16384;
-
-  const int nbins = kMaxBins + 1;
-  k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, chunk, bin_start, item_start);
-  LAUNCHED(c);
-  k_alloc_blocks<K><<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, nullptr, n, pair_bin, pair_nb, bin_start,
-                                                        bin_cursor, d.hoff, item_off, pair_item, list ? 1 : 0, blk);
-  LAUNCHED(c);
-
-  WfArgs<T> A;
-  A.blk = blk;
-  A.tab = tab;
-  A.hcodes = hcodes;
-  A.bin_start = bin_start;
-  A.item_start = item_start;
-  A.nbins = nbins;
-  A.bucket = c->bucket;
-  A.chunk_blocks = chunk;
-  A.item_counter = &scal->item_counter;
-  A.out = out;
-  A.ring_len = pi.max_ncols;
-  CUDA_TRY(cudaMemsetAsync(&scal->item_counter, 0, sizeof(unsigned int), s));
-  const bool timing_wf = (sizeof(T) == 4 || c->prec == PHMM_PREC_FP64);
-  if (timing_wf) ev_record(c, EV_WF0);
-  k_wavefront<T, K><<<(unsigned)(c->nsm * bps), kWarpsPerBlock * 32, smem, s>>>(A);
-  LAUNCHED(c);
-  if (timing_wf) ev_record(c, EV_WF1);
-  if (nbins_used) *nbins_used = 0;
-  return PHMM_OK;
-}
-
-// FP32 pass over all pairs with k_wavefront_f32 (after pass_prepare<float, F32_K>).
-phmm_status pass_run_f32(phmm_ctx* c, const DevBatch& d, const PassInfo& pi, int64_t total_tab, int64_t total_hc,
-                         float* out) {
-  cudaStream_t s = c->stream;
-  Scalars* scal;
-  ST_TRY(ws(c, B_SCAL, 1, &scal));
-  const int nb1 = kMaxBins + 2;
-  unsigned long long* bins;
-  ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
-  unsigned long long *bin_blocks = bins, *bin_cursor = bins + 2 * nb1, *bin_start = bins + 3 * nb1,
-                     *item_start = bins + 4 * nb1;
-  int32_t *pair_bin, *pair_nb;
-  ST_TRY(ws(c, B_PAIR_BIN, (size_t)d.n_pairs, &pair_bin));
-  ST_TRY(ws(c, B_PAIR_NB, (size_t)d.n_pairs, &pair_nb));
   int64_t *item_off, *hc_off;
-  ST_TRY(ws(c, B_ITEM_OFF, (size_t)d.n_reads + 1, &item_off));
+  ST_TRY(ws(c, B_ITEM_OFF, (size_t)n_items + 1, &item_off));
   ST_TRY(ws(c, B_HC_OFF, (size_t)d.n_haps + 1, &hc_off));
-  const int p_max = std::max(pi.max_ncols + F32_G, F32_MIN_P);
-  const int64_t pad_len = p_max + 256;
-  F32Block* tab;
+  TBlock<T>* tab;
   BlkDesc* blk;
-  uint8_t* hc;
-  ST_TRY(ws(c, B_TAB32, (size_t)total_tab, &tab));
+  ST_TRY(ws(c, sizeof(T) == 4 ? B_TAB32 : B_TAB64, (size_t)total_tab, &tab));
   ST_TRY(ws(c, B_BLK, (size_t)pi.total_blocks, &blk));
-  ST_TRY(ws(c, B_HCODES32, (size_t)(total_hc + pad_len), &hc));
-  CUDA_TRY(cudaMemsetAsync(hc + total_hc, F32_PAD * F32_CB, (size_t)pad_len, s));
   if (total_tab > 0) {
-    k_build_table_f32<<<grid_for(c, d.n_reads * 32), kTabThreads, 0, s>>>(
-        d.n_reads, item_off, item_off + d.n_reads, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
+    k_build_table_wf<T><<<grid_for(c, n_items * 32), kTabThreads, 0, s>>>(
+        item_read, n_items, item_off, d.roff, d.rb, d.q, d.qi, d.qd, d.qg, tab);
     LAUNCHED(c);
   }
-  k_hap_codes_f32<<<grid_for(c, d.n_haps * 32), kThreads, 0, s>>>(d.hap, d.hoff, d.n_haps, hc_off, c->bucket, hc);
-  LAUNCHED(c);
 
-  const int ring_len = p_max + 4;
-  const size_t smem = (size_t)F32_WARPS * (2 * F32_NCODE * F32_KC * 32 + ring_len) * sizeof(float4);
-  int bps = 0;
-  CUDA_TRY(wf32_occupancy(smem, &bps));
-  if (bps < 1) return PHMM_E_INVALID_ARG;
-  const int64_t nwarps = (int64_t)c->nsm * bps * F32_WARPS;
+  // launch classes: bins whose ring fits at full occupancy, then (if any) the longer bins
+  const int slot = (int)ring_slot_bytes<T>();
+  auto P_of = [](int ncols) { return std::max(ncols + WF_G, WF_MIN_P); };
+  const int p_max = P_of(pi.max_ncols);
+  int bps_full = 0;
+  CUDA_TRY(wf_occupancy<T>(WF_WARPS, wf_warp_smem<T>(WF_MIN_P + 4) * WF_WARPS, &bps_full));
+  if (bps_full < 1) return PHMM_E_CUDA;
+  const int64_t cta_budget = (int64_t)c->smem_per_sm / bps_full - c->smem_reserved;
+  const int ring_full = (int)std::min<int64_t>(
+      (cta_budget / WF_WARPS - (int64_t)wf_warp_smem<T>(0)) / slot, (int64_t)(c->smem_optin / WF_WARPS) / slot);
+  int bin_cut = kMaxBins + 1;  // bins < bin_cut run in the full-occupancy launch
+  if (p_max + 4 > ring_full) bin_cut = std::max(0, (ring_full - 4 - WF_G) / c->bucket + 1);
+  struct Launch { int bin_lo, bin_hi, warps, ring_len, bps; };
+  Launch L[2];
+  int nl = 0;
+  L[nl++] = Launch{0, std::min(bin_cut, kMaxBins + 1), WF_WARPS, std::min(p_max + 4, ring_full), bps_full};
+  if (bin_cut <= kMaxBins) {
+    Launch lb{bin_cut, kMaxBins + 1, 0, p_max + 4, 0};
+    int best = 0;
+    for (int w = WF_WARPS; w >= 1; w >>= 1) {
+      const size_t sm = wf_warp_smem<T>(lb.ring_len) * w;
+      if (sm > (size_t)c->smem_optin) continue;
+      int b = 0;
+      CUDA_TRY(wf_occupancy<T>(w, sm, &b));
+      if (b * w > best) { best = b * w; lb.warps = w; lb.bps = b; }
+    }
+    if (best < 1) return PHMM_E_INVALID_ARG;  // cannot happen for ncols <= kMaxHapLen + 8
+    L[nl++] = lb;
+  }
+
+  const int64_t nwarps = (int64_t)c->nsm * L[0].bps * L[0].warps;
   int64_t chunk = (int64_t)(pi.total_blocks / (unsigned long long)(nwarps * 4));
   if (chunk < 512) chunk = 512;
   if (chunk > 65536) chunk = 65536;
   const int nbins = kMaxBins + 1;
   k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, chunk, bin_start, item_start);
   LAUNCHED(c);
-  // stable sort of the pairs by bin, then contiguous block ranges by an exclusive scan
-  {
-    const int64_t n = d.n_pairs;
-    uint32_t* keys;
-    int32_t* vals;
-    int64_t *nbs, *blk_off;
-    ST_TRY(ws(c, B_SKEYS, (size_t)2 * n, &keys));
-    ST_TRY(ws(c, B_SVALS, (size_t)2 * n, &vals));
-    ST_TRY(ws(c, B_NBS, (size_t)n + 1, &nbs));
-    ST_TRY(ws(c, B_BLKOFF, (size_t)n + 1, &blk_off));
-    k_iota_keys<<<grid_for(c, n), kThreads, 0, s>>>(pair_bin, n, keys, vals);
-    LAUNCHED(c);
-    int end_bit = 1;
-    while ((1 << end_bit) <= kMaxBins + 1) ++end_bit;
-    size_t sort_bytes = 0, scan_bytes = 0;
-    CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
-    CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, nbs, blk_off, n + 1, s));
-    unsigned char* tmp;
-    ST_TRY(ws(c, B_SORT_TMP, std::max(sort_bytes, scan_bytes), &tmp));
-    CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
-    c->launches += 2;
-    k_sorted_nb<<<grid_for(c, n), kThreads, 0, s>>>(vals + n, pair_nb, n, nbs);
-    LAUNCHED(c);
-    CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, scan_bytes, nbs, blk_off, n + 1, s));
-    ++c->launches;
-    k_alloc_blocks_f32<<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, vals + n, n, pair_nb, blk_off, d.roff, d.hoff,
-                                                          hc_off, item_off, blk);
-    LAUNCHED(c);
-  }
-  F32Args A;
+  // stable sort of the pass's pairs by bin, then contiguous block ranges by an exclusive scan
+  uint32_t* keys;
+  int32_t* vals;
+  int64_t *nbs, *blk_off;
+  ST_TRY(ws(c, B_SKEYS, (size_t)2 * n, &keys));
+  ST_TRY(ws(c, B_SVALS, (size_t)2 * n, &vals));
+  ST_TRY(ws(c, B_NBS, (size_t)n + 1, &nbs));
+  ST_TRY(ws(c, B_BLKOFF, (size_t)n + 1, &blk_off));
+  k_iota_keys<<<grid_for(c, n), kThreads, 0, s>>>(pair_bin, n, keys, vals);
+  LAUNCHED(c);
+  int end_bit = 1;
+  while ((1 << end_bit) <= kMaxBins + 1) ++end_bit;
+  size_t sort_bytes = 0, scan_bytes = 0;
+  CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, nbs, blk_off, n + 1, s));
+  unsigned char* tmp;
+  ST_TRY(ws(c, B_SORT_TMP, std::max(sort_bytes, scan_bytes), &tmp));
+  CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+  c->launches += 2;
+  k_sorted_nb<<<grid_for(c, n), kThreads, 0, s>>>(vals + n, pair_nb, n, nbs);
+  LAUNCHED(c);
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, scan_bytes, nbs, blk_off, n + 1, s));
+  ++c->launches;
+  k_alloc_blocks_wf<K><<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, pair_item, vals + n, n, pair_nb, blk_off,
+                                                           d.roff, d.hoff, hc_off, item_off, blk);
+  LAUNCHED(c);
+
+  WfArgs2<T> A;
   A.blk = blk;
   A.tab = tab;
   A.hcodes = hc;
-  A.pad_idx = (uint32_t)total_hc;  // 4-aligned: every haplotype region is a multiple of 4
+  A.pad_idx = (uint32_t)total_hc;  // 4-aligned: every code region is a multiple of 4
   A.bin_start = bin_start;
   A.item_start = item_start;
-  A.nbins = nbins;
   A.bucket = c->bucket;
   A.chunk_blocks = chunk;
-  A.item_counter = &scal->item_counter;
   A.out = out;
-  A.ring_len = ring_len;
-  CUDA_TRY(cudaMemsetAsync(&scal->item_counter, 0, sizeof(unsigned int), s));
-  ev_record(c, EV_WF0);
-  CUDA_TRY(wf32_launch((unsigned)(c->nsm * bps), smem, s, A));
-  ++c->launches;
-  ev_record(c, EV_WF1);
+  CUDA_TRY(cudaMemsetAsync(scal->item_counter, 0, sizeof(scal->item_counter), s));
+  if (timed) ev_record(c, EV_WF0);
+  for (int i = 0; i < nl; ++i) {
+    A.bin_lo = L[i].bin_lo;
+    A.bin_hi = L[i].bin_hi;
+    A.ring_len = L[i].ring_len;
+    A.item_counter = &scal->item_counter[i];
+    CUDA_TRY(wf_launch<T>((unsigned)(c->nsm * L[i].bps), L[i].warps, wf_warp_smem<T>(L[i].ring_len) * L[i].warps,
+                          s, A));
+    ++c->launches;
+  }
+  if (timed) ev_record(c, EV_WF1);
   return PHMM_OK;
 }
-
-constexpr int K64 = 4;  // rows per lane, FP64 pass
 
 // The whole path on device-resident inputs. Writes dev_out (+ dev_status).
 phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status) {
@@ -463,18 +425,19 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   c->st = phmm_stats{};
   c->st.n_pairs = d.n_pairs;
   if (d.n_pairs == 0) return PHMM_OK;
-  uint8_t* hcodes = nullptr;
-  ST_TRY(run_validate(c, d, &hcodes));
+  ST_TRY(run_validate(c, d));
   PassInfo pi;
-  int64_t total_tab = 0;
+  int64_t total_tab = 0, total_hc = 0;
+  uint8_t* hc = nullptr;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   if (c->prec == PHMM_PREC_FP64) {
-    ST_TRY((pass_prepare<double, K64>(c, d, nullptr, d.n_pairs, &pi, &total_tab)));
+    ST_TRY((pass_prepare<double>(c, d, nullptr, d.n_pairs, &pi, &total_tab, &total_hc)));
+    ST_TRY(build_hap_codes(c, d, total_hc, pi.max_ncols, &hc));
     double* out64;
     ST_TRY(ws(c, B_OUT64, (size_t)d.n_pairs, &out64));
     ev_record(c, EV_PREP);
-    ST_TRY((pass_run<double, K64>(c, d, hcodes, nullptr, d.n_pairs, pi, total_tab, out64, nullptr)));
+    ST_TRY((pass_run<double>(c, d, nullptr, d.n_pairs, pi, total_tab, hc, total_hc, out64, true)));
     CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
     k_finalize_fp64<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out64, nullptr, nullptr, d.n_pairs, d.pairs,
                                                                   d.hoff, c->bucket, dev_out,
@@ -486,12 +449,12 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     CUDA_TRY(cudaStreamSynchronize(s));
     c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
   } else {
-    int64_t total_hc = 0;
-    ST_TRY((pass_prepare<float, F32_K>(c, d, nullptr, d.n_pairs, &pi, &total_tab, &total_hc)));
+    ST_TRY((pass_prepare<float>(c, d, nullptr, d.n_pairs, &pi, &total_tab, &total_hc)));
+    ST_TRY(build_hap_codes(c, d, total_hc, pi.max_ncols, &hc));
     float* out32;
     ST_TRY(ws(c, B_OUT32, (size_t)d.n_pairs, &out32));
     ev_record(c, EV_PREP);
-    ST_TRY(pass_run_f32(c, d, pi, total_tab, total_hc, out32));
+    ST_TRY(pass_run<float>(c, d, nullptr, d.n_pairs, pi, total_tab, hc, total_hc, out32, true));
     int32_t* rlist;
     ST_TRY(ws(c, B_RLIST, (size_t)d.n_pairs, &rlist));
     CUDA_TRY(cudaMemsetAsync(&scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
@@ -505,12 +468,13 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     const int64_t nr = c->host_scal->n_rescue;
     c->st.n_rescued = nr;
     if (nr > 0) {
+      // FP64 rescue of the listed pairs on the same kernel design (same code regions)
       PassInfo pr;
       int64_t tab_r = 0;
-      ST_TRY((pass_prepare<double, K64>(c, d, rlist, nr, &pr, &tab_r)));
+      ST_TRY((pass_prepare<double>(c, d, rlist, nr, &pr, &tab_r)));
       double* out64;
       ST_TRY(ws(c, B_OUT64, (size_t)nr, &out64));
-      ST_TRY((pass_run<double, K64>(c, d, hcodes, rlist, nr, pr, tab_r, out64, nullptr)));
+      ST_TRY((pass_run<double>(c, d, rlist, nr, pr, tab_r, hc, total_hc, out64, false)));
       CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
       k_finalize_fp64<<<grid_for(c, nr), kThreads, 0, s>>>(out64, rlist, nullptr, nr, d.pairs, d.hoff, c->bucket,
                                                            dev_out, dev_status,
@@ -537,7 +501,6 @@ phmm_status check_batch_args(const phmm_batch* b) {
   if (b->n_pairs == 0) return PHMM_OK;
   if (!b->pairs || !b->read_offsets || !b->hap_offsets) return PHMM_E_INVALID_ARG;
   if (b->total_read_bases < 0 || b->total_hap_bases < 0) return PHMM_E_INVALID_ARG;
-  if (b->total_hap_bases >= 0xffffffffLL - kHapPad) return PHMM_E_INVALID_ARG;
   if (b->total_read_bases > 0 &&
       (!b->read_bases || !b->base_quals || !b->ins_quals || !b->del_quals || !b->gcp_quals))
     return PHMM_E_INVALID_ARG;
@@ -617,7 +580,12 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
     return s;
   };
   if (cudaSetDevice(c->device) != cudaSuccess) return fail(PHMM_E_CUDA);
-  if (cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess)
+  if (cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess ||
+      cudaDeviceGetAttribute(&c->smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device) !=
+          cudaSuccess ||
+      cudaDeviceGetAttribute(&c->smem_reserved, cudaDevAttrReservedSharedMemoryPerBlock, c->device) !=
+          cudaSuccess ||
+      cudaDeviceGetAttribute(&c->smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, c->device) != cudaSuccess)
     return fail(PHMM_E_CUDA);
   if (cfg->cuda_stream) {
     c->stream = reinterpret_cast<cudaStream_t>(cfg->cuda_stream);
@@ -627,6 +595,10 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
   }
   if (cudaMallocHost(&c->host_scal, sizeof(Scalars)) != cudaSuccess) {
     c->host_scal = nullptr;
+    return fail(PHMM_E_OOM);
+  }
+  if (cudaMallocHost(&c->host_sizes, 2 * sizeof(int64_t)) != cudaSuccess) {
+    c->host_sizes = nullptr;
     return fail(PHMM_E_OOM);
   }
   for (int i = 0; i < kEvents; ++i)
@@ -644,6 +616,7 @@ void phmm_destroy(phmm_ctx* c) {
   for (int i = 0; i < kEvents; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
   if (c->host_scal) cudaFreeHost(c->host_scal);
+  if (c->host_sizes) cudaFreeHost(c->host_sizes);
   if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
   cudaGetLastError();
   delete c;

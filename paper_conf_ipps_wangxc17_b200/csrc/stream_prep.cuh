@@ -1,0 +1,206 @@
+// stream_prep.cuh -- prep kernels of a wavefront pass (FP32 main pass or FP64 pass):
+// haplotype code regions, per-read coefficient tables, stable length
+// binning and block descriptors (§8a-3). Included only by phmm_lib.cu.
+#pragma once
+#include "wavefront.cuh"
+
+namespace phmm {
+
+// ---------------------------------------------------------------- haplotype codes
+// Code region of one haplotype: 4 copies of wf_hc_copy_len(ncols) bytes; in copy k
+// column c sits at byte WF_HC_FRONT + k + c (so a lane picks the copy that makes its
+// code words 4-aligned). Byte = code * WF_CB with code A=0 C=1 G=2 T=3 N=4 PAD=5:
+// columns c < N carry the haplotype, c == N carries 'N' (matches every row), every
+// other byte is PAD (prior 0). BlkDesc.hap_off = region start + WF_HC_FRONT.
+// (Moved into bits 8..15 by the kernel, the byte becomes the offset of the code's rows
+// in a lane's shared-memory prior table.)
+__host__ __device__ inline int64_t wf_hc_region(int n, int bucket) {
+  return 4 * (int64_t)wf_hc_copy_len(ncols_of(n, bucket));
+}
+
+__global__ void k_hap_codes_wf(const uint8_t* __restrict__ hap, const int64_t* __restrict__ hoff, int64_t n_haps,
+                               const int64_t* __restrict__ hc_off, int bucket, uint8_t* __restrict__ codes) {
+  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t h = warp; h < n_haps; h += nwarps) {
+    const int64_t h0 = hoff[h];
+    const int n = (int)(hoff[h + 1] - h0);
+    if (n < 1 || n > kMaxHapLen) continue;
+    const int len = wf_hc_copy_len(ncols_of(n, bucket));  // multiple of 4, region start 4-aligned
+    uint32_t* dst = reinterpret_cast<uint32_t*>(codes + hc_off[h]);
+    const int wpc = len >> 2;  // words per copy
+    for (int k = 0; k < 4; ++k) {
+      for (int w = lane; w < wpc; w += 32) {
+        uint32_t word = 0;
+#pragma unroll
+        for (int by = 0; by < 4; ++by) {
+          const int c = 4 * w + by - (int)WF_HC_FRONT - k;  // column of this byte in copy k
+          uint32_t v = WF_PAD;
+          if (c >= 0 && c < n) {
+            switch (hap[h0 + c]) {
+              case 'A': v = 0; break;
+              case 'C': v = 1; break;
+              case 'G': v = 2; break;
+              case 'T': v = 3; break;
+              default: v = 4; break;  // 'N' (invalid bytes were rejected by validation)
+            }
+          } else if (c == n) {
+            v = 4;
+          }
+          word |= (v * WF_CB) << (8 * by);
+        }
+        dst[k * wpc + w] = word;
+      }
+    }
+  }
+}
+
+__global__ void k_hap_ncols(const int64_t* __restrict__ hoff, int64_t n_haps, int bucket, int64_t* __restrict__ nc) {
+  for (int64_t h = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; h < n_haps; h += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t n = hoff[h + 1] - hoff[h];
+    nc[h] = (n >= 1 && n <= kMaxHapLen) ? wf_hc_region((int)n, bucket) : 0;
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) nc[n_haps] = 0;
+}
+
+// ---------------------------------------------------------------- coefficient tables
+// Per table item (a read, or a rescued pair's read): nb = ceil((m+3)/K) blocks of K rows
+//   [f Z rows][R][read rows 1..m][S1][S2]          (phmm_common.cuh)
+// One warp per item, lanes over its padded rows; Phred -> error probability from a
+// 128-entry table built once per CUDA block (10^(-q/10) in double, rounded to T).
+constexpr int kTabThreads = 256;
+template <typename T>
+__global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
+    const int32_t* __restrict__ item_read, int64_t n_items, const int64_t* __restrict__ item_tab_off,
+    const int64_t* __restrict__ roff, const uint8_t* __restrict__ rb, const uint8_t* __restrict__ q,
+    const uint8_t* __restrict__ qi, const uint8_t* __restrict__ qd, const uint8_t* __restrict__ qg,
+    TBlock<T>* __restrict__ tab) {
+  constexpr int K = WfT<T>::K;
+  __shared__ T err[128];
+  for (int i = threadIdx.x; i < 128; i += blockDim.x) err[i] = qual_err<T>((uint32_t)i);
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t it = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; it < n_items; it += nwarps) {
+    const int64_t r = item_read ? item_read[it] : it;
+    const int64_t r0 = roff[r];
+    const int m = (int)(roff[r + 1] - r0);
+    if (m < 1) continue;
+    const int nb = nblocks_of<K>(m);
+    const int f = nb * K - (m + 3);
+    TBlock<T>* __restrict__ Tb = tab + item_tab_off[it];
+    for (int row = lane; row < nb * K; row += 32) {
+      T al = 0, be = 0, de = 0, ep = 0, ze = 0, mu = 0;
+      T p5[5] = {0, 0, 0, 0, 0};
+      if (row < f) {
+        // Z row: all zero
+      } else if (row == f) {  // R row: D = d0 on every column
+        mu = 1;
+      } else if (row <= f + m) {
+        const int64_t x = r0 + (row - f - 1);
+        const T ei = err[qi[x] & 127], ed = err[qd[x] & 127], eg = err[qg[x] & 127], eb = err[q[x] & 127];
+        const T sum = ei + ed;
+        al = (T)1 - (sum < (T)1 ? sum : (T)1);
+        be = (T)1 - eg;
+        de = ei;
+        ep = eg;
+        ze = ed;
+        mu = eg;
+        const T pm = (T)1 - eb, px = eb / (T)3;
+        const uint8_t base = rb[x];
+        p5[0] = (base == 'A' || base == 'N') ? pm : px;
+        p5[1] = (base == 'C' || base == 'N') ? pm : px;
+        p5[2] = (base == 'G' || base == 'N') ? pm : px;
+        p5[3] = (base == 'T' || base == 'N') ? pm : px;
+        p5[4] = pm;  // haplotype 'N' matches everything
+      } else if (row == f + m + 1) {  // S1: I = M(m,j) + I(m,j)
+        de = 1; ep = 1; mu = 1;
+      } else {  // S2: M = I_S1(j-1), D = running sum
+        be = 1; ze = 1; mu = 1;
+        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = 1;
+      }
+      TBlock<T>& B = Tb[row / K];
+      const int t = row % K;
+      B.coef[0][t] = al; B.coef[1][t] = be; B.coef[2][t] = de;
+      B.coef[3][t] = ep; B.coef[4][t] = ze; B.coef[5][t] = mu;
+#pragma unroll
+      for (int k = 0; k < 5; ++k) B.prior[k][t] = p5[k];
+    }
+  }
+}
+
+// ---------------------------------------------------------------- stable binning
+// Pairs are radix-sorted by bin (stable: read-major input order survives inside a bin,
+// the pairs of one read stay adjacent and its table is reused from L2), then each
+// sorted pair gets a contiguous block range from an exclusive scan. Deterministic.
+__global__ void k_iota_keys(const int32_t* __restrict__ pair_bin, int64_t n, uint32_t* __restrict__ keys,
+                            int32_t* __restrict__ vals) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    keys[i] = (uint32_t)pair_bin[i];
+    vals[i] = (int32_t)i;
+  }
+}
+
+__global__ void k_sorted_nb(const int32_t* __restrict__ sorted_idx, const int32_t* __restrict__ pair_nb, int64_t n,
+                            int64_t* __restrict__ nb_sorted) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    nb_sorted[i] = pair_nb[sorted_idx[i]];
+  if (blockIdx.x == 0 && threadIdx.x == 0) nb_sorted[n] = 0;
+}
+
+// Block descriptors: one warp per 32 sorted entries, the lanes of the warp write one
+// pair's descriptors together (coalesced 16-byte stores). Entry k of the pass is pair
+// list[k] (or k when list == nullptr); its table item is pair_item[k] (or its read),
+// its output slot k (list) or the pair id.
+template <int K>
+__global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32_t* __restrict__ list,
+                                  const int32_t* __restrict__ pair_item, const int32_t* __restrict__ sorted_idx,
+                                  int64_t n, const int32_t* __restrict__ pair_nb, const int64_t* __restrict__ blk_off,
+                                  const int64_t* __restrict__ roff, const int64_t* __restrict__ hoff,
+                                  const int64_t* __restrict__ hc_off, const int64_t* __restrict__ item_tab_off,
+                                  BlkDesc* __restrict__ blk) {
+  const int lane = threadIdx.x & 31;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < n; base += stride) {
+    const int64_t i = base + lane;
+    int nb = 0, m = 0, nh = 0;
+    int64_t g0 = 0, slot = 0;
+    uint32_t tab0 = 0, hap = 0;
+    if (i < n) {
+      const int64_t k = sorted_idx[i];
+      const int64_t p = list ? list[k] : k;
+      nb = pair_nb[k];
+      const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
+      m = (int)(roff[r + 1] - roff[r]);
+      nh = (int)(hoff[h + 1] - hoff[h]);
+      g0 = blk_off[i];
+      tab0 = (uint32_t)item_tab_off[pair_item ? pair_item[k] : r];
+      hap = (uint32_t)(hc_off[h] + WF_HC_FRONT);
+      slot = list ? k : p;
+    }
+    const int cnt = (int)min((int64_t)32, n - base);
+    for (int src = 0; src < cnt; ++src) {
+      const int nb_s = __shfl_sync(0xffffffffu, nb, src);
+      const int m_s = __shfl_sync(0xffffffffu, m, src);
+      const int nh_s = __shfl_sync(0xffffffffu, nh, src);
+      const int64_t g0_s = __shfl_sync(0xffffffffu, g0, src);
+      const int64_t slot_s = __shfl_sync(0xffffffffu, slot, src);
+      const uint32_t tab_s = __shfl_sync(0xffffffffu, tab0, src);
+      const uint32_t hap_s = __shfl_sync(0xffffffffu, hap, src);
+      const int f = nb_s * K - (m_s + 3);  // R row index within the pair's rows
+      for (int j = lane; j < nb_s; j += 32) {
+        BlkDesc d;
+        d.tab_blk = tab_s + j;
+        d.hap_off = hap_s;
+        d.out_idx = (int32_t)slot_s;
+        d.n = (uint16_t)nh_s;
+        const int rrow = (f / K == j) ? (f % K) : WF_RROW_NONE;
+        d.flags = (uint16_t)((j == nb_s - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) | (rrow << WF_RROW_SHIFT));
+        blk[g0_s + j] = d;
+      }
+    }
+  }
+}
+
+}  // namespace phmm

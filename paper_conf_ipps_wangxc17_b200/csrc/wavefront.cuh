@@ -1,0 +1,470 @@
+// wavefront.cuh -- the PairHMM wavefront kernel for sm_100a (the hot loop), FP32 and FP64.
+//
+// PRODUCT PATH. Computes Eq. 6 of PAPER.md (L18@541) over "tall streams" of
+// K-row blocks (see phmm_common.cuh for the Z/R/S1/S2 pad-row layout that makes
+// a pair's termination sum (L20@2262) fall out of the recurrence).
+//
+// The paper's PH2 kernel (L20@3509, Fig. 8) gives one warp one pair and lets each
+// thread own consecutive rows, passing the row-above values by shuffle (its Design
+// B, Listing 2b, L20@44). This kernel keeps the row ownership and the shuffle and
+// changes the rest for Blackwell:
+//  * a warp streams through a long sequence of blocks of one length bin; it has 64
+//    VIRTUAL lanes v = 2*lane + h (h = 0/1: the two halves of a register pair), each
+//    owning one K-row block per pass (blocks 64q + v); virtual lane v computes column
+//    x of its block at step T_q + 1 + v + x.
+//  * FP32: the halves are the two floats of a 64-bit register, so every FP op of
+//    Eq. 6 is one packed FFMA2/FMUL2/FADD2 for two independent cells (K = 8 rows).
+//    FP64 (the rescue pass): the halves are two doubles, scalar DFMA (K = 4 rows).
+//  * the emission prior P(i,j): a per-half table prior[code][row] in shared memory
+//    (code = haplotype base A,C,G,T,N or PAD); 16-byte LDS per chunk of rows.
+//  * no per-lane "is this column real" branch: columns outside a block read the PAD
+//    code (prior 0); by induction down the lanes an idle virtual lane then computes
+//    exactly the boundary column (M = I = 0, D = D(i,0)) before its block and freezes
+//    the S2 running sum after it.
+//  * virtual lanes switch blocks in groups of G = 8 (8 switch events per pass); a pass
+//    is P = max(ncols + G, 72) steps.
+//  * row above: half B of a lane takes its own half A one step later (no shuffle);
+//    half A takes lane-1's half B by __shfl_sync; virtual lane 0 takes virtual lane
+//    63 of the previous pass through a per-warp shared-memory ring indexed by column
+//    + 1 (slot 0 = boundary column); lane 31 substitutes the ring slot into what it
+//    shuffles.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "phmm_common.cuh"
+
+namespace phmm {
+
+#if defined(PHMM_DBG_TRACE) && defined(PHMM_DEFINE_WF)
+// debug builds only: per-step last-row state (FP32 pass) of the warp that runs work item 0
+__device__ float g_trace[4096 * 32 * 2 * 3];
+__device__ int g_trace_steps;
+#endif
+
+#ifndef PHMM_F32_K
+#define PHMM_F32_K 8
+#endif
+
+constexpr int WF_G = 8;           // virtual lanes per switch group
+constexpr int WF_NCODE = 6;       // A C G T N PAD
+constexpr int WF_PAD = 5;
+constexpr int WF_WARPS = 4;       // warps per CTA
+constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
+constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
+constexpr int WF_KC = 2;          // 16-byte chunks per row set (FP32 K=8 and FP64 K=4 alike)
+// code byte in the haplotype code arrays = code * WF_CB; moved into bits 8..15 it is
+// code * WF_KC * 512 bytes = the stride of one code's rows in a lane's prior table
+constexpr int WF_CB = 2 * WF_KC;
+
+// BlkDesc.flags: bit0 last, bit1 first, bits 8-11 R row (15 = none)
+constexpr uint16_t WF_RROW_SHIFT = 8;
+constexpr uint16_t WF_RROW_NONE = 15;
+
+// ---------------------------------------------------------------- precision traits
+typedef unsigned long long v2f;           // two floats in a 64-bit register pair
+struct alignas(16) v2d { double a, b; };  // two doubles
+
+template <typename T> struct WfT;
+template <> struct WfT<float> {
+  using V = v2f;
+  static constexpr int K = PHMM_F32_K;
+  static constexpr int kScaleExp = 120;
+};
+template <> struct WfT<double> {
+  using V = v2d;
+  static constexpr int K = 4;
+  static constexpr int kScaleExp = 1020;
+};
+static_assert(WfT<float>::K * 4 == WF_KC * 16 && WfT<double>::K * 8 == WF_KC * 16, "chunk layout");
+
+__device__ __forceinline__ v2f pk(float lo, float hi) {
+  v2f r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+  return r;
+}
+__device__ __forceinline__ float lo(v2f v) {
+  float a, b;
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v));
+  (void)b;
+  return a;
+}
+__device__ __forceinline__ float hi(v2f v) {
+  float a, b;
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v));
+  (void)a;
+  return b;
+}
+__device__ __forceinline__ v2f fma2(v2f a, v2f b, v2f c) {
+  v2f d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+__device__ __forceinline__ v2f mul2(v2f a, v2f b) {
+  v2f d;
+  asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ v2f add2(v2f a, v2f b) {
+  v2f d;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ v2d pk(double lo, double hi) { return v2d{lo, hi}; }
+__device__ __forceinline__ double lo(v2d v) { return v.a; }
+__device__ __forceinline__ double hi(v2d v) { return v.b; }
+__device__ __forceinline__ v2d fma2(v2d a, v2d b, v2d c) { return v2d{fma(a.a, b.a, c.a), fma(a.b, b.b, c.b)}; }
+__device__ __forceinline__ v2d mul2(v2d a, v2d b) { return v2d{a.a * b.a, a.b * b.b}; }
+__device__ __forceinline__ v2d add2(v2d a, v2d b) { return v2d{a.a + b.a, a.b + b.b}; }
+
+template <int H, typename V, typename S>
+__device__ __forceinline__ V set_half(V r, S v) {
+  return H == 0 ? pk(v, hi(r)) : pk(lo(r), v);
+}
+template <typename V> __device__ __forceinline__ V vzero();
+template <> __device__ __forceinline__ v2f vzero<v2f>() { return 0ull; }
+template <> __device__ __forceinline__ v2d vzero<v2d>() { return v2d{0.0, 0.0}; }
+
+// per-block coefficient table: 6 transition fields + 5 prior codes, K rows each
+template <typename T>
+struct alignas(16) TBlock {
+  T coef[6][WfT<T>::K];   // alpha, beta, delta, eps, zeta, mu
+  T prior[5][WfT<T>::K];  // P(row, code) for code = A, C, G, T, N
+};
+static_assert(sizeof(TBlock<float>) == 11 * WF_KC * 16 && sizeof(TBlock<double>) == 11 * WF_KC * 16, "TBlock");
+
+template <typename T>
+struct WfArgs2 {
+  const BlkDesc* blk;
+  const TBlock<T>* tab;
+  const uint8_t* hcodes;                 // per-haplotype code regions (4 shifted copies)
+  uint32_t pad_idx;                      // index of an all-PAD region (idle lanes)
+  const unsigned long long* bin_start;   // [nbins+1] first block of each bin
+  const unsigned long long* item_start;  // [nbins+1] first work item of each bin
+  int bin_lo, bin_hi;                    // this launch runs the work items of bins [bin_lo, bin_hi)
+  int bucket;
+  int64_t chunk_blocks;
+  unsigned int* item_counter;
+  T* out;
+  int ring_len;  // slots, >= P + 4
+};
+
+template <typename T>
+struct Lane {
+  using V = typename WfT<T>::V;
+  static constexpr int K = WfT<T>::K;
+  V al[K], be[K], de[K], ep[K], ze[K], mu[K];
+  V M[K], I[K], D[K];
+};
+
+// One column for both halves, in place. dg* = row above at column x-1, up* = row above at column x.
+template <typename T>
+__device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K], const T (&prB)[WfT<T>::K],
+                                          const typename WfT<T>::V dgM, const typename WfT<T>::V dgI,
+                                          const typename WfT<T>::V dgD, const typename WfT<T>::V upM,
+                                          const typename WfT<T>::V upI) {
+  using V = typename WfT<T>::V;
+  constexpr int K = WfT<T>::K;
+  // M and D: rows descending so that row u-1's old values are intact when row u reads them
+#pragma unroll
+  for (int u = K - 1; u >= 0; --u) {
+    const V md = (u == 0) ? dgM : L.M[u - 1];
+    const V id = (u == 0) ? dgI : L.I[u - 1];
+    const V dd = (u == 0) ? dgD : L.D[u - 1];
+    // D(i,j) = zeta*M(i,j-1) + mu*D(i,j-1)
+    L.D[u] = fma2(L.ze[u], L.M[u], mul2(L.mu[u], L.D[u]));
+    // M(i,j) = P(i,j) * (alpha*M(i-1,j-1) + beta*(I(i-1,j-1) + D(i-1,j-1)))
+    const V x = fma2(L.al[u], md, mul2(L.be[u], add2(id, dd)));
+    L.M[u] = pk(prA[u] * lo(x), prB[u] * hi(x));
+  }
+  // I(i,j) = delta*M(i-1,j) + eps*I(i-1,j), rows ascending (a K-deep chain)
+  V m_up = upM, i_up = upI;
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    const V ni = fma2(L.ep[u], i_up, mul2(L.de[u], m_up));
+    m_up = L.M[u];
+    i_up = ni;
+    L.I[u] = ni;
+  }
+}
+
+// ---- shared-memory accessors (inline PTX with "memory" clobbers: the ring and the prior
+// tables are only touched through these, so no compiler reordering or aliasing games)
+__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void ring_put3(uint32_t a, float x, float y, float z) {
+  asm volatile("st.shared.f32 [%0], %1;\n\tst.shared.f32 [%0+4], %2;\n\tst.shared.f32 [%0+8], %3;"
+               :: "r"(a), "f"(x), "f"(y), "f"(z) : "memory");
+}
+__device__ __forceinline__ void ring_get3(uint32_t a, float& x, float& y, float& z) {
+  float w;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(x), "=f"(y), "=f"(z), "=f"(w) : "r"(a) : "memory");
+  (void)w;
+}
+__device__ __forceinline__ void ring_put3(uint32_t a, double x, double y, double z) {
+  asm volatile("st.shared.f64 [%0], %1;\n\tst.shared.f64 [%0+8], %2;\n\tst.shared.f64 [%0+16], %3;"
+               :: "r"(a), "d"(x), "d"(y), "d"(z) : "memory");
+}
+__device__ __forceinline__ void ring_get3(uint32_t a, double& x, double& y, double& z) {
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%3];\n\tld.shared.f64 %2, [%3+16];"
+               : "=d"(x), "=d"(y), "=d"(z) : "r"(a) : "memory");
+}
+template <typename T> __host__ __device__ constexpr uint32_t ring_slot_bytes() { return sizeof(T) == 4 ? 16u : 32u; }
+
+// 16-byte shared load reinterpreted as 4 floats or 2 doubles
+__device__ __forceinline__ void lds16(uint32_t a, float* v) {
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3])
+               : "r"(a) : "memory");
+}
+__device__ __forceinline__ void lds16(uint32_t a, double* v) {
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v[0]), "=d"(v[1]) : "r"(a) : "memory");
+}
+__device__ __forceinline__ void sts16(uint32_t a, const uint4 v) {
+  asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" :: "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+
+// Haplotype code regions: 4 shifted copies per haplotype so that every lane reads its
+// codes as aligned 32-bit words, 4 columns at a time.
+__host__ __device__ inline int wf_hc_copy_len(int ncols) {
+  const int p = (ncols + WF_G > WF_MIN_P) ? ncols + WF_G : WF_MIN_P;
+  return ((int)WF_HC_FRONT + p + 24 + 3) & ~3;  // + prefetch distance
+}
+
+// Load a block (or nothing) into half H of a lane. Returns the 32-bit-aligned code
+// pointer for the lane's first step (column -1 - gi).
+template <int H, typename T>
+__device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>& L, uint32_t tab_s, bool have,
+                                                   const BlkDesc& d, T d0, int& out_idx, int gi, int copy_len) {
+  constexpr int K = WfT<T>::K;
+  constexpr int PER = 16 / sizeof(T);  // values per 16-byte chunk
+  if (have) {
+    const uint4* __restrict__ s4 = reinterpret_cast<const uint4*>(A.tab + d.tab_blk);
+    union { uint4 u[6 * WF_KC]; T v[6][K]; } cw;
+#pragma unroll
+    for (int k = 0; k < 6 * WF_KC; ++k) cw.u[k] = __ldg(s4 + k);
+#pragma unroll
+    for (int k = 0; k < 5 * WF_KC; ++k) sts16(tab_s + 512u * k, __ldg(s4 + 6 * WF_KC + k));  // prior[code][chunk]
+    const int rrow = (d.flags >> WF_RROW_SHIFT) & 15;
+#pragma unroll
+    for (int u = 0; u < K; ++u) {
+      L.al[u] = set_half<H>(L.al[u], cw.v[0][u]); L.be[u] = set_half<H>(L.be[u], cw.v[1][u]);
+      L.de[u] = set_half<H>(L.de[u], cw.v[2][u]); L.ep[u] = set_half<H>(L.ep[u], cw.v[3][u]);
+      L.ze[u] = set_half<H>(L.ze[u], cw.v[4][u]); L.mu[u] = set_half<H>(L.mu[u], cw.v[5][u]);
+      L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
+      L.D[u] = set_half<H>(L.D[u], rrow == u ? d0 : (T)0);
+    }
+    (void)PER;
+    out_idx = (d.flags & BLK_LAST) ? d.out_idx : -1;
+    // copy k = (1 + gi) mod 4 has column 0 at hap_off + k*(copy_len + 1), so the byte
+    // of column (-1 - gi) is 4-aligned
+    const int k = (1 + gi) & 3;
+    const uint32_t col0 = d.hap_off + (uint32_t)(k * (copy_len + 1));
+    return reinterpret_cast<const uint32_t*>(A.hcodes + (col0 - 1u - (uint32_t)gi));
+  }
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    L.al[u] = set_half<H>(L.al[u], (T)0); L.be[u] = set_half<H>(L.be[u], (T)0);
+    L.de[u] = set_half<H>(L.de[u], (T)0); L.ep[u] = set_half<H>(L.ep[u], (T)0);
+    L.ze[u] = set_half<H>(L.ze[u], (T)0); L.mu[u] = set_half<H>(L.mu[u], (T)0);
+    L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
+    L.D[u] = set_half<H>(L.D[u], (T)0);
+  }
+  out_idx = -1;
+  return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
+}
+
+// One warp streams through blocks [s, s+nblk) of one bin (ncols columns each).
+template <typename T>
+__device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s, int lane,
+                                          int64_t s, int nblk, int ncols, bool trace = false) {
+  using V = typename WfT<T>::V;
+  constexpr int K = WfT<T>::K;
+  constexpr int PER = 16 / sizeof(T);
+  constexpr int G = WF_G;            // virtual lanes per switch group
+  constexpr int NGRP = 64 / G;       // switch events per pass
+  constexpr int LPG = G / 2;         // physical lanes per group
+  constexpr uint32_t RS = ring_slot_bytes<T>();
+  const int grp = lane / LPG;
+  const int giA = 2 * (lane % LPG), giB = giA + 1;  // position of each half inside its group
+  const T d0 = (T)ldexp(1.0, WfT<T>::kScaleExp) / (T)ncols;  // virtual row 0
+  const int P = max(ncols + G, WF_MIN_P);                     // multiple of 4 (ncols is)
+  const int npass = (nblk + 63) >> 6;
+  const int copy_len = wf_hc_copy_len(ncols);
+  Lane<T> L;
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    L.al[u] = L.be[u] = L.de[u] = L.ep[u] = L.ze[u] = L.mu[u] = vzero<V>();
+    L.M[u] = L.I[u] = L.D[u] = vzero<V>();
+  }
+  const uint32_t* pA = reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);  // next code word
+  const uint32_t* pB = pA;
+  constexpr uint32_t kPadW = (uint32_t)(WF_PAD * WF_CB) * 0x01010101u;  // four PAD codes
+  // code words: current group, next group, the one after (prefetch distance 2 groups)
+  uint32_t wA = kPadW, wB = kPadW, wA_nx = kPadW, wB_nx = kPadW, wA_nx2 = kPadW, wB_nx2 = kPadW;
+  int outA = -1, outB = -1;
+  V upM = vzero<V>(), upI = vzero<V>(), upD = vzero<V>(), dgM = vzero<V>(), dgI = vzero<V>(), dgD = vzero<V>();
+  const uint32_t tabA_s = ptab_s + 16u * lane;                              // [code][chunk][lane] 16 B
+  const uint32_t tabB_s = ptab_s + 16u * (WF_NCODE * WF_KC * 32 + lane);   // half B
+  const int src = (lane + 31) & 31;
+  const bool is0 = lane == 0, is31 = lane == 31;
+  int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
+  int c31B = -(1 << 20);  // (uniform) column of virtual lane 63 (lane 31, half B)
+  T rvM = 0, rvI = 0, rvD = 0;  // lane 31: ring slot for virtual lane 0's next column
+  BlkDesc dnA, dnB;  // next pass's block descriptors (prefetched)
+  dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.n = 1; dnA.flags = 0;
+  dnB = dnA;
+#ifdef PHMM_DBG_TRACE
+  int tstep = 0;
+#endif
+
+  auto step = [&](const int r) {
+    if (is31) ring_get3(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
+    // code byte r (= code*WF_CB) placed in byte 1 -> the code's rows in the table
+    const uint32_t oA = __byte_perm(wA, 0, 0x4404 + (r << 4)), oB = __byte_perm(wB, 0, 0x4404 + (r << 4));
+    T prA[K], prB[K];
+#pragma unroll
+    for (int ch = 0; ch < WF_KC; ++ch) {
+      lds16(tabA_s + oA + 512u * ch, prA + PER * ch);
+      lds16(tabB_s + oB + 512u * ch, prB + PER * ch);
+    }
+    wf_column<T>(L, prA, prB, dgM, dgI, dgD, upM, upI);
+    constexpr int LR = K - 1;  // last row of a block
+    const T m3a = lo(L.M[LR]), i3a = lo(L.I[LR]), d3a = lo(L.D[LR]);
+    const T m3b = hi(L.M[LR]), i3b = hi(L.I[LR]), d3b = hi(L.D[LR]);
+    // half B of lane-1 -> half A of lane; lane 31 sends the ring slot instead (virtual 63 -> 0)
+    const T sM = is31 ? rvM : m3b;
+    const T sI = is31 ? rvI : i3b;
+    const T sD = is31 ? rvD : d3b;
+    if (is31 && (unsigned)(c31B + 1) <= (unsigned)ncols)  // -1 <= c31B < ncols
+      ring_put3(ring_s + RS * (uint32_t)(c31B + 1), m3b, i3b, d3b);
+    __syncwarp();
+    dgM = upM; dgI = upI; dgD = upD;
+    // next step: half A's row above = lane-1's half B; half B's row above = this lane's half A
+    upM = pk(__shfl_sync(0xffffffffu, sM, src), m3a);
+    upI = pk(__shfl_sync(0xffffffffu, sI, src), i3a);
+    upD = pk(__shfl_sync(0xffffffffu, sD, src), d3a);
+#if defined(PHMM_DBG_TRACE) && defined(PHMM_DEFINE_WF)
+    if (sizeof(T) == 4 && trace && tstep < 4096) {
+      float* t = g_trace + ((size_t)tstep * 32 + lane) * 6;
+      t[0] = (float)m3a; t[1] = (float)i3a; t[2] = (float)d3a;
+      t[3] = (float)m3b; t[4] = (float)i3b; t[5] = (float)d3b;
+      if (lane == 0) g_trace_steps = tstep + 1;
+    }
+    ++tstep;
+#endif
+    ++c0;
+    ++c31B;
+  };
+  // 4 steps sharing one code word per half; the next words are prefetched
+  auto group4 = [&]() {
+    wA = wA_nx; wB = wB_nx;
+    wA_nx = wA_nx2; wB_nx = wB_nx2;
+    wA_nx2 = __ldg(pA); wB_nx2 = __ldg(pB);
+    ++pA; ++pB;
+    step(0); step(1); step(2); step(3);
+  };
+
+  for (int q = 0; q <= npass; ++q) {
+#pragma unroll 1
+    for (int e = 0; e < NGRP; ++e) {
+      if (e == 0) c0 = -1;                      // virtual lane 0 starts its pass: column -1 next
+      if (e == NGRP - 1) c31B = -1 - (G - 1);  // virtual lane 63
+      if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
+        const int bA = q * 64 + 2 * lane, bB = bA + 1;
+        const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
+        // this pass's descriptors were prefetched one pass ago (pass 0: loaded now)
+        BlkDesc dA = dnA, dB = dnB;
+        if (q == 0) {
+          if (hA) dA = A.blk[s + bA];
+          if (hB) dB = A.blk[s + bB];
+        }
+        if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S2 row: the last-row M+I sum (L20@2262)
+        if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
+        pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
+        pB = wf_load<1, T>(A, L, tabB_s, hB, dB, d0, outB, giB, copy_len);
+        wA_nx = __ldg(pA); wA_nx2 = __ldg(pA + 1); pA += 2;
+        wB_nx = __ldg(pB); wB_nx2 = __ldg(pB + 1); pB += 2;
+        // prefetch the next pass's descriptors after this pass's loads are issued (a load
+        // issued before the consumers of the previous prefetch would share its scoreboard)
+        if (bA + 64 < nblk) dnA = A.blk[s + bA + 64];
+        if (bB + 64 < nblk) dnB = A.blk[s + bB + 64];
+        if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
+          T a, bb, c;
+          ring_get3(ring_s, a, bb, c);
+          upM = set_half<0>(upM, a); upI = set_half<0>(upI, bb); upD = set_half<0>(upD, c);
+        }
+      }
+      const int ngroups = (e < NGRP - 1) ? G / 4 : (q < npass ? (P - (NGRP - 1) * G) / 4 : 0);
+#pragma unroll 1
+      for (int k = 0; k < ngroups; ++k) group4();
+    }
+  }
+}
+
+// The kernels are defined in wf.cu (their own translation unit, compiled with
+// -Xptxas -O1: ptxas -O2/-O3 mis-schedules the FP32 kernel -- results silently differ
+// from the -O0/-O1 builds and from the CPU model of the schedule).
+// phmm_lib.cu reaches them through these host functions.
+// shared memory of one warp: its prior tables and its ring
+template <typename T> size_t wf_warp_smem(int ring_len) {
+  return (size_t)2 * WF_NCODE * WF_KC * 32 * 16 + (size_t)ring_len * ring_slot_bytes<T>();
+}
+template <typename T> cudaError_t wf_occupancy(int warps, size_t smem, int* blocks_per_sm);
+template <typename T>
+cudaError_t wf_launch(unsigned grid, int warps, size_t smem, cudaStream_t stream, const WfArgs2<T>& args);
+
+#ifdef PHMM_DEFINE_WF
+#ifndef PHMM_F32_MINB
+#define PHMM_F32_MINB 2  // CTAs (of 4 warps) per SM the register budget must allow (255 regs)
+#endif
+template <typename T>
+__global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfArgs2<T> A) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const int lane = threadIdx.x & 31;
+  const int wib = threadIdx.x >> 5;
+  // per warp: prior tables [2 halves][6 codes][WF_KC chunks][32 lanes] x 16 B, then the ring
+  constexpr uint32_t kTabBytes = 2 * WF_NCODE * WF_KC * 32 * 16;
+  const uint32_t per_warp = kTabBytes + (uint32_t)A.ring_len * ring_slot_bytes<T>();
+  unsigned char* base = smem_raw + (size_t)wib * per_warp;
+  for (uint32_t i = 4 * lane; i < per_warp; i += 128) *reinterpret_cast<uint32_t*>(base + i) = 0u;
+  __syncwarp();
+  const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
+  // work item it of the launch: chunk k of bin b (binary search in item_start)
+  const unsigned long long it0 = A.item_start[A.bin_lo], it1 = A.item_start[A.bin_hi];
+  while (true) {
+    unsigned long long it = 0;
+    if (lane == 0) it = it0 + atomicAdd(A.item_counter, 1u);
+    it = __shfl_sync(0xffffffffu, it, 0);
+    if (it >= it1) break;
+    int lo_ = A.bin_lo, hi_ = A.bin_hi - 1;
+    while (lo_ < hi_) {
+      const int mid = (lo_ + hi_ + 1) >> 1;
+      if (A.item_start[mid] <= it) lo_ = mid; else hi_ = mid - 1;
+    }
+    const int bin = lo_;
+    const int64_t b0 = (int64_t)A.bin_start[bin], b1 = (int64_t)A.bin_start[bin + 1];
+    const int64_t k = (int64_t)(it - A.item_start[bin]);
+    int64_t s = b0 + k * A.chunk_blocks;
+    int64_t e = s + A.chunk_blocks;
+    if (e > b1) e = b1;
+    auto advance = [&](int64_t x) -> int64_t {
+      while (x < b1) {
+        const int64_t y = x + lane;
+        const bool first = (y < b1) ? ((A.blk[y].flags & BLK_FIRST) != 0) : true;
+        const unsigned bal = __ballot_sync(0xffffffffu, first);
+        if (bal) return x + __ffs(bal) - 1;
+        x += 32;
+      }
+      return b1;
+    };
+    s = advance(s);
+    e = (e >= b1) ? b1 : advance(e);
+    if (e <= s) continue;
+    wf_stream<T>(A, ptab_s, ring_s, lane, s, (int)(e - s), bin * A.bucket, it == 0);
+    __syncwarp();
+  }
+}
+#endif  // PHMM_DEFINE_WF
+
+}  // namespace phmm

@@ -219,3 +219,46 @@ def test_full_c2_sampled(ctx32):
     _check(out[sample], ref, "fp32")
     # decoy reads (2 %) make some pairs need the rescue
     assert 0 < np.sum(st == 1) < b.n_pairs // 10
+
+
+def _long_short_mix(seed, n_long, n_short, long_range=(4000, 4094)):
+    """Haplotypes up to the maximum length (4094) mixed with short ones: the long
+    bins run in the second, reduced-occupancy wavefront launch."""
+    long_ = synth.random_pairs_batch(seed, n_long, m_range=(1, 150), n_range=long_range, qual_range=(20, 40))
+    short = synth.random_pairs_batch(seed + 1, n_short, m_range=(1, 120), n_range=(1, 300))
+    b = synth.concat_batches([short, long_])
+    return b
+
+
+def test_max_hap_length_fp32(ctx32):
+    b = _long_short_mix(31, 12, 300)
+    assert int(b.hap_lengths().max()) <= 4094
+    got, _ = ctx32.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp32")
+
+
+def test_max_hap_length_fp64(ctx64):
+    b = _long_short_mix(33, 8, 200)
+    got, _ = ctx64.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp64")
+
+
+def test_exact_max_hap_length(ctx32, ctx64):
+    b = synth.random_pairs_batch(35, 6, m_range=(1, 80), n_range=(4094, 4094))
+    ref = oracle.batch_log10(b)
+    _check(ctx32.compute_batch(b)[0], ref, "fp32")
+    _check(ctx64.compute_batch(b)[0], ref, "fp64")
+
+
+def test_hap_too_long_is_invalid_arg(ctx32):
+    b = synth.random_pairs_batch(36, 2, m_range=(5, 10), n_range=(4095, 4095))
+    with pytest.raises(phmm.PhmmError) as ei:
+        ctx32.compute_batch(b)
+    assert ei.value.code == -1
+
+
+def test_c4_reduced_fp64(ctx64):
+    """FP64 mode with 1500-column haplotypes (32-byte ring slots: the second launch class)."""
+    b = synth.config_batch("C4", n_regions=1)
+    got, _ = ctx64.compute_batch(b)
+    _check(got, oracle.batch_log10(b), "fp64")

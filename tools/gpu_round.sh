@@ -5,6 +5,6 @@ python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
 python bench.py --steps 10 --warmup 3 > gpurun_out/bench.json 2> gpurun_out/bench.err; tail -2 gpurun_out/bench.err; cat gpurun_out/bench.json
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
     python bench.py --steps 2 --warmup 1 --profile-steps --no-e2e --no-cpu-baseline > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:k_wavefront_f32 -s 1 -c 1 -o gpurun_out/prof_wf32 \
+ncu --set full --clock-control none --import-source on --kernel-name-base mangled -k regex:k_wavefrontIf -s 1 -c 1 -o gpurun_out/prof_wf32 \
     python bench.py --steps 1 --warmup 1 --profile-steps --no-e2e --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
 tail -1 gpurun_out/ncu_full.log

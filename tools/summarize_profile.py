@@ -50,7 +50,7 @@ want = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "sm__cycles_elapsed.avg.per_second"]
 vals = {}
 with open(f"{out_dir}/{tag}_ncu_wavefront_f32.txt", "w") as f:
-    f.write("# ncu --set full --clock-control none --import-source on -k regex:k_wavefront_f32 (C2, 1 launch)\n")
+    f.write("# ncu --set full --clock-control none --import-source on -k regex:k_wavefront (C2, 1 launch)\n")
     for w in want:
         if w in H:
             i = H.index(w)
@@ -69,7 +69,7 @@ def to_bytes(v, u):
 
 
 traffic = to_bytes(*vals["dram__bytes_read.sum"]) + to_bytes(*vals["dram__bytes_write.sum"])
-json.dump({"kernel": "k_wavefront_f32", "workload": "C2 (bench.py default), one launch",
+json.dump({"kernel": "k_wavefront<float>", "workload": "C2 (bench.py default), one launch",
            "dram_bytes_read_plus_write": traffic, "source": f"profiles/{tag}_ncu_wavefront_f32.txt"},
           open(f"{out_dir}/{tag}_wavefront_traffic.json", "w"), indent=1)
 try:
