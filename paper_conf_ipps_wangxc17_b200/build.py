@@ -40,8 +40,10 @@ def needs_build() -> bool:
     return any(os.path.getmtime(p) > t for p in _deps())
 
 
-def build(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
-    """Build libphmm.so (or a variant at ``out`` with extra -D ``defines``, for A/B runs)."""
+def build(force: bool = False, verbose: bool = False, out: str = None, defines=(), source_flags=None) -> str:
+    """Build libphmm.so (or a variant at ``out`` with extra -D ``defines`` and/or
+    per-source flags ``source_flags``, for A/B runs)."""
+    sflags = SOURCE_FLAGS if source_flags is None else source_flags
     target = out or LIB
     if not force and out is None and not needs_build():
         return LIB
@@ -49,7 +51,7 @@ def build(force: bool = False, verbose: bool = False, out: str = None, defines=(
     objs, log = [], []
     for src in SOURCES:
         obj = f"{tmp}.{os.path.basename(src)}.o"
-        cmd = ([nvcc()] + NVCC_FLAGS + SOURCE_FLAGS.get(os.path.basename(src), []) + [f"-D{d}" for d in defines]
+        cmd = ([nvcc()] + NVCC_FLAGS + sflags.get(os.path.basename(src), []) + [f"-D{d}" for d in defines]
                + ["-I", os.path.join(ROOT, "include"), "-c", "-o", obj, src])
         res = subprocess.run(cmd, capture_output=True, text=True)
         if res.returncode != 0:

@@ -91,7 +91,8 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
     const int f = nb * K - (m + 3);
     TBlock<T>* __restrict__ Tb = tab + item_tab_off[it];
     for (int row = lane; row < nb * K; row += 32) {
-      T al = 0, be = 0, de = 0, ep = 0, ze = 0, mu = 0;
+      // gamma = beta/alpha, delta, eps, zeta, mu, and alpha*P per haplotype code
+      T ga = 0, de = 0, ep = 0, ze = 0, mu = 0;
       T p5[5] = {0, 0, 0, 0, 0};
       if (row < f) {
         // Z row: all zero
@@ -101,13 +102,13 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
         const int64_t x = r0 + (row - f - 1);
         const T ei = err[qi[x] & 127], ed = err[qd[x] & 127], eg = err[qg[x] & 127], eb = err[q[x] & 127];
         const T sum = ei + ed;
-        al = (T)1 - (sum < (T)1 ? sum : (T)1);
-        be = (T)1 - eg;
+        const T al = (T)1 - (sum < (T)1 ? sum : (T)1);  // > 0.0065 after validation (R16)
+        ga = ((T)1 - eg) / al;
         de = ei;
         ep = eg;
         ze = ed;
         mu = eg;
-        const T pm = (T)1 - eb, px = eb / (T)3;
+        const T pm = al * ((T)1 - eb), px = al * (eb / (T)3);
         const uint8_t base = rb[x];
         p5[0] = (base == 'A' || base == 'N') ? pm : px;
         p5[1] = (base == 'C' || base == 'N') ? pm : px;
@@ -116,14 +117,14 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
         p5[4] = pm;  // haplotype 'N' matches everything
       } else if (row == f + m + 1) {  // S1: I = M(m,j) + I(m,j)
         de = 1; ep = 1; mu = 1;
-      } else {  // S2: M = I_S1(j-1), D = running sum
-        be = 1; ze = 1; mu = 1;
+      } else {  // S2: M = I_S1(j-1) (M_S1 = D_S1 = 0), D = running sum
+        ga = 1; ze = 1; mu = 1;
         p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = 1;
       }
       TBlock<T>& B = Tb[row / K];
       const int t = row % K;
-      B.coef[0][t] = al; B.coef[1][t] = be; B.coef[2][t] = de;
-      B.coef[3][t] = ep; B.coef[4][t] = ze; B.coef[5][t] = mu;
+      B.coef[0][t] = ga; B.coef[1][t] = de; B.coef[2][t] = ep;
+      B.coef[3][t] = ze; B.coef[4][t] = mu;
 #pragma unroll
       for (int k = 0; k < 5; ++k) B.prior[k][t] = p5[k];
     }

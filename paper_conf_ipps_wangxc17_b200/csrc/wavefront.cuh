@@ -126,13 +126,18 @@ template <typename V> __device__ __forceinline__ V vzero();
 template <> __device__ __forceinline__ v2f vzero<v2f>() { return 0ull; }
 template <> __device__ __forceinline__ v2d vzero<v2d>() { return v2d{0.0, 0.0}; }
 
-// per-block coefficient table: 6 transition fields + 5 prior codes, K rows each
+// per-block coefficient table: 5 transition fields + 5 prior codes, K rows each.
+// Eq. 6's match update P*(alpha*M + beta*(I + D)) is evaluated as
+// (alpha*P) * (M + gamma*(I + D)) with gamma = beta/alpha (alpha >= 0.0065 for every
+// validated read row, R16): the table holds alpha*P per code, so alpha and
+// beta leave the registers and one multiply per cell disappears.
+constexpr int WF_NCOEF = 5;
 template <typename T>
 struct alignas(16) TBlock {
-  T coef[6][WfT<T>::K];   // alpha, beta, delta, eps, zeta, mu
-  T prior[5][WfT<T>::K];  // P(row, code) for code = A, C, G, T, N
+  T coef[WF_NCOEF][WfT<T>::K];  // gamma, delta, eps, zeta, mu
+  T prior[5][WfT<T>::K];        // alpha * P(row, code) for code = A, C, G, T, N
 };
-static_assert(sizeof(TBlock<float>) == 11 * WF_KC * 16 && sizeof(TBlock<double>) == 11 * WF_KC * 16, "TBlock");
+static_assert(sizeof(TBlock<float>) == 10 * WF_KC * 16 && sizeof(TBlock<double>) == 10 * WF_KC * 16, "TBlock");
 
 template <typename T>
 struct WfArgs2 {
@@ -154,7 +159,7 @@ template <typename T>
 struct Lane {
   using V = typename WfT<T>::V;
   static constexpr int K = WfT<T>::K;
-  V al[K], be[K], de[K], ep[K], ze[K], mu[K];
+  V ga[K], de[K], ep[K], ze[K], mu[K];
   V M[K], I[K], D[K];
 };
 
@@ -175,7 +180,8 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
     // D(i,j) = zeta*M(i,j-1) + mu*D(i,j-1)
     L.D[u] = fma2(L.ze[u], L.M[u], mul2(L.mu[u], L.D[u]));
     // M(i,j) = P(i,j) * (alpha*M(i-1,j-1) + beta*(I(i-1,j-1) + D(i-1,j-1)))
-    const V x = fma2(L.al[u], md, mul2(L.be[u], add2(id, dd)));
+    //        = (alpha*P) * (M(i-1,j-1) + gamma*(I(i-1,j-1) + D(i-1,j-1)))
+    const V x = fma2(L.ga[u], add2(id, dd), md);
     L.M[u] = pk(prA[u] * lo(x), prB[u] * hi(x));
   }
   // I(i,j) = delta*M(i-1,j) + eps*I(i-1,j), rows ascending (a K-deep chain)
@@ -193,8 +199,7 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
 // tables are only touched through these, so no compiler reordering or aliasing games)
 __device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void ring_put3(uint32_t a, float x, float y, float z) {
-  asm volatile("st.shared.f32 [%0], %1;\n\tst.shared.f32 [%0+4], %2;\n\tst.shared.f32 [%0+8], %3;"
-               :: "r"(a), "f"(x), "f"(y), "f"(z) : "memory");
+  asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %3};" :: "r"(a), "f"(x), "f"(y), "f"(z) : "memory");
 }
 __device__ __forceinline__ void ring_get3(uint32_t a, float& x, float& y, float& z) {
   float w;
@@ -202,7 +207,7 @@ __device__ __forceinline__ void ring_get3(uint32_t a, float& x, float& y, float&
   (void)w;
 }
 __device__ __forceinline__ void ring_put3(uint32_t a, double x, double y, double z) {
-  asm volatile("st.shared.f64 [%0], %1;\n\tst.shared.f64 [%0+8], %2;\n\tst.shared.f64 [%0+16], %3;"
+  asm volatile("st.shared.v2.f64 [%0], {%1, %2};\n\tst.shared.f64 [%0+16], %3;"
                :: "r"(a), "d"(x), "d"(y), "d"(z) : "memory");
 }
 __device__ __forceinline__ void ring_get3(uint32_t a, double& x, double& y, double& z) {
@@ -240,17 +245,18 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   constexpr int PER = 16 / sizeof(T);  // values per 16-byte chunk
   if (have) {
     const uint4* __restrict__ s4 = reinterpret_cast<const uint4*>(A.tab + d.tab_blk);
-    union { uint4 u[6 * WF_KC]; T v[6][K]; } cw;
+    union { uint4 u[WF_NCOEF * WF_KC]; T v[WF_NCOEF][K]; } cw;
 #pragma unroll
-    for (int k = 0; k < 6 * WF_KC; ++k) cw.u[k] = __ldg(s4 + k);
+    for (int k = 0; k < WF_NCOEF * WF_KC; ++k) cw.u[k] = __ldg(s4 + k);
 #pragma unroll
-    for (int k = 0; k < 5 * WF_KC; ++k) sts16(tab_s + 512u * k, __ldg(s4 + 6 * WF_KC + k));  // prior[code][chunk]
+    for (int k = 0; k < 5 * WF_KC; ++k)  // prior[code][chunk]
+      sts16(tab_s + 512u * k, __ldg(s4 + WF_NCOEF * WF_KC + k));
     const int rrow = (d.flags >> WF_RROW_SHIFT) & 15;
 #pragma unroll
     for (int u = 0; u < K; ++u) {
-      L.al[u] = set_half<H>(L.al[u], cw.v[0][u]); L.be[u] = set_half<H>(L.be[u], cw.v[1][u]);
-      L.de[u] = set_half<H>(L.de[u], cw.v[2][u]); L.ep[u] = set_half<H>(L.ep[u], cw.v[3][u]);
-      L.ze[u] = set_half<H>(L.ze[u], cw.v[4][u]); L.mu[u] = set_half<H>(L.mu[u], cw.v[5][u]);
+      L.ga[u] = set_half<H>(L.ga[u], cw.v[0][u]); L.de[u] = set_half<H>(L.de[u], cw.v[1][u]);
+      L.ep[u] = set_half<H>(L.ep[u], cw.v[2][u]); L.ze[u] = set_half<H>(L.ze[u], cw.v[3][u]);
+      L.mu[u] = set_half<H>(L.mu[u], cw.v[4][u]);
       L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
       L.D[u] = set_half<H>(L.D[u], rrow == u ? d0 : (T)0);
     }
@@ -264,7 +270,7 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   }
 #pragma unroll
   for (int u = 0; u < K; ++u) {
-    L.al[u] = set_half<H>(L.al[u], (T)0); L.be[u] = set_half<H>(L.be[u], (T)0);
+    L.ga[u] = set_half<H>(L.ga[u], (T)0);
     L.de[u] = set_half<H>(L.de[u], (T)0); L.ep[u] = set_half<H>(L.ep[u], (T)0);
     L.ze[u] = set_half<H>(L.ze[u], (T)0); L.mu[u] = set_half<H>(L.mu[u], (T)0);
     L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
@@ -294,7 +300,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   Lane<T> L;
 #pragma unroll
   for (int u = 0; u < K; ++u) {
-    L.al[u] = L.be[u] = L.de[u] = L.ep[u] = L.ze[u] = L.mu[u] = vzero<V>();
+    L.ga[u] = L.de[u] = L.ep[u] = L.ze[u] = L.mu[u] = vzero<V>();
     L.M[u] = L.I[u] = L.D[u] = vzero<V>();
   }
   const uint32_t* pA = reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);  // next code word
@@ -311,9 +317,11 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
   int c31B = -(1 << 20);  // (uniform) column of virtual lane 63 (lane 31, half B)
   T rvM = 0, rvI = 0, rvD = 0;  // lane 31: ring slot for virtual lane 0's next column
-  BlkDesc dnA, dnB;  // next pass's block descriptors (prefetched)
+  BlkDesc dnA, dnB;  // descriptors of the lane's next blocks (loaded one pass ahead)
   dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.n = 1; dnA.flags = 0;
   dnB = dnA;
+  if (2 * lane < nblk) dnA = A.blk[s + 2 * lane];
+  if (2 * lane + 1 < nblk) dnB = A.blk[s + 2 * lane + 1];
 #ifdef PHMM_DBG_TRACE
   int tstep = 0;
 #endif
@@ -373,12 +381,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
       if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
         const int bA = q * 64 + 2 * lane, bB = bA + 1;
         const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
-        // this pass's descriptors were prefetched one pass ago (pass 0: loaded now)
-        BlkDesc dA = dnA, dB = dnB;
-        if (q == 0) {
-          if (hA) dA = A.blk[s + bA];
-          if (hB) dB = A.blk[s + bB];
-        }
+        const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
         if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S2 row: the last-row M+I sum (L20@2262)
         if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
         pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
