@@ -332,16 +332,19 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
 
   // launch classes: bins whose ring fits at full occupancy, then (if any) the longer bins
   const int slot = (int)ring_slot_bytes<T>();
-  auto P_of = [](int ncols) { return std::max(ncols + WF_G, WF_MIN_P); };
+  auto P_of = [](int ncols) { return wf_pass_len(ncols); };
   const int p_max = P_of(pi.max_ncols);
   int bps_full = 0;
-  CUDA_TRY(wf_occupancy<T>(WF_WARPS, wf_warp_smem<T>(WF_MIN_P + 4) * WF_WARPS, &bps_full));
+  CUDA_TRY(wf_occupancy<T>(WF_WARPS, wf_warp_smem<T>(wf_pass_len(0) + 4) * WF_WARPS, &bps_full));
   if (bps_full < 1) return PHMM_E_CUDA;
   const int64_t cta_budget = (int64_t)c->smem_per_sm / bps_full - c->smem_reserved;
   const int ring_full = (int)std::min<int64_t>(
       (cta_budget / WF_WARPS - (int64_t)wf_warp_smem<T>(0)) / slot, (int64_t)(c->smem_optin / WF_WARPS) / slot);
   int bin_cut = kMaxBins + 1;  // bins < bin_cut run in the full-occupancy launch
-  if (p_max + 4 > ring_full) bin_cut = std::max(0, (ring_full - 4 - WF_G) / c->bucket + 1);
+  if (p_max + 4 > ring_full) {
+    bin_cut = 0;
+    while (bin_cut <= kMaxBins && P_of(bin_cut * c->bucket) + 4 <= ring_full) ++bin_cut;
+  }
   struct Launch { int bin_lo, bin_hi, warps, ring_len, bps; };
   Launch L[2];
   int nl = 0;

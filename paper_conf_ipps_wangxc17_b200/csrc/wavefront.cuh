@@ -199,7 +199,8 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
 // tables are only touched through these, so no compiler reordering or aliasing games)
 __device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void ring_put3(uint32_t a, float x, float y, float z) {
-  asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %3};" :: "r"(a), "f"(x), "f"(y), "f"(z) : "memory");
+  asm volatile("st.shared.f32 [%0], %1;\n\tst.shared.f32 [%0+4], %2;\n\tst.shared.f32 [%0+8], %3;"
+               :: "r"(a), "f"(x), "f"(y), "f"(z) : "memory");
 }
 __device__ __forceinline__ void ring_get3(uint32_t a, float& x, float& y, float& z) {
   float w;
@@ -229,11 +230,16 @@ __device__ __forceinline__ void sts16(uint32_t a, const uint4 v) {
                : "memory");
 }
 
+// Steps per pass: every virtual lane sweeps its ncols columns plus the G-step stagger of
+// its switch group; P >= 72 keeps the ring slot of a column written (virtual lane 63)
+// before it is read (virtual lane 0 of the next pass).
+__host__ __device__ inline int wf_pass_len(int ncols) {
+  return (ncols + WF_G > WF_MIN_P) ? ncols + WF_G : WF_MIN_P;
+}
 // Haplotype code regions: 4 shifted copies per haplotype so that every lane reads its
 // codes as aligned 32-bit words, 4 columns at a time.
 __host__ __device__ inline int wf_hc_copy_len(int ncols) {
-  const int p = (ncols + WF_G > WF_MIN_P) ? ncols + WF_G : WF_MIN_P;
-  return ((int)WF_HC_FRONT + p + 24 + 3) & ~3;  // + prefetch distance
+  return ((int)WF_HC_FRONT + wf_pass_len(ncols) + 24 + 3) & ~3;  // + prefetch distance
 }
 
 // Load a block (or nothing) into half H of a lane. Returns the 32-bit-aligned code
@@ -294,7 +300,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   const int grp = lane / LPG;
   const int giA = 2 * (lane % LPG), giB = giA + 1;  // position of each half inside its group
   const T d0 = (T)ldexp(1.0, WfT<T>::kScaleExp) / (T)ncols;  // virtual row 0
-  const int P = max(ncols + G, WF_MIN_P);                     // multiple of 4 (ncols is)
+  const int P = wf_pass_len(ncols);                           // multiple of 4 (ncols is)
   const int npass = (nblk + 63) >> 6;
   const int copy_len = wf_hc_copy_len(ncols);
   Lane<T> L;
