@@ -18,41 +18,52 @@ __host__ __device__ inline int64_t wf_hc_region(int n, int bucket) {
   return 4 * (int64_t)wf_hc_copy_len(ncols_of(n, bucket));
 }
 
-__global__ void k_hap_codes_wf(const uint8_t* __restrict__ hap, const int64_t* __restrict__ hoff, int64_t n_haps,
-                               const int64_t* __restrict__ hc_off, int bucket, uint8_t* __restrict__ codes) {
-  const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+// One warp per haplotype: its code bytes (copy 0, PAD front and tail) are built once in
+// shared memory, then the 4 shifted copies are written as coalesced 32-bit words
+// (funnel shifts of two aligned words).
+constexpr int kHcThreads = 256;
+constexpr int kHcBuf = 4352;  // >= wf_hc_copy_len(ncols_of(kMaxHapLen, 64)) + 4
+__global__ void __launch_bounds__(kHcThreads) k_hap_codes_wf(const uint8_t* __restrict__ hap,
+                                                             const int64_t* __restrict__ hoff, int64_t n_haps,
+                                                             const int64_t* __restrict__ hc_off, int bucket,
+                                                             uint8_t* __restrict__ codes) {
+  __shared__ __align__(16) uint8_t sbuf[kHcThreads / 32][kHcBuf];
   const int lane = threadIdx.x & 31;
+  uint8_t* buf = sbuf[threadIdx.x >> 5];
+  const uint32_t* buf32 = reinterpret_cast<const uint32_t*>(buf);
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t h = warp; h < n_haps; h += nwarps) {
+  constexpr uint32_t kPadW = (uint32_t)(WF_PAD * WF_CB) * 0x01010101u;
+  for (int64_t h = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; h < n_haps; h += nwarps) {
     const int64_t h0 = hoff[h];
     const int n = (int)(hoff[h + 1] - h0);
     if (n < 1 || n > kMaxHapLen) continue;
     const int len = wf_hc_copy_len(ncols_of(n, bucket));  // multiple of 4, region start 4-aligned
+    __syncwarp();
+    for (int b = lane; b < len + 4; b += 32) {  // byte b of copy 0 = column b - WF_HC_FRONT
+      const int c = b - (int)WF_HC_FRONT;
+      uint32_t v = WF_PAD;
+      if (c >= 0 && c < n) {
+        switch (hap[h0 + c]) {
+          case 'A': v = 0; break;
+          case 'C': v = 1; break;
+          case 'G': v = 2; break;
+          case 'T': v = 3; break;
+          default: v = 4; break;  // 'N' (invalid bytes were rejected by validation)
+        }
+      } else if (c == n) {
+        v = 4;
+      }
+      buf[b] = (uint8_t)(v * WF_CB);
+    }
+    __syncwarp();
     uint32_t* dst = reinterpret_cast<uint32_t*>(codes + hc_off[h]);
     const int wpc = len >> 2;  // words per copy
-    for (int k = 0; k < 4; ++k) {
+    // copy k, word w = bytes [4w - k, 4w - k + 4) of copy 0 (PAD before byte 0)
+    for (int k = 0; k < 4; ++k)
       for (int w = lane; w < wpc; w += 32) {
-        uint32_t word = 0;
-#pragma unroll
-        for (int by = 0; by < 4; ++by) {
-          const int c = 4 * w + by - (int)WF_HC_FRONT - k;  // column of this byte in copy k
-          uint32_t v = WF_PAD;
-          if (c >= 0 && c < n) {
-            switch (hap[h0 + c]) {
-              case 'A': v = 0; break;
-              case 'C': v = 1; break;
-              case 'G': v = 2; break;
-              case 'T': v = 3; break;
-              default: v = 4; break;  // 'N' (invalid bytes were rejected by validation)
-            }
-          } else if (c == n) {
-            v = 4;
-          }
-          word |= (v * WF_CB) << (8 * by);
-        }
-        dst[k * wpc + w] = word;
+        const uint32_t lo = w > 0 ? buf32[w - 1] : kPadW, hi = buf32[w];
+        dst[k * wpc + w] = __funnelshift_rc(lo, hi, 8 * (4 - k));
       }
-    }
   }
 }
 
