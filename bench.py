@@ -20,6 +20,7 @@ the three M/I/D updates of one cell count as one cell update).
 from __future__ import annotations
 
 import argparse
+import glob
 import json
 import os
 import statistics
@@ -48,6 +49,29 @@ WORKLOADS = {
     "C5": "C5-shaped shard: mixed 100-250 bp reads, N ~ U{m..2m}",
 }
 DEFAULT_REGIONS = {"C2": 8192, "C3": 4096, "C4": 256, "C5": 8192}
+
+
+def _ncu_traffic(workload):
+    """dram__bytes_read.sum + dram__bytes_write.sum of one k_wavefront<float> launch from the
+    latest committed ncu --set full capture (profiles/r*_wavefront_traffic.json), for the
+    workload that capture was taken on (C2); None otherwise."""
+    if workload != "C2":
+        return None, None
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "r*_wavefront_traffic.json")))
+    for fn in reversed(files):
+        try:
+            d = json.load(open(fn))
+        except (OSError, ValueError):
+            continue
+        if d.get("kernel") == "k_wavefront<float>":
+            return float(d["dram_bytes_read_plus_write"]), os.path.relpath(fn, ROOT)
+    return None, None
+
+
+def _algorithmic_bytes(b):
+    """Bytes the FP32 pass must move at least once: read bases + 4 quality
+    arrays, haplotype bases, pair indices, one float result per pair."""
+    return int(5 * b.read_bases.size + b.hap_bases.size + 8 * b.n_pairs + 4 * b.n_pairs)
 
 
 def _measured_peaks():
@@ -322,8 +346,11 @@ def main():
     wf = float(np.mean(wf_ms)) if wf_ms else float("nan")
     achieved = cells / (wf / 1e3) / 1e9 if wf > 0 else None
     sm_run = clocks.get("sm_mhz") if clocks else None
+    traffic, traffic_src = _ncu_traffic(args.workload if args.regions is None else None)
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak_gcups, "unit": "GCUPS",
-                "frac": (achieved / peak_gcups) if achieved else None, "traffic": None,
+                "frac": (achieved / peak_gcups) if achieved else None, "traffic": traffic,
+                "traffic_unit": "bytes per launch (dram read + write)", "traffic_source": traffic_src,
+                "algorithmic_bytes_per_launch": _algorithmic_bytes(batch),
                 "kernel": "k_wavefront<float>",
                 "peak_basis": f"{nsm} SM x {FP32_LANES_PER_SM} FP32 lanes x {sm_max:.0f} MHz (MEASURED_PEAKS sm_max_mhz)"
                               f" / {FP32_OPS_PER_CELL} FP32-pipe ops per cell (3 FFMA + 4 FMUL + 1 FADD)",

@@ -50,7 +50,7 @@ want = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "sm__cycles_elapsed.avg.per_second"]
 vals = {}
 with open(f"{out_dir}/{tag}_ncu_wavefront_f32.txt", "w") as f:
-    f.write("# ncu --set full --clock-control none --import-source on -k regex:k_wavefront (C2, 1 launch)\n")
+    f.write("# ncu --set full --clock-control none --import-source on -k regex:k_wavefrontIf (k_wavefront<float>, C2, 1 launch)\n")
     for w in want:
         if w in H:
             i = H.index(w)
@@ -72,6 +72,26 @@ traffic = to_bytes(*vals["dram__bytes_read.sum"]) + to_bytes(*vals["dram__bytes_
 json.dump({"kernel": "k_wavefront<float>", "workload": "C2 (bench.py default), one launch",
            "dram_bytes_read_plus_write": traffic, "source": f"profiles/{tag}_ncu_wavefront_f32.txt"},
           open(f"{out_dir}/{tag}_wavefront_traffic.json", "w"), indent=1)
+# ---- FP64 rescue kernel capture (if present) and per-opcode stall summaries
+import os
+for rep, name in (("gpurun_out/prof_wf64.ncu-rep", "k_wavefront<double>"),):
+    if not os.path.exists(rep):
+        continue
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rr = list(csv.reader(raw.splitlines()))
+    H, U, V = rr[0], rr[1], rr[2]
+    with open(f"{out_dir}/{tag}_ncu_wavefront_f64.txt", "w") as f:
+        f.write(f"# ncu --set full --clock-control none -k regex:k_wavefrontId ({name}, C2 rescue pass, 1 launch)\n")
+        for w in want + ["sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
+                         "sm__inst_executed_pipe_fp64.avg.pct_of_peak_sustained_active"]:
+            if w in H:
+                i = H.index(w)
+                f.write(f"{w} = {V[i]} {U[i]}\n")
+for rep, sfx in (("gpurun_out/prof_wf32.ncu-rep", "f32"), ("gpurun_out/prof_wf64.ncu-rep", "f64")):
+    if os.path.exists(rep):
+        st = subprocess.run([sys.executable, "tools/ncu_stalls.py", rep, "25"], capture_output=True, text=True).stdout
+        open(f"{out_dir}/{tag}_stalls_wavefront_{sfx}.txt", "w").write(
+            f"# tools/ncu_stalls.py {rep} (warp-stall samples per SASS instruction)\n" + st)
 try:
     b = json.load(open("gpurun_out/bench.json"))
     json.dump(b, open(f"{out_dir}/{tag}_bench.json", "w"), indent=1)
