@@ -40,6 +40,43 @@ def needs_build() -> bool:
     return any(os.path.getmtime(p) > t for p in _deps())
 
 
+LATENCY_LIB = os.path.join(PKG, "liblatency.so")
+LATENCY_SRC = os.path.join(CSRC, "latency.cu")
+# Design-A ablation of the wavefront kernel (row-above exchange through a shared-memory
+# line buffer instead of __shfl_sync)
+XSMEM_LIB = os.path.join(PKG, "libphmm_xsmem.so")
+
+
+def build_latency(force: bool = False) -> str:
+    """liblatency.so: the paper's Listing 1 latency microbenchmarks (not on the hot path)."""
+    if not force and os.path.exists(LATENCY_LIB) and os.path.getmtime(LATENCY_LIB) >= max(
+            os.path.getmtime(LATENCY_SRC), os.path.getmtime(os.path.abspath(__file__))):
+        return LATENCY_LIB
+    tmp = LATENCY_LIB + f".tmp{os.getpid()}"
+    cmd = [nvcc(), "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
+           "-Xcompiler", "-fPIC", "-shared", "-o", tmp, LATENCY_SRC]
+    res = subprocess.run(cmd, capture_output=True, text=True)
+    if res.returncode != 0:
+        sys.stderr.write(res.stdout + res.stderr)
+        raise RuntimeError("nvcc failed building liblatency.so")
+    os.replace(tmp, LATENCY_LIB)
+    return LATENCY_LIB
+
+
+def build_xsmem(force: bool = False) -> str:
+    """libphmm_xsmem.so: libphmm with the shared-memory (design A) row exchange."""
+    if not force and os.path.exists(XSMEM_LIB) and os.path.getmtime(XSMEM_LIB) >= max(
+            os.path.getmtime(p) for p in _deps()):
+        return XSMEM_LIB
+    return build(out=XSMEM_LIB, defines=["PHMM_XCHG_SMEM=1"])
+
+
+def build_all(force: bool = False, verbose: bool = False) -> None:
+    build(force=force, verbose=verbose)
+    build_xsmem(force=force)
+    build_latency(force=force)
+
+
 def build(force: bool = False, verbose: bool = False, out: str = None, defines=(), source_flags=None) -> str:
     """Build libphmm.so (or a variant at ``out`` with extra -D ``defines`` and/or
     per-source flags ``source_flags``, for A/B runs)."""
@@ -75,5 +112,5 @@ def build(force: bool = False, verbose: bool = False, out: str = None, defines=(
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose=True)
+    build_all(force="--force" in sys.argv, verbose=True)
     print(LIB)

@@ -46,6 +46,9 @@ __device__ int g_trace_steps;
 #ifndef PHMM_F32_K
 #define PHMM_F32_K 8
 #endif
+#ifndef PHMM_XCHG_SMEM
+#define PHMM_XCHG_SMEM 0  // 1: design-A ablation build (row exchange through shared memory)
+#endif
 
 constexpr int WF_G = 8;           // virtual lanes per switch group
 constexpr int WF_NCODE = 6;       // A C G T N PAD
@@ -288,8 +291,8 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
 
 // One warp streams through blocks [s, s+nblk) of one bin (ncols columns each).
 template <typename T>
-__device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s, int lane,
-                                          int64_t s, int nblk, int ncols, bool trace = false) {
+__device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s, uint32_t xbuf_s,
+                                          int lane, int64_t s, int nblk, int ncols, bool trace = false) {
   using V = typename WfT<T>::V;
   constexpr int K = WfT<T>::K;
   constexpr int PER = 16 / sizeof(T);
@@ -352,12 +355,25 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     const T sD = is31 ? rvD : d3b;
     if (is31 && (unsigned)(c31B + 1) <= (unsigned)ncols)  // -1 <= c31B < ncols
       ring_put3(ring_s + RS * (uint32_t)(c31B + 1), m3b, i3b, d3b);
-    __syncwarp();
     dgM = upM; dgI = upI; dgD = upD;
     // next step: half A's row above = lane-1's half B; half B's row above = this lane's half A
+#if PHMM_XCHG_SMEM
+    // design A (Listing 2a, L20@44): write, synchronise, read through a
+    // shared-memory line buffer (one slot per lane) instead of the shuffle
+    ring_put3(xbuf_s + RS * (uint32_t)lane, sM, sI, sD);
+    __syncwarp();
+    T xM, xI, xD;
+    ring_get3(xbuf_s + RS * (uint32_t)src, xM, xI, xD);
+    __syncwarp();
+    upM = pk(xM, m3a);
+    upI = pk(xI, i3a);
+    upD = pk(xD, d3a);
+#else
+    __syncwarp();
     upM = pk(__shfl_sync(0xffffffffu, sM, src), m3a);
     upI = pk(__shfl_sync(0xffffffffu, sI, src), i3a);
     upD = pk(__shfl_sync(0xffffffffu, sD, src), d3a);
+#endif
 #if defined(PHMM_DBG_TRACE) && defined(PHMM_DEFINE_WF)
     if (sizeof(T) == 4 && trace && tstep < 4096) {
       float* t = g_trace + ((size_t)tstep * 32 + lane) * 6;
@@ -416,8 +432,10 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 // from the -O0/-O1 builds and from the CPU model of the schedule).
 // phmm_lib.cu reaches them through these host functions.
 // shared memory of one warp: its prior tables and its ring
-template <typename T> size_t wf_warp_smem(int ring_len) {
-  return (size_t)2 * WF_NCODE * WF_KC * 32 * 16 + (size_t)ring_len * ring_slot_bytes<T>();
+template <typename T> __host__ __device__ size_t wf_warp_smem(int ring_len) {
+  // prior tables, ring, and (design-A ablation only) the exchange line buffer
+  return (size_t)2 * WF_NCODE * WF_KC * 32 * 16 +
+         (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) * ring_slot_bytes<T>();
 }
 template <typename T> cudaError_t wf_occupancy(int warps, size_t smem, int* blocks_per_sm);
 template <typename T>
@@ -434,11 +452,12 @@ __global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfAr
   const int wib = threadIdx.x >> 5;
   // per warp: prior tables [2 halves][6 codes][WF_KC chunks][32 lanes] x 16 B, then the ring
   constexpr uint32_t kTabBytes = 2 * WF_NCODE * WF_KC * 32 * 16;
-  const uint32_t per_warp = kTabBytes + (uint32_t)A.ring_len * ring_slot_bytes<T>();
+  const uint32_t per_warp = (uint32_t)wf_warp_smem<T>(A.ring_len);
   unsigned char* base = smem_raw + (size_t)wib * per_warp;
   for (uint32_t i = 4 * lane; i < per_warp; i += 128) *reinterpret_cast<uint32_t*>(base + i) = 0u;
   __syncwarp();
   const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
+  const uint32_t xbuf_s = ring_s + (uint32_t)A.ring_len * ring_slot_bytes<T>();  // design A only
   // work item it of the launch: chunk k of bin b (binary search in item_start)
   const unsigned long long it0 = A.item_start[A.bin_lo], it1 = A.item_start[A.bin_hi];
   while (true) {
@@ -470,7 +489,7 @@ __global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfAr
     s = advance(s);
     e = (e >= b1) ? b1 : advance(e);
     if (e <= s) continue;
-    wf_stream<T>(A, ptab_s, ring_s, lane, s, (int)(e - s), bin * A.bucket, it == 0);
+    wf_stream<T>(A, ptab_s, ring_s, xbuf_s, lane, s, (int)(e - s), bin * A.bucket, it == 0);
     __syncwarp();
   }
 }
