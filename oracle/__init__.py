@@ -1,4 +1,4 @@
-"""PairHMM forward ORACLE -- test infrastructure only.
+"""PairHMM forward and Smith-Waterman ORACLES -- test infrastructure only.
 
 Only ``tests/``, ``__graft_entry__.smoke()`` and the ``cpu_baseline`` /
 ``--impl reference`` legs of ``bench.py`` may import anything from this
@@ -11,4 +11,8 @@ Modules:
                       (``phmm_oracle.c``), built with gcc on first use.
   ``oracle.brute`` -- explicit enumeration of every HMM path (Fractions or
                       mpmath), the independent pin for the DP on tiny inputs.
+  ``oracle.sw``    -- ctypes binding of the plain-C Smith-Waterman oracle
+                      (``sw_oracle.c``: Eq. 5 literally and in its running-max form,
+                      end cell over the last row and column, traceback).
+  ``oracle.sw_brute`` -- explicit enumeration of every Eq. 5 move path (tiny inputs).
 """
