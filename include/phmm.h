@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define PHMM_ABI_VERSION 1
+#define PHMM_ABI_VERSION 2
 
 typedef struct phmm_ctx phmm_ctx; /* opaque */
 
@@ -164,6 +164,59 @@ phmm_status phmm_get_stats(const phmm_ctx* ctx, phmm_stats* out);
 
 /* ABI version of the loaded library (PHMM_ABI_VERSION). */
 int phmm_abi_version(void);
+
+/* ======================================================================
+ * Smith-Waterman, HaplotypeCaller variant (the paper's second workload,
+ * PAPER.md Eq. 5, L16@3413, §III-B; readings R20-R25 in
+ * DESIGN.md §12). Integer scores:
+ *   H(i,0) = H(0,j) = 0,
+ *   H(i,j) = max{0, H(i-1,j-1) + s(a_i,b_j), max_k H(i-k,j) + W_k, max_l H(i,j-l) + W_l}
+ * for rows i = 1..M of the "ref" sequence a and columns j = 1..N of the "alt"
+ * sequence b; s = match if the bytes are equal else mismatch; W_k = gap_open +
+ * (k-1)*gap_extend. Ties: diagonal, then horizontal, then vertical; within a
+ * direction the longest gap; H = 0 from the 0 term when every other term is
+ * negative (the traceback stops there). The end cell is the maximum of row M and
+ * column N ("the cell with the maximal value in the last row and column",
+ * L16@3960; ties: smallest |i-j|, then largest i+j, then largest i); the alignment
+ * is traced back from it until a 0-term cell or row/column 0.
+ * ====================================================================== */
+typedef struct {
+  int32_t match;       /* > 0 */
+  int32_t mismatch;    /* <= match */
+  int32_t gap_open;    /* W_1, <= gap_extend */
+  int32_t gap_extend;  /* <= 0 */
+} phmm_sw_params;      /* HaplotypeCaller: {200, -150, -260, -11} */
+
+typedef struct {
+  const uint8_t* ref_bases;    /* concatenated rows sequences, 'A','C','G','T','N' */
+  const int64_t* ref_offsets;  /* n_refs + 1; 1 <= M <= 32767 per task */
+  int64_t n_refs;
+  const uint8_t* alt_bases;    /* concatenated column sequences */
+  const int64_t* alt_offsets;  /* n_alts + 1; 1 <= N <= 4096 per task */
+  int64_t n_alts;
+  const int32_t* tasks;        /* 2 * n_tasks: (ref_idx, alt_idx) */
+  int64_t n_tasks;
+  int64_t total_ref_bases;     /* = ref_offsets[n_refs] */
+  int64_t total_alt_bases;     /* = alt_offsets[n_alts] */
+} phmm_sw_batch;
+
+/*
+ * Align every task. out_res: n_tasks x 6 int32 per task, in task order:
+ *   score, end_i, end_j (1-based end cell), start_i, start_j (first aligned cell;
+ *   end + 1 for an empty alignment), n_ops.
+ * out_ops: CIGAR runs (len << 4 | op; op 0 = 'M', 1 = 'I' (gap in the ref row
+ * sequence: consumes alt bases), 2 = 'D' (consumes ref bases)), from start to end,
+ * the tasks' runs back to back in task order: task t's start at element
+ * sum_{t' < t} n_ops[t']. Capacity: sum_t (M_t + N_t) uint32 always suffices.
+ * Host variant: caller-owned host buffers, returns when they are written. Errors: PHMM_E_INVALID_ARG (NULL pointers, sizes, parameters
+ * outside the ranges above, M or N too long), PHMM_E_INVALID_BASE, PHMM_E_EMPTY_SEQ,
+ * PHMM_E_INDEX, PHMM_E_CUDA, PHMM_E_OOM; outputs are untouched on error.
+ */
+phmm_status phmm_sw_align_batch(phmm_ctx* ctx, const phmm_sw_batch* b, const phmm_sw_params* p,
+                                int32_t* out_res, uint32_t* out_ops);
+/* Device-buffer variant: every array in *b, dev_res and dev_ops are device pointers. */
+phmm_status phmm_sw_align_batch_dev(phmm_ctx* ctx, const phmm_sw_batch* b, const phmm_sw_params* p,
+                                    int32_t* dev_res, uint32_t* dev_ops);
 
 #ifdef __cplusplus
 }

@@ -19,6 +19,7 @@
 #include "../../include/phmm.h"
 #include "phmm_device.cuh"
 #include "stream_prep.cuh"
+#include "sw.cuh"
 
 using namespace phmm;
 
@@ -30,6 +31,9 @@ enum BufId {
   B_PAIR_BIN, B_PAIR_NB, B_BINS, B_ITEM_NB, B_ITEM_OFF, B_SCAN_TMP,
   B_TAB32, B_TAB64, B_BLK, B_OUT32, B_OUT64, B_RLIST, B_ITEM_READ, B_PAIR_ITEM,
   B_OUT_LOG10, B_OUT_STATUS, B_HNC, B_HC_OFF,
+  B_SW_REF, B_SW_ROFF, B_SW_ALT, B_SW_AOFF, B_SW_TASKS, B_SW_RES, B_SW_OPS,  // SW host-variant staging
+  B_SW_BTSZ, B_SW_BTOFF, B_SW_OPCAP, B_SW_OPOFF, B_SW_BT, B_SW_KEYS, B_SW_VALS, B_SW_OPTMP, B_SW_NOPS,
+  B_SW_NOPOFF,
   B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_COUNT
 };
 
@@ -67,6 +71,7 @@ struct phmm_ctx {
   int smem_per_sm = 0, smem_reserved = 0, smem_optin = 0;  // bytes (device attributes)
   Scalars* host_scal = nullptr;  // pinned
   int64_t* host_sizes = nullptr;  // pinned, 2 values
+  int64_t sw_ops_cap = 0;         // last SW call: sum over tasks of M + N
   cudaEvent_t ev[kEvents] = {};
   phmm_stats st{};
   int launches = 0;
@@ -497,6 +502,127 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   return PHMM_OK;
 }
 
+
+// ============================================================ Smith-Waterman (§8f row 2)
+struct SwDev {
+  const uint8_t *ref, *alt;
+  const int64_t *roff, *aoff;
+  const int32_t* tasks;
+  int64_t n_refs, n_alts, n_tasks, n_rb, n_ab;
+};
+
+phmm_status sw_check_args(const phmm_sw_batch* b, const phmm_sw_params* p) {
+  if (!b || !p) return PHMM_E_INVALID_ARG;
+  if (b->n_refs < 0 || b->n_alts < 0 || b->n_tasks < 0) return PHMM_E_INVALID_ARG;
+  if (b->n_tasks > 0x7fffffffLL || b->n_refs > 0x7fffffffLL || b->n_alts > 0x7fffffffLL) return PHMM_E_INVALID_ARG;
+  if (p->match <= 0 || p->mismatch > p->match || p->gap_extend > 0 || p->gap_open > p->gap_extend)
+    return PHMM_E_INVALID_ARG;
+  // |score| <= match * 4096 and gap totals stay far from int32 overflow
+  if (p->match > (1 << 18) || p->mismatch < -(1 << 18) || p->gap_open < -(1 << 18)) return PHMM_E_INVALID_ARG;
+  if (b->n_tasks == 0) return PHMM_OK;
+  if (!b->tasks || !b->ref_offsets || !b->alt_offsets) return PHMM_E_INVALID_ARG;
+  if (b->total_ref_bases < 0 || b->total_alt_bases < 0) return PHMM_E_INVALID_ARG;
+  if (b->total_ref_bases > 0 && !b->ref_bases) return PHMM_E_INVALID_ARG;
+  if (b->total_alt_bases > 0 && !b->alt_bases) return PHMM_E_INVALID_ARG;
+  return PHMM_OK;
+}
+
+int64_t ops_total_cap(const phmm_ctx* c, const int64_t*, int64_t) { return c->sw_ops_cap; }
+
+phmm_status sw_compute_dev(phmm_ctx* c, const SwDev& d, const phmm_sw_params* prm, int32_t* dev_res,
+                           uint32_t* dev_ops) {
+  cudaStream_t s = c->stream;
+  c->st = phmm_stats{};
+  c->st.n_pairs = d.n_tasks;
+  if (d.n_tasks == 0) return PHMM_OK;
+  Scalars* scal;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
+  if (d.n_rb > 0) {
+    k_validate_haps<<<grid_for(c, d.n_rb), kThreads, 0, s>>>(d.ref, d.n_rb, &scal->err);
+    LAUNCHED(c);
+  }
+  if (d.n_ab > 0) {
+    k_validate_haps<<<grid_for(c, d.n_ab), kThreads, 0, s>>>(d.alt, d.n_ab, &scal->err);
+    LAUNCHED(c);
+  }
+  k_validate_offsets<<<grid_for(c, d.n_refs + 1), kThreads, 0, s>>>(d.roff, d.n_refs, d.n_rb, &scal->err);
+  LAUNCHED(c);
+  k_validate_offsets<<<grid_for(c, d.n_alts + 1), kThreads, 0, s>>>(d.aoff, d.n_alts, d.n_ab, &scal->err);
+  LAUNCHED(c);
+  const int64_t n = d.n_tasks;
+  int64_t *bt_sz, *bt_off, *op_cap, *op_off;
+  ST_TRY(ws(c, B_SW_BTSZ, (size_t)n + 1, &bt_sz));
+  ST_TRY(ws(c, B_SW_BTOFF, (size_t)n + 1, &bt_off));
+  ST_TRY(ws(c, B_SW_OPCAP, (size_t)n + 1, &op_cap));
+  ST_TRY(ws(c, B_SW_OPOFF, (size_t)n + 1, &op_off));
+  k_sw_sizes<<<grid_for(c, n), kThreads, 0, s>>>(d.tasks, n, d.roff, d.n_refs, d.aoff, d.n_alts, bt_sz, op_cap,
+                                                  reinterpret_cast<int64_t*>(&scal->cells), &scal->max_ncols,
+                                                  &scal->err);
+  LAUNCHED(c);
+  size_t scan_bytes = 0, sort_bytes = 0;
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, bt_sz, bt_off, n + 1, s));
+  uint64_t* keys;
+  int32_t* vals;
+  ST_TRY(ws(c, B_SW_KEYS, (size_t)2 * n, &keys));
+  ST_TRY(ws(c, B_SW_VALS, (size_t)2 * n, &vals));
+  CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, keys + n, vals, vals + n, n, 0, 64, s));
+  unsigned char* tmp;
+  ST_TRY(ws(c, B_SORT_TMP, std::max(scan_bytes, sort_bytes), &tmp));
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, scan_bytes, bt_sz, bt_off, n + 1, s));
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, scan_bytes, op_cap, op_off, n + 1, s));
+  c->launches += 2;
+  CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+  int64_t* hsz = c->host_sizes;
+  CUDA_TRY(cudaMemcpyAsync(&hsz[0], bt_off + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(&hsz[1], op_off + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  if (c->host_scal->err) return map_err(c->host_scal->err);
+  const int64_t total_bt = hsz[0];
+  c->sw_ops_cap = hsz[1];
+  const int max_n = c->host_scal->max_ncols;
+  c->st.cells = (int64_t)c->host_scal->cells;
+  int16_t* bt;
+  ST_TRY(ws(c, B_SW_BT, (size_t)total_bt, &bt));
+  // largest tasks first (persistent warps: the tail is the smallest tasks)
+  k_sw_keys<<<grid_for(c, n), kThreads, 0, s>>>(d.tasks, n, d.roff, d.aoff, keys, vals);
+  LAUNCHED(c);
+  CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sort_bytes, keys, keys + n, vals, vals + n, n, 0, 64, s));
+  ++c->launches;
+
+  SwArgs A;
+  A.ref = d.ref; A.ref_off = d.roff; A.alt = d.alt; A.alt_off = d.aoff; A.tasks = d.tasks;
+  A.order = vals + n; A.n_tasks = n; A.bt_off = bt_off; A.bt = bt; A.res = dev_res;
+  A.counter = &scal->item_counter[0];
+  A.p = SwParams{prm->match, prm->mismatch, prm->gap_open, prm->gap_extend};
+  A.max_n = max_n;
+  const size_t per_warp = (size_t)(max_n + 1) * 12 + (size_t)((max_n + 15) & ~15);
+  const size_t smem = per_warp * SW_WARPS;
+  CUDA_TRY(cudaFuncSetAttribute(k_sw_fill, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int bps = 0;
+  CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_sw_fill, SW_WARPS * 32, smem));
+  if (bps < 1) return PHMM_E_INVALID_ARG;
+  CUDA_TRY(cudaMemsetAsync(A.counter, 0, sizeof(unsigned int), s));
+  ev_record(c, EV_WF0);
+  k_sw_fill<<<(unsigned)(c->nsm * bps), SW_WARPS * 32, smem, s>>>(A);
+  LAUNCHED(c);
+  ev_record(c, EV_WF1);
+  // traceback into capacity-laid-out scratch, then pack the runs back to back
+  uint32_t* ops_tmp;
+  int64_t *nops, *nops_off;
+  ST_TRY(ws(c, B_SW_OPTMP, (size_t)std::max<int64_t>(ops_total_cap(c, op_off, n), 1), &ops_tmp));
+  ST_TRY(ws(c, B_SW_NOPS, (size_t)n + 1, &nops));
+  ST_TRY(ws(c, B_SW_NOPOFF, (size_t)n + 1, &nops_off));
+  k_sw_traceback<<<grid_for(c, n), 128, 0, s>>>(A, op_off, ops_tmp, nops);
+  LAUNCHED(c);
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, scan_bytes, nops, nops_off, n + 1, s));
+  ++c->launches;
+  k_sw_compact<<<grid_for(c, n * 32), kThreads, 0, s>>>(ops_tmp, op_off, nops_off, n, dev_ops);
+  LAUNCHED(c);
+  ev_record(c, EV_FIN);
+  return PHMM_OK;
+}
+
 phmm_status check_batch_args(const phmm_batch* b) {
   if (!b) return PHMM_E_INVALID_ARG;
   if (b->n_reads < 0 || b->n_haps < 0 || b->n_pairs < 0) return PHMM_E_INVALID_ARG;
@@ -723,6 +849,105 @@ phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log
   CUDA_TRY(cudaStreamSynchronize(s));
   finish_stats(c);
   c->st.ms_h2d = ev_ms(c, EV_START, EV_H2D);
+  c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
+  return PHMM_OK;
+}
+
+phmm_status phmm_sw_align_batch_dev(phmm_ctx* c, const phmm_sw_batch* b, const phmm_sw_params* p, int32_t* dev_res,
+                                    uint32_t* dev_ops) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  ST_TRY(sw_check_args(b, p));
+  if (b->n_tasks > 0 && (!dev_res || !dev_ops)) return PHMM_E_INVALID_ARG;
+  if (cudaSetDevice(c->device) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  c->launches = 0;
+  SwDev d{b->ref_bases, b->alt_bases, b->ref_offsets, b->alt_offsets, b->tasks, b->n_refs, b->n_alts, b->n_tasks,
+          b->total_ref_bases, b->total_alt_bases};
+  ev_record(c, EV_START);
+  ev_record(c, EV_H2D);
+  phmm_status st = sw_compute_dev(c, d, p, dev_res, dev_ops);
+  if (st != PHMM_OK) {
+    cudaStreamSynchronize(c->stream);
+    cudaGetLastError();
+    return st;
+  }
+  ev_record(c, EV_END);
+  CUDA_TRY(cudaStreamSynchronize(c->stream));
+  c->st.kernel_launches = c->launches;
+  c->st.ms_total = ev_ms(c, EV_START, EV_END);
+  c->st.ms_wavefront = ev_ms(c, EV_WF0, EV_WF1);
+  c->st.ms_finalize = ev_ms(c, EV_WF1, EV_FIN);
+  c->st.ms_prep = ev_ms(c, EV_H2D, EV_WF0);
+  c->st.ms_h2d = c->st.ms_d2h = 0.f;
+  return PHMM_OK;
+}
+
+phmm_status phmm_sw_align_batch(phmm_ctx* c, const phmm_sw_batch* b, const phmm_sw_params* p, int32_t* out_res,
+                                uint32_t* out_ops) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  ST_TRY(sw_check_args(b, p));
+  if (b->n_tasks > 0 && (!out_res || !out_ops)) return PHMM_E_INVALID_ARG;
+  if (cudaSetDevice(c->device) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  c->launches = 0;
+  if (b->n_tasks == 0) {
+    c->st = phmm_stats{};
+    return PHMM_OK;
+  }
+  if (b->ref_offsets[b->n_refs] != b->total_ref_bases || b->alt_offsets[b->n_alts] != b->total_alt_bases)
+    return PHMM_E_INVALID_ARG;
+  // output capacity: sum over tasks of M + N (indices checked here, lengths on the device)
+  int64_t ops_total = 0;
+  for (int64_t t = 0; t < b->n_tasks; ++t) {
+    const int32_t r = b->tasks[2 * t], a = b->tasks[2 * t + 1];
+    if (r < 0 || r >= b->n_refs || a < 0 || a >= b->n_alts) return PHMM_E_INDEX;
+    ops_total += (b->ref_offsets[r + 1] - b->ref_offsets[r]) + (b->alt_offsets[a + 1] - b->alt_offsets[a]);
+  }
+  cudaStream_t s = c->stream;
+  uint8_t *ref, *alt;
+  int64_t *roff, *aoff;
+  int32_t *tasks, *res;
+  uint32_t* ops;
+  const size_t nr = (size_t)b->total_ref_bases, na = (size_t)b->total_alt_bases;
+  ST_TRY(ws(c, B_SW_REF, nr, &ref));
+  ST_TRY(ws(c, B_SW_ALT, na, &alt));
+  ST_TRY(ws(c, B_SW_ROFF, (size_t)b->n_refs + 1, &roff));
+  ST_TRY(ws(c, B_SW_AOFF, (size_t)b->n_alts + 1, &aoff));
+  ST_TRY(ws(c, B_SW_TASKS, (size_t)b->n_tasks * 2, &tasks));
+  ST_TRY(ws(c, B_SW_RES, (size_t)b->n_tasks * 6, &res));
+  ST_TRY(ws(c, B_SW_OPS, (size_t)std::max<int64_t>(ops_total, 1), &ops));
+  ev_record(c, EV_START);
+  if (nr) CUDA_TRY(cudaMemcpyAsync(ref, b->ref_bases, nr, cudaMemcpyHostToDevice, s));
+  if (na) CUDA_TRY(cudaMemcpyAsync(alt, b->alt_bases, na, cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(roff, b->ref_offsets, sizeof(int64_t) * (b->n_refs + 1), cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(aoff, b->alt_offsets, sizeof(int64_t) * (b->n_alts + 1), cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(tasks, b->tasks, sizeof(int32_t) * 2 * b->n_tasks, cudaMemcpyHostToDevice, s));
+  ev_record(c, EV_H2D);
+  SwDev d{ref, alt, roff, aoff, tasks, b->n_refs, b->n_alts, b->n_tasks, (int64_t)nr, (int64_t)na};
+  phmm_status st = sw_compute_dev(c, d, p, res, ops);
+  if (st != PHMM_OK) {
+    cudaStreamSynchronize(s);
+    cudaGetLastError();
+    return st;
+  }
+  ev_record(c, EV_D2H);
+  CUDA_TRY(cudaMemcpyAsync(out_res, res, sizeof(int32_t) * 6 * b->n_tasks, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  int64_t used = 0;  // packed runs: only these travel back
+  for (int64_t t = 0; t < b->n_tasks; ++t) used += out_res[6 * t + 5];
+  if (used > 0) CUDA_TRY(cudaMemcpyAsync(out_ops, ops, sizeof(uint32_t) * used, cudaMemcpyDeviceToHost, s));
+  ev_record(c, EV_END);
+  CUDA_TRY(cudaStreamSynchronize(s));
+  c->st.kernel_launches = c->launches;
+  c->st.ms_total = ev_ms(c, EV_START, EV_END);
+  c->st.ms_h2d = ev_ms(c, EV_START, EV_H2D);
+  c->st.ms_prep = ev_ms(c, EV_H2D, EV_WF0);
+  c->st.ms_wavefront = ev_ms(c, EV_WF0, EV_WF1);
+  c->st.ms_finalize = ev_ms(c, EV_WF1, EV_FIN);
   c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
   return PHMM_OK;
 }

@@ -66,9 +66,26 @@ class _Stats(ctypes.Structure):
                 ("ms_finalize", ctypes.c_float), ("ms_d2h", ctypes.c_float)]
 
 
+class _SwBatch(ctypes.Structure):
+    _fields_ = [("ref_bases", ctypes.c_void_p), ("ref_offsets", ctypes.c_void_p), ("n_refs", ctypes.c_int64),
+                ("alt_bases", ctypes.c_void_p), ("alt_offsets", ctypes.c_void_p), ("n_alts", ctypes.c_int64),
+                ("tasks", ctypes.c_void_p), ("n_tasks", ctypes.c_int64), ("total_ref_bases", ctypes.c_int64),
+                ("total_alt_bases", ctypes.c_int64)]
+
+
+class _SwParams(ctypes.Structure):
+    _fields_ = [("match", ctypes.c_int32), ("mismatch", ctypes.c_int32), ("gap_open", ctypes.c_int32),
+                ("gap_extend", ctypes.c_int32)]
+
+
+# HaplotypeCaller's haplotype-to-reference Smith-Waterman parameters (R20)
+SW_GATK_HC = (200, -150, -260, -11)
+SW_OPS = "MID"
+
 # every symbol include/phmm.h declares (checked by tests/test_abi.py)
 EXPORTED_SYMBOLS = ("phmm_create", "phmm_compute_batch", "phmm_compute_batch_dev", "phmm_destroy",
-                    "phmm_status_string", "phmm_get_stats", "phmm_abi_version")
+                    "phmm_status_string", "phmm_get_stats", "phmm_abi_version", "phmm_sw_align_batch",
+                    "phmm_sw_align_batch_dev")
 
 _lib = None
 
@@ -96,6 +113,10 @@ def load_library(path: str = LIB_PATH):
     L.phmm_get_stats.restype = ctypes.c_int
     L.phmm_abi_version.argtypes = []
     L.phmm_abi_version.restype = ctypes.c_int
+    for f in (L.phmm_sw_align_batch, L.phmm_sw_align_batch_dev):
+        f.argtypes = [ctypes.c_void_p, ctypes.POINTER(_SwBatch), ctypes.POINTER(_SwParams), ctypes.c_void_p,
+                      ctypes.c_void_p]
+        f.restype = ctypes.c_int
     _lib = L
     return L
 
@@ -247,6 +268,56 @@ class PairHMM:
         if rc != PHMM_OK:
             raise PhmmError(rc, "phmm_compute_batch_dev")
         return out, status
+
+    # ------------------------------------------------------------ Smith-Waterman
+    def sw_align_batch(self, b, params=SW_GATK_HC):
+        """``phmm_sw_align_batch`` on a synth.SwBatch-like object (host numpy arrays).
+        Returns (res int32 (n, 6): score, end_i, end_j, start_i, start_j, n_ops;
+        ops uint32 CIGAR runs, all tasks back to back; ops_off int64 (n+1): where task
+        t's runs start = prefix sums of n_ops)."""
+        keep = [np.ascontiguousarray(b.ref_bases, dtype=np.uint8), np.ascontiguousarray(b.ref_offsets, dtype=np.int64),
+                np.ascontiguousarray(b.alt_bases, dtype=np.uint8), np.ascontiguousarray(b.alt_offsets, dtype=np.int64),
+                np.ascontiguousarray(np.asarray(b.tasks, dtype=np.int32).reshape(-1, 2))]
+        rb, ro, ab, ao, t = keep
+        n = t.shape[0]
+        s = _SwBatch(rb.ctypes.data if rb.size else None, ro.ctypes.data, ro.size - 1,
+                     ab.ctypes.data if ab.size else None, ao.ctypes.data, ao.size - 1,
+                     t.ctypes.data if n else None, n, int(ro[-1]), int(ao[-1]))
+        # output capacity sum(M + N) (indices clipped here; the library reports bad ones)
+        ti, tj = np.clip(t[:, 0], 0, max(ro.size - 2, 0)), np.clip(t[:, 1], 0, max(ao.size - 2, 0))
+        cap = (ro[ti + 1] - ro[ti]) + (ao[tj + 1] - ao[tj]) if n else np.zeros(0, np.int64)
+        off = np.concatenate([[0], np.cumsum(cap)]).astype(np.int64)
+        res = np.zeros((n, 6), dtype=np.int32)
+        ops = np.zeros(max(int(off[-1]), 1), dtype=np.uint32)
+        p = _SwParams(*params)
+        rc = self._L.phmm_sw_align_batch(self._h, ctypes.byref(s), ctypes.byref(p), res.ctypes.data,
+                                         ops.ctypes.data)
+        del keep
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_sw_align_batch")
+        packed = np.concatenate([[0], np.cumsum(res[:, 5].astype(np.int64))]).astype(np.int64)
+        return res, ops[: max(int(packed[-1]), 0)], packed
+
+    def sw_align_batch_dev(self, tensors: dict, params=SW_GATK_HC, res=None, ops=None):
+        """``phmm_sw_align_batch_dev`` on torch CUDA tensors {ref_bases, ref_offsets,
+        alt_bases, alt_offsets, tasks}; ``ops`` (int32 tensor) must hold sum(M + N)
+        elements; the runs come back packed (task t's at the prefix sum of n_ops)."""
+        import torch
+
+        T = tensors
+        n = int(T["tasks"].shape[0])
+        s = _SwBatch(T["ref_bases"].data_ptr(), T["ref_offsets"].data_ptr(), T["ref_offsets"].numel() - 1,
+                     T["alt_bases"].data_ptr(), T["alt_offsets"].data_ptr(), T["alt_offsets"].numel() - 1,
+                     T["tasks"].data_ptr(), n, int(T["total_ref_bases"]), int(T["total_alt_bases"]))
+        dev = T["tasks"].device
+        if res is None:
+            res = torch.empty((n, 6), dtype=torch.int32, device=dev)
+        p = _SwParams(*params)
+        rc = self._L.phmm_sw_align_batch_dev(self._h, ctypes.byref(s), ctypes.byref(p), res.data_ptr(),
+                                             ops.data_ptr())
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_sw_align_batch_dev")
+        return res, ops
 
     def stats(self) -> dict:
         st = _Stats()

@@ -347,3 +347,108 @@ def concat_batches(batches: Sequence[Batch]) -> Batch:
                  read_offsets=np.concatenate(ro_parts), hap_bases=cat("hap_bases"),
                  hap_offsets=np.concatenate(ho_parts),
                  pairs=np.ascontiguousarray(np.concatenate(pairs), dtype=np.int32))
+
+
+# ---------------------------------------------------------------- Smith-Waterman tasks
+@dataclass
+class SwBatch:
+    """Smith-Waterman tasks in the C-ABI layout of include/phmm.h (phmm_sw_batch)."""
+
+    ref_bases: np.ndarray   # uint8 rows sequences, concatenated
+    ref_offsets: np.ndarray  # int64, n_refs + 1
+    alt_bases: np.ndarray   # uint8 column sequences
+    alt_offsets: np.ndarray  # int64, n_alts + 1
+    tasks: np.ndarray       # int32 (n_tasks, 2): (ref_idx, alt_idx)
+    meta: dict = field(default_factory=dict)
+
+    @property
+    def n_tasks(self) -> int:
+        return int(self.tasks.shape[0])
+
+    def ref(self, r: int) -> bytes:
+        return self.ref_bases[self.ref_offsets[r]:self.ref_offsets[r + 1]].tobytes()
+
+    def alt(self, a: int) -> bytes:
+        return self.alt_bases[self.alt_offsets[a]:self.alt_offsets[a + 1]].tobytes()
+
+    def cells(self) -> int:
+        t = self.tasks
+        m = self.ref_offsets[t[:, 0] + 1] - self.ref_offsets[t[:, 0]]
+        n = self.alt_offsets[t[:, 1] + 1] - self.alt_offsets[t[:, 1]]
+        return int(np.sum(m.astype(np.int64) * n))
+
+    def ops_capacity(self) -> np.ndarray:
+        """Per-task CIGAR capacity offsets (prefix sums of M + N), the ABI's layout."""
+        t = self.tasks
+        cap = (self.ref_offsets[t[:, 0] + 1] - self.ref_offsets[t[:, 0]]) + \
+              (self.alt_offsets[t[:, 1] + 1] - self.alt_offsets[t[:, 1]])
+        return np.concatenate([[0], np.cumsum(cap)]).astype(np.int64)
+
+
+# The paper's SW workload: per HaplotypeCaller region, each candidate haplotype is aligned
+# against the reference window (L16@3860: "the algorithm has been modified to adapt to the
+# needs of HaplotypeCaller"); batches average four tasks (L24@560) and were re-batched to
+# 3,200 tasks (L24@1700). SW1 = that re-batched size, SW2 = a large batch.
+SW_CONFIGS = {
+    "SW1": dict(n_regions=800, n_haps=4, window=(300, 500), seed=21,
+                desc="3,200 tasks: 4 haplotypes x 800 regions against 300-500 bp reference windows"),
+    "SW2": dict(n_regions=16384, n_haps=4, window=(300, 500), seed=22,
+                desc="65,536 tasks: 4 haplotypes x 16,384 regions, 300-500 bp windows"),
+}
+
+
+def sw_region(seed: int, region: int, n_haps: int, window) -> tuple:
+    """One region: the reference window and n_haps haplotypes (SNPs 1 %, 1-5 bp indels
+    0.5 %, so the alignments have gaps)."""
+    rng = _rng(seed, region)
+    w = _uniform_int(rng, window)
+    ref = _reference(rng, w)
+    haps = [_mutate(rng, ref, 0.01, 0.005) for _ in range(n_haps)]
+    return ref, haps
+
+
+def sw_config_batch(name: str, n_regions: Optional[int] = None, seed: Optional[int] = None) -> SwBatch:
+    cfg = SW_CONFIGS[name]
+    R = cfg["n_regions"] if n_regions is None else n_regions
+    s = cfg["seed"] if seed is None else seed
+    refs, alts, tasks = [], [], []
+    for reg in range(R):
+        ref, haps = sw_region(s, reg, cfg["n_haps"], cfg["window"])
+        refs.append(ref)
+        for h in haps:
+            tasks.append((len(refs) - 1, len(alts)))
+            alts.append(h)
+    return _sw_pack(refs, alts, tasks, dict(config=name, seed=s, n_regions=R))
+
+
+def sw_random_batch(seed: int, n_tasks: int, m_range=(1, 60), n_range=(1, 60), alphabet=b"ACGTN",
+                    related: float = 0.5) -> SwBatch:
+    """Ragged random tasks for parity edge cases; a fraction `related` of the columns
+    sequences are mutated copies of their row sequence (long alignments with gaps)."""
+    rng = _rng(seed, 0)
+    alph = np.frombuffer(alphabet, dtype=np.uint8)
+    refs, alts, tasks = [], [], []
+    for t in range(n_tasks):
+        m = int(rng.integers(m_range[0], m_range[1] + 1))
+        n = int(rng.integers(n_range[0], n_range[1] + 1))
+        a = alph[rng.integers(0, alph.size, size=m)]
+        if rng.random() < related:
+            b = _mutate(rng, np.where(a == ord("N"), ord("A"), a).astype(np.uint8), 0.05, 0.03)[:n]
+            if b.size < n:
+                b = np.concatenate([b, alph[rng.integers(0, alph.size, size=n - b.size)]])
+        else:
+            b = alph[rng.integers(0, alph.size, size=n)]
+        refs.append(a.astype(np.uint8))
+        alts.append(b.astype(np.uint8))
+        tasks.append((t, t))
+    return _sw_pack(refs, alts, tasks, dict(seed=seed))
+
+
+def _sw_pack(refs, alts, tasks, meta) -> SwBatch:
+    ro = np.zeros(len(refs) + 1, dtype=np.int64)
+    np.cumsum([r.size for r in refs], out=ro[1:])
+    ao = np.zeros(len(alts) + 1, dtype=np.int64)
+    np.cumsum([a.size for a in alts], out=ao[1:])
+    cat = lambda xs: np.ascontiguousarray(np.concatenate(xs) if xs else np.zeros(0, np.uint8), dtype=np.uint8)
+    return SwBatch(ref_bases=cat(refs), ref_offsets=ro, alt_bases=cat(alts), alt_offsets=ao,
+                   tasks=np.ascontiguousarray(np.asarray(tasks, dtype=np.int32).reshape(-1, 2)), meta=meta)

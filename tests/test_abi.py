@@ -39,7 +39,10 @@ def test_library_exports_every_declared_symbol(lib):
 
 
 def test_abi_version_and_status_strings(lib):
-    assert lib.phmm_abi_version() == 1
+    import re
+
+    hdr = open(os.path.join(ROOT, "include", "phmm.h")).read()
+    assert lib.phmm_abi_version() == int(re.search(r"#define PHMM_ABI_VERSION (\d+)", hdr).group(1))
     for code in (0, -1, -2, -3, -4, -5, -6, -7):
         s = lib.phmm_status_string(code).decode()
         assert s and s != "unknown status"
@@ -85,3 +88,9 @@ def test_product_path_does_not_import_the_oracle():
                 txt = open(os.path.join(dirpath, f), errors="ignore").read()
                 assert "import oracle" not in txt and "from oracle" not in txt, f
                 assert "phmm_oracle" not in txt and "liboracle" not in txt, f
+
+
+def test_sw_entry_points_reject_null_without_gpu(lib):
+    """The Smith-Waterman calls validate their arguments before touching the device."""
+    assert lib.phmm_sw_align_batch(None, None, None, None, None) == -1
+    assert lib.phmm_sw_align_batch_dev(None, None, None, None, None) == -1
