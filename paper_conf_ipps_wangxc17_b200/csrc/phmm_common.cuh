@@ -9,22 +9,23 @@
 //
 // How (DESIGN.md §4 -- differs from the paper's one-warp-per-pair PH2):
 //  * "tall stream" layout: every pair is laid out as a whole number of K-row
-//    BLOCKS: [Z..Z][R][read rows 1..m][S1][S2] where the pad rows are plain
-//    rows of the same recurrence with special coefficients:
-//      Z  (zero)   : every coefficient 0            -> M = I = D = 0
-//      R  (reset)  : prior 0, delta=eps=zeta=0, mu=1, boundary D(.,0)=s/N
-//                    -> M = I = 0, D = s/N on every column: the virtual row 0
+//    BLOCKS: [Z..Z][R][read rows 1..m][S] (at least one Z row) where the pad rows
+//    are plain rows of the same recurrence (the kernel's rescaled 5-op form,
+//    wavefront.cuh) with special coefficients:
+//      Z  (zero)   : T = u = w = ep' = mu = 0      -> M = D = 0 (I = M of the row
+//                    above: finite garbage that the next Z/R row, with ep' = 0, drops)
+//      R  (reset)  : T = 0, ep' = 0, mu = 1, boundary D(.,0) = s/ncols
+//                    -> M = I = 0, D = s/ncols on every column: the virtual row 0
 //                       of Eq. 6 (D(0,j) = 1/N, scaled by s)
-//      S1 (sum)    : prior 0, delta=eps=1, zeta=0   -> I(j) = M(m,j) + I(m,j)
-//      S2 (scan)   : prior 1, alpha=0, beta=1, zeta=mu=1
-//                    -> M(j) = I_S1(j-1), D(j) = sum_{j'<j} M(j'),
-//                       so D_S2(N+2) = sum_{j=1..N} M(m,j) + I(m,j)
+//      S  (sum)    : T = 1/a_m, u = a_m/b_m, w = 0, mu = 1
+//                    -> M(j) = M(m,j-1) + I(m,j-1) (unscaled), D(j) = sum_{j'<j} M(j'),
+//                       so D_S(N+2) = sum_{j=1..N} M(m,j) + I(m,j)
 //    The termination sum of L20@2262 therefore falls out of the recurrence
-//    itself, read as D of the S2 row at column N+2 (0-based c = N+1), and
-//    consecutive pairs can be stacked into one tall DP: a Z/R row ignores
-//    whatever (finite) values are above it. One warp streams through a long
-//    sequence of blocks of equal column count (a length bin) without
-//    draining between pairs.
+//    itself, read as D of the S row at column N+2 (0-based c = N+1), and
+//    consecutive pairs can be stacked into one tall DP: a Z row followed by a
+//    Z/R row ignores whatever (finite) values are above it. One warp streams
+//    through a long sequence of blocks of equal column count (a length bin)
+//    without draining between pairs.
 //  * lane l of a warp owns one K-row block per "pass" (blocks l, l+32, ...),
 //    processes one column per step (a K-row column tile), lags lane l-1 by
 //    one step, receives the (M,I,D) of the row above by __shfl_sync
@@ -78,6 +79,7 @@ __host__ __device__ inline int ncols_of(int n, int bucket) {
   return c < lo ? lo : c;
 }
 __host__ __device__ inline int bin_of_ncols(int ncols, int bucket) { return ncols / bucket; }
+// rows: f >= 1 Z rows, R, m read rows, S  ->  nb*K >= m + 3
 template <int K>
 __host__ __device__ inline int nblocks_of(int m) { return (m + 3 + K - 1) / K; }
 

@@ -77,9 +77,37 @@ __global__ void k_hap_ncols(const int64_t* __restrict__ hoff, int64_t n_haps, in
 
 // ---------------------------------------------------------------- coefficient tables
 // Per table item (a read, or a rescued pair's read): nb = ceil((m+3)/K) blocks of K rows
-//   [f Z rows][R][read rows 1..m][S1][S2]          (phmm_common.cuh)
-// One warp per item, lanes over its padded rows; Phred -> error probability from a
-// 128-entry table built once per CUDA block (10^(-q/10) in double, rounded to T).
+//   [f >= 1 Z rows][R][read rows 1..m][S]          (phmm_common.cuh)
+// One warp per item, lanes over its padded rows. The coefficients of the kernel's
+// 5-op form of Eq. 6 (wavefront.cuh) are computed in double from a
+// 128-entry Phred table (10^(-q/10)) and rounded once to T. Row i stores
+//   M^ = a_i M, I^ = b_i I, D^ = d_i D,   a_i = k_i zeta_i, d_i = k_i, b_i = a_{i-1}/delta_i,
+//   k_i = min(1, delta_{i+1}/zeta_i) (k_m = 1),   R row: a = delta_1, b = d = 1,
+// so that no stored value exceeds its unscaled one (b_i <= 1, k_i <= 1) and
+//   D^ = M^(left) + mu D^(left),  I^ = M^(up) + ep' I^(up),
+//   M^ = T[code] * (M^(diag) + u I^(diag) + w D^(diag)).
+struct RowScale {
+  double a, b, d;  // storage scales of M, I, D
+};
+// storage scales of read row i (1..m; 0 = the R row); e(q) from the table
+__device__ __forceinline__ RowScale row_scale(int i, int m, const uint8_t* __restrict__ qi,
+                                              const uint8_t* __restrict__ qd, int64_t x1, const double* err) {
+  // x1 = offset of read row 1's qualities
+  auto de = [&](int r) { return err[qi[x1 + r - 1] & 127]; };
+  auto ze = [&](int r) { return err[qd[x1 + r - 1] & 127]; };
+  auto kf = [&](int r) { return r < m ? fmin(1.0, de(r + 1) / ze(r)) : 1.0; };
+  RowScale S;
+  if (i == 0) {
+    S.a = de(1); S.b = 1.0; S.d = 1.0;
+  } else {
+    const double k = kf(i);
+    S.a = k * ze(i);
+    S.d = k;
+    S.b = (i == 1) ? 1.0 : kf(i - 1) * ze(i - 1) / de(i);
+  }
+  return S;
+}
+
 constexpr int kTabThreads = 256;
 template <typename T>
 __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
@@ -88,8 +116,8 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
     const uint8_t* __restrict__ qi, const uint8_t* __restrict__ qd, const uint8_t* __restrict__ qg,
     TBlock<T>* __restrict__ tab) {
   constexpr int K = WfT<T>::K;
-  __shared__ T err[128];
-  for (int i = threadIdx.x; i < 128; i += blockDim.x) err[i] = qual_err<T>((uint32_t)i);
+  __shared__ double err[128];
+  for (int i = threadIdx.x; i < 128; i += blockDim.x) err[i] = qual_err<double>((uint32_t)i);
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -99,45 +127,45 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
     const int m = (int)(roff[r + 1] - r0);
     if (m < 1) continue;
     const int nb = nblocks_of<K>(m);
-    const int f = nb * K - (m + 3);
+    const int f = nb * K - (m + 2);  // >= 1 Z rows
     TBlock<T>* __restrict__ Tb = tab + item_tab_off[it];
     for (int row = lane; row < nb * K; row += 32) {
-      // gamma = beta/alpha, delta, eps, zeta, mu, and alpha*P per haplotype code
-      T ga = 0, de = 0, ep = 0, ze = 0, mu = 0;
-      T p5[5] = {0, 0, 0, 0, 0};
+      double uu = 0, ww = 0, ep = 0, mu = 0;
+      double p5[5] = {0, 0, 0, 0, 0};
       if (row < f) {
-        // Z row: all zero
+        // Z row: all zero (absorbs whatever finite values are above it)
       } else if (row == f) {  // R row: D = d0 on every column
         mu = 1;
       } else if (row <= f + m) {
-        const int64_t x = r0 + (row - f - 1);
-        const T ei = err[qi[x] & 127], ed = err[qd[x] & 127], eg = err[qg[x] & 127], eb = err[q[x] & 127];
-        const T sum = ei + ed;
-        const T al = (T)1 - (sum < (T)1 ? sum : (T)1);  // > 0.0065 after validation (R16)
-        ga = ((T)1 - eg) / al;
-        de = ei;
-        ep = eg;
-        ze = ed;
+        const int i = row - f;
+        const int64_t x = r0 + (i - 1);
+        const RowScale Sp = row_scale(i - 1, m, qi, qd, r0, err), Si = row_scale(i, m, qi, qd, r0, err);
+        const double ei = err[qi[x] & 127], ed = err[qd[x] & 127], eg = err[qg[x] & 127], eb = err[q[x] & 127];
+        const double al = 1.0 - fmin(ei + ed, 1.0);  // > 0.0065 after validation (R16)
+        const double be = 1.0 - eg;
+        uu = be * Sp.a / (al * Sp.b);
+        ww = be * Sp.a / (al * Sp.d);
+        ep = eg * Si.b / Sp.b;
         mu = eg;
-        const T pm = al * ((T)1 - eb), px = al * (eb / (T)3);
+        const double t = Si.a * al / Sp.a;
+        const double pm = t * (1.0 - eb), px = t * (eb / 3.0);
         const uint8_t base = rb[x];
         p5[0] = (base == 'A' || base == 'N') ? pm : px;
         p5[1] = (base == 'C' || base == 'N') ? pm : px;
         p5[2] = (base == 'G' || base == 'N') ? pm : px;
         p5[3] = (base == 'T' || base == 'N') ? pm : px;
         p5[4] = pm;  // haplotype 'N' matches everything
-      } else if (row == f + m + 1) {  // S1: I = M(m,j) + I(m,j)
-        de = 1; ep = 1; mu = 1;
-      } else {  // S2: M = I_S1(j-1) (M_S1 = D_S1 = 0), D = running sum
-        ga = 1; ze = 1; mu = 1;
-        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = 1;
+      } else {  // S: M^ = (M + I)(m, j-1), D^ = running sum (the L20@2262 termination)
+        const RowScale Sm = row_scale(m, m, qi, qd, r0, err);
+        uu = Sm.a / Sm.b;
+        mu = 1;
+        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = 1.0 / Sm.a;
       }
       TBlock<T>& B = Tb[row / K];
       const int t = row % K;
-      B.coef[0][t] = ga; B.coef[1][t] = de; B.coef[2][t] = ep;
-      B.coef[3][t] = ze; B.coef[4][t] = mu;
+      B.coef[0][t] = (T)uu; B.coef[1][t] = (T)ww; B.coef[2][t] = (T)ep; B.coef[3][t] = (T)mu;
 #pragma unroll
-      for (int k = 0; k < 5; ++k) B.prior[k][t] = p5[k];
+      for (int k = 0; k < 5; ++k) B.prior[k][t] = (T)p5[k];
     }
   }
 }
@@ -200,7 +228,7 @@ __global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32
       const int64_t slot_s = __shfl_sync(0xffffffffu, slot, src);
       const uint32_t tab_s = __shfl_sync(0xffffffffu, tab0, src);
       const uint32_t hap_s = __shfl_sync(0xffffffffu, hap, src);
-      const int f = nb_s * K - (m_s + 3);  // R row index within the pair's rows
+      const int f = nb_s * K - (m_s + 2);  // R row index within the pair's rows (f >= 1 Z rows before it)
       for (int j = lane; j < nb_s; j += 32) {
         BlkDesc d;
         d.tab_blk = tab_s + j;

@@ -129,18 +129,21 @@ template <typename V> __device__ __forceinline__ V vzero();
 template <> __device__ __forceinline__ v2f vzero<v2f>() { return 0ull; }
 template <> __device__ __forceinline__ v2d vzero<v2d>() { return v2d{0.0, 0.0}; }
 
-// per-block coefficient table: 5 transition fields + 5 prior codes, K rows each.
-// Eq. 6's match update P*(alpha*M + beta*(I + D)) is evaluated as
-// (alpha*P) * (M + gamma*(I + D)) with gamma = beta/alpha (alpha >= 0.0065 for every
-// validated read row, R16): the table holds alpha*P per code, so alpha and
-// beta leave the registers and one multiply per cell disappears.
-constexpr int WF_NCOEF = 5;
+// per-block coefficient table: 4 transition fields + 5 prior codes, K rows each.
+// The kernel evaluates Eq. 6 in a rescaled 5-op form: row i stores
+// M^ = a_i M, I^ = b_i I, D^ = d_i D with per-row scales chosen so that the coefficient
+// of M in the D update and of M(up) in the I update are exactly 1:
+//   D^ = M^(i,j-1) + mu D^(i,j-1)                                    1 FFMA
+//   I^ = M^(i-1,j) + ep' I^(i-1,j)                                   1 FFMA
+//   M^ = T[code] * (M^(i-1,j-1) + u I^(i-1,j-1) + w D^(i-1,j-1))     2 FFMA + 1 FMUL
+// (stream_prep.cuh k_build_table_wf has the scales; none exceeds the unscaled value).
+constexpr int WF_NCOEF = 4;
 template <typename T>
 struct alignas(16) TBlock {
-  T coef[WF_NCOEF][WfT<T>::K];  // gamma, delta, eps, zeta, mu
-  T prior[5][WfT<T>::K];        // alpha * P(row, code) for code = A, C, G, T, N
+  T coef[WF_NCOEF][WfT<T>::K];  // u, w, ep', mu
+  T prior[5][WfT<T>::K];        // T(row, code) for code = A, C, G, T, N
 };
-static_assert(sizeof(TBlock<float>) == 10 * WF_KC * 16 && sizeof(TBlock<double>) == 10 * WF_KC * 16, "TBlock");
+static_assert(sizeof(TBlock<float>) == 9 * WF_KC * 16 && sizeof(TBlock<double>) == 9 * WF_KC * 16, "TBlock");
 
 template <typename T>
 struct WfArgs2 {
@@ -162,7 +165,7 @@ template <typename T>
 struct Lane {
   using V = typename WfT<T>::V;
   static constexpr int K = WfT<T>::K;
-  V ga[K], de[K], ep[K], ze[K], mu[K];
+  V uu[K], ww[K], ep[K], mu[K];
   V M[K], I[K], D[K];
 };
 
@@ -180,18 +183,17 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
     const V md = (u == 0) ? dgM : L.M[u - 1];
     const V id = (u == 0) ? dgI : L.I[u - 1];
     const V dd = (u == 0) ? dgD : L.D[u - 1];
-    // D(i,j) = zeta*M(i,j-1) + mu*D(i,j-1)
-    L.D[u] = fma2(L.ze[u], L.M[u], mul2(L.mu[u], L.D[u]));
-    // M(i,j) = P(i,j) * (alpha*M(i-1,j-1) + beta*(I(i-1,j-1) + D(i-1,j-1)))
-    //        = (alpha*P) * (M(i-1,j-1) + gamma*(I(i-1,j-1) + D(i-1,j-1)))
-    const V x = fma2(L.ga[u], add2(id, dd), md);
+    // D^(i,j) = M^(i,j-1) + mu*D^(i,j-1)
+    L.D[u] = fma2(L.mu[u], L.D[u], L.M[u]);
+    // M^(i,j) = T(i, h_j) * (M^(i-1,j-1) + u*I^(i-1,j-1) + w*D^(i-1,j-1))
+    const V x = fma2(L.ww[u], dd, fma2(L.uu[u], id, md));
     L.M[u] = pk(prA[u] * lo(x), prB[u] * hi(x));
   }
-  // I(i,j) = delta*M(i-1,j) + eps*I(i-1,j), rows ascending (a K-deep chain)
+  // I^(i,j) = M^(i-1,j) + ep'*I^(i-1,j), rows ascending (a K-deep chain)
   V m_up = upM, i_up = upI;
 #pragma unroll
   for (int u = 0; u < K; ++u) {
-    const V ni = fma2(L.ep[u], i_up, mul2(L.de[u], m_up));
+    const V ni = fma2(L.ep[u], i_up, m_up);
     m_up = L.M[u];
     i_up = ni;
     L.I[u] = ni;
@@ -263,9 +265,8 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
     const int rrow = (d.flags >> WF_RROW_SHIFT) & 15;
 #pragma unroll
     for (int u = 0; u < K; ++u) {
-      L.ga[u] = set_half<H>(L.ga[u], cw.v[0][u]); L.de[u] = set_half<H>(L.de[u], cw.v[1][u]);
-      L.ep[u] = set_half<H>(L.ep[u], cw.v[2][u]); L.ze[u] = set_half<H>(L.ze[u], cw.v[3][u]);
-      L.mu[u] = set_half<H>(L.mu[u], cw.v[4][u]);
+      L.uu[u] = set_half<H>(L.uu[u], cw.v[0][u]); L.ww[u] = set_half<H>(L.ww[u], cw.v[1][u]);
+      L.ep[u] = set_half<H>(L.ep[u], cw.v[2][u]); L.mu[u] = set_half<H>(L.mu[u], cw.v[3][u]);
       L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
       L.D[u] = set_half<H>(L.D[u], rrow == u ? d0 : (T)0);
     }
@@ -279,9 +280,8 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   }
 #pragma unroll
   for (int u = 0; u < K; ++u) {
-    L.ga[u] = set_half<H>(L.ga[u], (T)0);
-    L.de[u] = set_half<H>(L.de[u], (T)0); L.ep[u] = set_half<H>(L.ep[u], (T)0);
-    L.ze[u] = set_half<H>(L.ze[u], (T)0); L.mu[u] = set_half<H>(L.mu[u], (T)0);
+    L.uu[u] = set_half<H>(L.uu[u], (T)0); L.ww[u] = set_half<H>(L.ww[u], (T)0);
+    L.ep[u] = set_half<H>(L.ep[u], (T)0); L.mu[u] = set_half<H>(L.mu[u], (T)0);
     L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
     L.D[u] = set_half<H>(L.D[u], (T)0);
   }
@@ -309,7 +309,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   Lane<T> L;
 #pragma unroll
   for (int u = 0; u < K; ++u) {
-    L.ga[u] = L.de[u] = L.ep[u] = L.ze[u] = L.mu[u] = vzero<V>();
+    L.uu[u] = L.ww[u] = L.ep[u] = L.mu[u] = vzero<V>();
     L.M[u] = L.I[u] = L.D[u] = vzero<V>();
   }
   const uint32_t* pA = reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);  // next code word
@@ -404,7 +404,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
         const int bA = q * 64 + 2 * lane, bB = bA + 1;
         const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
         const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
-        if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S2 row: the last-row M+I sum (L20@2262)
+        if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S row: the last-row M+I sum (L20@2262)
         if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
         pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
         pB = wf_load<1, T>(A, L, tabB_s, hB, dB, d0, outB, giB, copy_len);

@@ -3,7 +3,7 @@ virtual lanes of a warp). It models what the kernel computes, independent of how
 virtual lanes are packed into physical lanes / register halves:
 
 * a warp streams through the blocks of one length bin; pass q gives block 64q+v to
-  virtual lane v (K rows each, the Z/R/read/S1/S2 pad-row layout of DESIGN.md §4.2);
+  virtual lane v (K rows each, the Z/R/read/S pad-row layout of DESIGN.md §4.2);
 * virtual lane v computes column x of its block at step T_q + 1 + v + x; a pass is
   P = max(ncols + G, 72) steps; virtual lanes switch blocks in groups of G = 8 at the
   events T_q + 8e (e = 0..7), taking column -1 - (v mod 8) next;
@@ -11,7 +11,7 @@ virtual lanes are packed into physical lanes / register halves:
 * virtual lane v takes the row above from v-1's last row one step later; v = 0 from
   a ring indexed by column + 1 (slot 0 = boundary column) written by v = 63 of the
   previous pass;
-* the result of a pair is D of its S2 row, read at the next switch event.
+* the result of a pair is D of its S row, read at the next switch event.
 
 The GPU kernel's per-step state was compared against this model with a trace build
 (DESIGN.md §4.4); tests/test_schedule_emulation.py checks the model against the oracle.
@@ -33,33 +33,55 @@ def qerr(q):
 
 
 def read_rows(rb, q, qi, qd, qg, K):
-    """(nb*K rows of (al, be, de, ep, ze, mu, prior[5])), nb, f = number of Z rows."""
+    """(nb*K rows of (u, w, ep', mu, prior[5])), nb, f = number of Z rows (>= 1).
+
+    The kernel's 5-op form of Eq. 6: per row i the stored values are
+    M^ = a_i M, I^ = b_i I, D^ = d_i D with a_i = k_i zeta_i, d_i = k_i, b_i = a_{i-1}/delta_i,
+    k_i = min(1, delta_{i+1}/zeta_i) (k_m = 1), a_R = delta_1, b_R = d_R = 1, so that
+      D^ = M^(left) + mu D^(left)
+      I^ = M^(up) + ep' I^(up)                  ep' = eps_i b_i / b_{i-1}
+      M^ = T[code] (M^(diag) + u I^(diag) + w D^(diag))
+           T = a_i alpha_i P / a_{i-1},  u = beta_i a_{i-1} / (alpha_i b_{i-1}),
+           w = beta_i a_{i-1} / (alpha_i d_{i-1})
+    and the S row: T = 1/a_m, u = a_m/b_m, w = 0, ep' = 0, mu = 1 -> M^_S(j) = (M+I)(m,j-1),
+    D^_S = running sum."""
     m = len(rb)
     nb = (m + 3 + K - 1) // K
-    f = nb * K - (m + 3)
+    f = nb * K - (m + 2)
+    e = lambda qq: 10.0 ** (-float(qq) / 10.0)
+    de = [None] + [e(qi[x]) for x in range(m)]
+    ze = [None] + [e(qd[x]) for x in range(m)]
+    kk = [1.0] + [min(1.0, de[i + 1] / ze[i]) if i < m else 1.0 for i in range(1, m + 1)]
+    a = [de[1]] + [kk[i] * ze[i] for i in range(1, m + 1)]
+    b = [1.0, 1.0] + [a[i - 1] / de[i] for i in range(2, m + 1)]
+    d = [1.0] + [kk[i] for i in range(1, m + 1)]
     rows = []
     for row in range(nb * K):
-        al = be = de = ep = ze = mu = E(0)
-        pr = [E(0)] * 5
+        uu = ww = ep = mu = 0.0
+        pr = [0.0] * 5
         if row < f:
             pass  # Z
         elif row == f:
-            mu = E(1)  # R
+            mu = 1.0  # R
         elif row <= f + m:
-            x = row - f - 1
-            ei, ed, eg, eb = qerr(qi[x]), qerr(qd[x]), qerr(qg[x]), qerr(q[x])
-            s = E(ei + ed)
-            al = E(E(1) - min(s, E(1)))
-            be = E(E(1) - eg); de = ei; ep = eg; ze = ed; mu = eg
-            pm, px = E(E(1) - eb), E(eb / E(3))
+            i = row - f
+            x = i - 1
+            ei, ed, eg, eb = de[i], ze[i], e(qg[x]), e(q[x])
+            al = 1.0 - min(ei + ed, 1.0)
+            be = 1.0 - eg
+            uu = be * a[i - 1] / (al * b[i - 1])
+            ww = be * a[i - 1] / (al * d[i - 1])
+            ep = eg * b[i] / b[i - 1]
+            mu = eg
+            pm, px = 1.0 - eb, eb / 3.0
             base = chr(rb[x])
-            pr = [pm if (base == c or base == 'N') else px for c in "ACGT"] + [pm]
-        elif row == f + m + 1:
-            de = ep = mu = E(1)  # S1
-        else:
-            be = ze = mu = E(1)  # S2
-            pr = [E(1)] * 5
-        rows.append((al, be, de, ep, ze, mu, pr))
+            t = a[i] * al / a[i - 1]
+            pr = [t * (pm if (base == c or base == 'N') else px) for c in "ACGT"] + [t * pm]
+        else:  # S
+            uu = a[m] / b[m]
+            mu = 1.0
+            pr = [1.0 / a[m]] * 5
+        rows.append((E(uu), E(ww), E(ep), E(mu), [E(v) for v in pr]))
     return rows, nb, f
 
 
@@ -83,7 +105,7 @@ def run_stream(blocks, ncols, K):
     npass = (nblk + 63) // 64
     d0 = E(2.0 ** 120) / E(ncols)
     V = 64
-    co = np.zeros((6, V, K), E)
+    co = np.zeros((4, V, K), E)
     pri = np.zeros((V, 6, K), E)
     M = np.zeros((V, K), E); I = np.zeros_like(M); D = np.zeros_like(M)
     up = np.zeros((V, 3), E); dg = np.zeros((V, 3), E)
@@ -105,19 +127,19 @@ def run_stream(blocks, ncols, K):
 
     def step():
         pr = np.stack([pri[v, code_of(v)] for v in range(V)])
-        al, be, de, ep, ze, mu = co
-        lastM, lastI, lastD = M[:, K - 1].copy(), I[:, K - 1].copy(), D[:, K - 1].copy()
+        uu, ww, ep, mu = co
         for u in range(K - 1, -1, -1):
             md = dg[:, 0] if u == 0 else M[:, u - 1]
             id_ = dg[:, 1] if u == 0 else I[:, u - 1]
             dd = dg[:, 2] if u == 0 else D[:, u - 1]
-            nD = (ze[:, u] * M[:, u] + mu[:, u] * D[:, u]).astype(E)
-            x = (al[:, u] * md + be[:, u] * (id_ + dd).astype(E)).astype(E)
+            nD = (mu[:, u] * D[:, u] + M[:, u]).astype(E)
+            y = (uu[:, u] * id_ + md).astype(E)
+            x = (ww[:, u] * dd + y).astype(E)
             M[:, u] = (pr[:, u] * x).astype(E)
             D[:, u] = nD
         m_up, i_up = up[:, 0].copy(), up[:, 1].copy()
         for u in range(K):
-            ni = (ep[:, u] * i_up + de[:, u] * m_up).astype(E)
+            ni = (ep[:, u] * i_up + m_up).astype(E)
             m_up = M[:, u].copy(); i_up = ni; I[:, u] = ni
         # exchange: v <- v-1 (this step's last row); v = 0 <- ring slot of its next column
         c63 = col[63]
@@ -144,10 +166,10 @@ def run_stream(blocks, ncols, K):
                     blk = blocks[b]
                     for u in range(K):
                         r = blk["rows"][u]
-                        for fi in range(6):
+                        for fi in range(4):
                             co[fi, v, u] = r[fi]
                         for cc in range(5):
-                            pri[v, cc, u] = r[6][cc]
+                            pri[v, cc, u] = r[4][cc]
                         M[v, u] = 0; I[v, u] = 0
                         D[v, u] = d0 if blk["rrow"] == u else E(0)
                     codes[v], offs[v] = blk["codes"]
