@@ -79,35 +79,14 @@ __global__ void k_hap_ncols(const int64_t* __restrict__ hoff, int64_t n_haps, in
 // Per table item (a read, or a rescued pair's read): nb = ceil((m+3)/K) blocks of K rows
 //   [f >= 1 Z rows][R][read rows 1..m][S]          (phmm_common.cuh)
 // One warp per item, lanes over its padded rows. The coefficients of the kernel's
-// 5-op form of Eq. 6 (wavefront.cuh) are computed in double from a
-// 128-entry Phred table (10^(-q/10)) and rounded once to T. Row i stores
+// 5-op form of Eq. 6 (wavefront.cuh) are computed from a 128-entry
+// Phred table (10^(-q/10), rounded once to T); each lane computes its row's storage
+// scales and takes the row above's by __shfl_up_sync. Row i stores
 //   M^ = a_i M, I^ = b_i I, D^ = d_i D,   a_i = k_i zeta_i, d_i = k_i, b_i = a_{i-1}/delta_i,
 //   k_i = min(1, delta_{i+1}/zeta_i) (k_m = 1),   R row: a = delta_1, b = d = 1,
 // so that no stored value exceeds its unscaled one (b_i <= 1, k_i <= 1) and
 //   D^ = M^(left) + mu D^(left),  I^ = M^(up) + ep' I^(up),
 //   M^ = T[code] * (M^(diag) + u I^(diag) + w D^(diag)).
-struct RowScale {
-  double a, b, d;  // storage scales of M, I, D
-};
-// storage scales of read row i (1..m; 0 = the R row); e(q) from the table
-__device__ __forceinline__ RowScale row_scale(int i, int m, const uint8_t* __restrict__ qi,
-                                              const uint8_t* __restrict__ qd, int64_t x1, const double* err) {
-  // x1 = offset of read row 1's qualities
-  auto de = [&](int r) { return err[qi[x1 + r - 1] & 127]; };
-  auto ze = [&](int r) { return err[qd[x1 + r - 1] & 127]; };
-  auto kf = [&](int r) { return r < m ? fmin(1.0, de(r + 1) / ze(r)) : 1.0; };
-  RowScale S;
-  if (i == 0) {
-    S.a = de(1); S.b = 1.0; S.d = 1.0;
-  } else {
-    const double k = kf(i);
-    S.a = k * ze(i);
-    S.d = k;
-    S.b = (i == 1) ? 1.0 : kf(i - 1) * ze(i - 1) / de(i);
-  }
-  return S;
-}
-
 constexpr int kTabThreads = 256;
 template <typename T>
 __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
@@ -115,9 +94,11 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
     const int64_t* __restrict__ roff, const uint8_t* __restrict__ rb, const uint8_t* __restrict__ q,
     const uint8_t* __restrict__ qi, const uint8_t* __restrict__ qd, const uint8_t* __restrict__ qg,
     TBlock<T>* __restrict__ tab) {
+  // computed in the table's precision T: a few roundings per coefficient (FP32: well
+  // inside the 1e-3 log10 tolerance; FP64: ~1e-16 per row)
   constexpr int K = WfT<T>::K;
-  __shared__ double err[128];
-  for (int i = threadIdx.x; i < 128; i += blockDim.x) err[i] = qual_err<double>((uint32_t)i);
+  __shared__ T err[128];
+  for (int i = threadIdx.x; i < 128; i += blockDim.x) err[i] = qual_err<T>((uint32_t)i);
   __syncthreads();
   const int lane = threadIdx.x & 31;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -129,43 +110,70 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
     const int nb = nblocks_of<K>(m);
     const int f = nb * K - (m + 2);  // >= 1 Z rows
     TBlock<T>* __restrict__ Tb = tab + item_tab_off[it];
-    for (int row = lane; row < nb * K; row += 32) {
-      double uu = 0, ww = 0, ep = 0, mu = 0;
-      double p5[5] = {0, 0, 0, 0, 0};
-      if (row < f) {
+    const T de1 = err[qi[r0] & 127];
+    // storage scales (a, b, d) of the row above the lane's row, carried across iterations
+    T ca = 1, cb = 1, cd = 1;
+    for (int base = 0; base < nb * K; base += 32) {  // warp-uniform trip count
+      const int row = base + lane;
+      const int i = row - f;  // < 0 Z, 0 R, 1..m read rows, m+1 S
+      const bool real = (i >= 1) && (i <= m);
+      const int64_t x = r0 + (real ? i - 1 : 0);
+      T ei = 0, ed = 0, eg = 0, eb = 0;
+      uint8_t base_c = 'N';
+      if (real) {
+        ei = err[qi[x] & 127]; ed = err[qd[x] & 127]; eg = err[qg[x] & 127]; eb = err[q[x] & 127];
+        base_c = rb[x];
+      }
+      // own a = k zeta, d = k with k = min(1, delta_{i+1}/zeta_i) (k_m = 1); R row: a = delta_1
+      T a = 1, d = 1;
+      if (i == 0) {
+        a = de1;
+      } else if (real) {
+        const T k = (i < m) ? fmin((T)1, err[qi[x + 1] & 127] / ed) : (T)1;
+        a = k * ed;
+        d = k;
+      }
+      T ap = __shfl_up_sync(0xffffffffu, a, 1);
+      if (lane == 0) ap = ca;
+      // b = a_{i-1} / delta_i (b_1 = 1)
+      const T b = (real && i >= 2) ? ap / ei : (T)1;
+      T bp = __shfl_up_sync(0xffffffffu, b, 1), dp = __shfl_up_sync(0xffffffffu, d, 1);
+      if (lane == 0) { bp = cb; dp = cd; }
+      ca = __shfl_sync(0xffffffffu, a, 31);
+      cb = __shfl_sync(0xffffffffu, b, 31);
+      cd = __shfl_sync(0xffffffffu, d, 31);
+      if (row >= nb * K) continue;
+      T uu = 0, ww = 0, ep = 0, mu = 0;
+      T p5[5] = {0, 0, 0, 0, 0};
+      if (i < 0) {
         // Z row: all zero (absorbs whatever finite values are above it)
-      } else if (row == f) {  // R row: D = d0 on every column
+      } else if (i == 0) {  // R row: D = d0 on every column
         mu = 1;
-      } else if (row <= f + m) {
-        const int i = row - f;
-        const int64_t x = r0 + (i - 1);
-        const RowScale Sp = row_scale(i - 1, m, qi, qd, r0, err), Si = row_scale(i, m, qi, qd, r0, err);
-        const double ei = err[qi[x] & 127], ed = err[qd[x] & 127], eg = err[qg[x] & 127], eb = err[q[x] & 127];
-        const double al = 1.0 - fmin(ei + ed, 1.0);  // > 0.0065 after validation (R16)
-        const double be = 1.0 - eg;
-        uu = be * Sp.a / (al * Sp.b);
-        ww = be * Sp.a / (al * Sp.d);
-        ep = eg * Si.b / Sp.b;
+      } else if (real) {
+        const T al = (T)1 - fmin(ei + ed, (T)1);  // > 0.0065 after validation (R16)
+        const T be = (T)1 - eg;
+        const T g = be * ap / al;
+        uu = g / bp;
+        ww = g / dp;
+        ep = eg * b / bp;
         mu = eg;
-        const double t = Si.a * al / Sp.a;
-        const double pm = t * (1.0 - eb), px = t * (eb / 3.0);
-        const uint8_t base = rb[x];
-        p5[0] = (base == 'A' || base == 'N') ? pm : px;
-        p5[1] = (base == 'C' || base == 'N') ? pm : px;
-        p5[2] = (base == 'G' || base == 'N') ? pm : px;
-        p5[3] = (base == 'T' || base == 'N') ? pm : px;
+        const T t = a * al / ap;
+        const T pm = t * ((T)1 - eb), px = t * (eb / (T)3);
+        p5[0] = (base_c == 'A' || base_c == 'N') ? pm : px;
+        p5[1] = (base_c == 'C' || base_c == 'N') ? pm : px;
+        p5[2] = (base_c == 'G' || base_c == 'N') ? pm : px;
+        p5[3] = (base_c == 'T' || base_c == 'N') ? pm : px;
         p5[4] = pm;  // haplotype 'N' matches everything
       } else {  // S: M^ = (M + I)(m, j-1), D^ = running sum (the L20@2262 termination)
-        const RowScale Sm = row_scale(m, m, qi, qd, r0, err);
-        uu = Sm.a / Sm.b;
+        uu = ap / bp;
         mu = 1;
-        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = 1.0 / Sm.a;
+        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = (T)1 / ap;
       }
       TBlock<T>& B = Tb[row / K];
       const int t = row % K;
-      B.coef[0][t] = (T)uu; B.coef[1][t] = (T)ww; B.coef[2][t] = (T)ep; B.coef[3][t] = (T)mu;
+      B.coef[0][t] = uu; B.coef[1][t] = ww; B.coef[2][t] = ep; B.coef[3][t] = mu;
 #pragma unroll
-      for (int k = 0; k < 5; ++k) B.prior[k][t] = (T)p5[k];
+      for (int k = 0; k < 5; ++k) B.prior[k][t] = p5[k];
     }
   }
 }

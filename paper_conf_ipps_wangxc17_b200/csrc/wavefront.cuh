@@ -53,7 +53,10 @@ __device__ int g_trace_steps;
 constexpr int WF_G = 8;           // virtual lanes per switch group
 constexpr int WF_NCODE = 6;       // A C G T N PAD
 constexpr int WF_PAD = 5;
-constexpr int WF_WARPS = 4;       // warps per CTA
+#ifndef PHMM_WF_WARPS
+#define PHMM_WF_WARPS 4
+#endif
+constexpr int WF_WARPS = PHMM_WF_WARPS;  // warps per CTA
 constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
 constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
 constexpr int WF_KC = 2;          // 16-byte chunks per row set (FP32 K=8 and FP64 K=4 alike)
