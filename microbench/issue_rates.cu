@@ -136,6 +136,34 @@ __global__ void k_x2(const float* in, Out* out) {
   if (s == 1234.5f) out[blockIdx.x].sink = s;
 }
 
+// --- the wavefront cell's FP mix: 2 FFMA2 : 1 scalar FMUL, 8 independent chains ---
+__global__ void k_x2_fmul(const float* in, Out* out) {
+  float2 b = make_float2(in[0], in[3]), c = make_float2(in[1], in[4]);
+  float2 a[8];
+  float f[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) { a[j] = make_float2(in[2] + threadIdx.x + j, in[2] - j); f[j] = in[0] + j; }
+  unsigned long long B = PK(b), C = PK(c);
+  const float g = in[3];
+  __syncthreads();
+  unsigned long long t0 = clock64();
+#pragma unroll 4
+  for (int i = 0; i < ITER; ++i) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(PK(a[j])) : "l"(B), "l"(C));
+      if (j & 1) asm volatile("mul.rn.f32 %0, %0, %1;" : "+f"(f[j]) : "f"(g));
+    }
+  }
+  __syncthreads();
+  unsigned long long t1 = clock64();
+  if (threadIdx.x == 0) out[blockIdx.x].cyc = t1 - t0;
+  float s = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) s += a[j].x + a[j].y + f[j];
+  if (s == 1234.5f) out[blockIdx.x].sink = s;
+}
+
 // --- FFMA2 interleaved 1:1 with an ALU op (LOP3 / FSEL via predicate / PRMT) --
 template <int ALU>  // 0 = lop3, 1 = fsel (setp+selp), 2 = prmt, 3 = mov-free iadd3
 __global__ void k_x2_alu(const float* in, Out* out) {
@@ -382,6 +410,9 @@ int main() {
   run("ffma_rrr_distinct", k_ffma_rrr_distinct, T, Bk, 8, ITER, din, dout, nsm, "fp32 lane-ops (FFMA)");
   run("ffma_imm", k_ffma_imm, T, Bk, 8, ITER, din, dout, nsm, "fp32 lane-ops (FFMA)");
   run("ffma2", k_x2<0>, T, Bk, 16, ITER, din, dout, nsm, "fp32 lane-ops (2 per FFMA2)");
+  run("ffma2_8warps", k_x2<0>, 256, Bk, 16, ITER, din, dout, nsm, "fp32 lane-ops (2 per FFMA2), 8 warps/SM");
+  run("ffma2_fmul_2to1", k_x2_fmul, T, Bk, 20, ITER, din, dout, nsm, "fp32 lane-ops (8 FFMA2 + 4 FMUL)");
+  run("ffma2_fmul_2to1_8warps", k_x2_fmul, 256, Bk, 20, ITER, din, dout, nsm, "fp32 lane-ops, 8 warps/SM");
   run("fmul2", k_x2<1>, T, Bk, 16, ITER, din, dout, nsm, "fp32 lane-ops (2 per FMUL2)");
   run("fadd2", k_x2<2>, T, Bk, 16, ITER, din, dout, nsm, "fp32 lane-ops (2 per FADD2)");
   run("lop3", k_lop3, T, Bk, 8, ITER, din, dout, nsm, "alu lane-ops");

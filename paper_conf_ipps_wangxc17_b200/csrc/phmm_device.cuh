@@ -141,18 +141,22 @@ __device__ __forceinline__ double start_mass_correction(const int32_t* __restric
   return log10((double)ncols_of(n, bucket) / (double)n);
 }
 
-__global__ void k_finalize_fp32(const float* __restrict__ s32, int64_t n_pairs, const int32_t* __restrict__ pairs,
+__global__ void k_finalize_fp32(const float* __restrict__ s32, const int32_t* __restrict__ exp32, int64_t n_pairs,
+                                const int32_t* __restrict__ pairs,
                                 const int64_t* __restrict__ hoff, int bucket, double* __restrict__ out,
                                 uint8_t* __restrict__ status, int32_t* __restrict__ rescue_list,
                                 int64_t* __restrict__ n_rescue, int write_status) {
   const double off = 120.0 * 0.30102999566398119521;
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n_pairs; p += (int64_t)gridDim.x * blockDim.x) {
     const float s = s32[p];
-    if (!(s >= 1e-28f) || !isfinite(s)) {  // NaN-safe: also catches s < 1e-28
+    // NaN-safe: also catches s < 1e-28; exp32 < 0 by 2^23: the ring rescale saturated
+    if (!(s >= 1e-28f) || !isfinite(s) || exp32[p] < -(1 << 23)) {
       const unsigned long long k = atomicAdd(reinterpret_cast<unsigned long long*>(n_rescue), 1ull);
       rescue_list[k] = (int32_t)p;
     } else {
-      out[p] = log10((double)s) - off + start_mass_correction(pairs, hoff, p, bucket);
+      // the ring rescale multiplied the pair's later rows by 2^exp32[p]
+      out[p] = log10((double)s) - (off + (double)exp32[p] * 0.30102999566398119521) +
+               start_mass_correction(pairs, hoff, p, bucket);
       if (write_status) status[p] = 0;
     }
   }

@@ -34,7 +34,7 @@ enum BufId {
   B_SW_REF, B_SW_ROFF, B_SW_ALT, B_SW_AOFF, B_SW_TASKS, B_SW_RES, B_SW_OPS,  // SW host-variant staging
   B_SW_BTSZ, B_SW_BTOFF, B_SW_OPCAP, B_SW_OPOFF, B_SW_BT, B_SW_KEYS, B_SW_VALS, B_SW_OPTMP, B_SW_NOPS,
   B_SW_NOPOFF,
-  B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_COUNT
+  B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_EXP32, B_COUNT
 };
 
 struct Buf {
@@ -305,7 +305,8 @@ phmm_status build_hap_codes(phmm_ctx* c, const DevBatch& d, int64_t total_hc, in
 // (hc, pad region at total_hc) were built by build_hap_codes.
 template <typename T>
 phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_t n, const PassInfo& pi,
-                     int64_t total_tab, const uint8_t* hc, int64_t total_hc, T* out, bool timed) {
+                     int64_t total_tab, const uint8_t* hc, int64_t total_hc, T* out, bool timed,
+                     int32_t* exp_out = nullptr) {
   constexpr int K = WfT<T>::K;
   cudaStream_t s = c->stream;
   Scalars* scal;
@@ -340,7 +341,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   auto P_of = [](int ncols) { return wf_pass_len(ncols); };
   const int p_max = P_of(pi.max_ncols);
   int bps_full = 0;
-  CUDA_TRY(wf_occupancy<T>(WF_WARPS, wf_warp_smem<T>(wf_pass_len(0) + 4) * WF_WARPS, &bps_full));
+  CUDA_TRY(wf_occupancy<T>(false, WF_WARPS, wf_warp_smem<T>(wf_pass_len(0) + 4) * WF_WARPS, &bps_full));
   if (bps_full < 1) return PHMM_E_CUDA;
   const int64_t cta_budget = (int64_t)c->smem_per_sm / bps_full - c->smem_reserved;
   const int ring_full = (int)std::min<int64_t>(
@@ -350,6 +351,10 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     bin_cut = 0;
     while (bin_cut <= kMaxBins && P_of(bin_cut * c->bucket) + 4 <= ring_full) ++bin_cut;
   }
+  // FP32: rows of >= WF_RESCALE_COLS columns run in the long launch (the kernel variant with
+  // the ring rescale)
+  if (sizeof(T) == 4 && pi.max_ncols >= WF_RESCALE_COLS)
+    bin_cut = std::min(bin_cut, (WF_RESCALE_COLS + c->bucket - 1) / c->bucket);
   struct Launch { int bin_lo, bin_hi, warps, ring_len, bps; };
   Launch L[2];
   int nl = 0;
@@ -361,7 +366,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
       const size_t sm = wf_warp_smem<T>(lb.ring_len) * w;
       if (sm > (size_t)c->smem_optin) continue;
       int b = 0;
-      CUDA_TRY(wf_occupancy<T>(w, sm, &b));
+      CUDA_TRY(wf_occupancy<T>(true, w, sm, &b));
       if (b * w > best) { best = b * w; lb.warps = w; lb.bps = b; }
     }
     if (best < 1) return PHMM_E_INVALID_ARG;  // cannot happen for ncols <= kMaxHapLen + 8
@@ -369,8 +374,10 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   }
 
   const int64_t nwarps = (int64_t)c->nsm * L[0].bps * L[0].warps;
+  // work items: ~4 per warp for load balance; a small pass (e.g. the FP64 rescue list)
+  // gets one item per warp instead of fewer, larger items that leave warps idle
   int64_t chunk = (int64_t)(pi.total_blocks / (unsigned long long)(nwarps * 4));
-  if (chunk < 512) chunk = 512;
+  if (chunk < 512) chunk = std::max<int64_t>(64, ((int64_t)pi.total_blocks + nwarps - 1) / nwarps);
   if (chunk > 65536) chunk = 65536;
   const int nbins = kMaxBins + 1;
   k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, chunk, bin_start, item_start);
@@ -412,6 +419,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   A.bucket = c->bucket;
   A.chunk_blocks = chunk;
   A.out = out;
+  A.exp_out = exp_out;
   CUDA_TRY(cudaMemsetAsync(scal->item_counter, 0, sizeof(scal->item_counter), s));
   if (timed) ev_record(c, EV_WF0);
   for (int i = 0; i < nl; ++i) {
@@ -419,8 +427,8 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     A.bin_hi = L[i].bin_hi;
     A.ring_len = L[i].ring_len;
     A.item_counter = &scal->item_counter[i];
-    CUDA_TRY(wf_launch<T>((unsigned)(c->nsm * L[i].bps), L[i].warps, wf_warp_smem<T>(L[i].ring_len) * L[i].warps,
-                          s, A));
+    CUDA_TRY(wf_launch<T>(i == 1, (unsigned)(c->nsm * L[i].bps), L[i].warps,
+                          wf_warp_smem<T>(L[i].ring_len) * L[i].warps, s, A));
     ++c->launches;
   }
   if (timed) ev_record(c, EV_WF1);
@@ -461,12 +469,15 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     ST_TRY(build_hap_codes(c, d, total_hc, pi.max_ncols, &hc));
     float* out32;
     ST_TRY(ws(c, B_OUT32, (size_t)d.n_pairs, &out32));
+    int32_t* exp32;  // powers of 2 applied by the ring rescale of long pairs
+    ST_TRY(ws(c, B_EXP32, (size_t)d.n_pairs, &exp32));
+    CUDA_TRY(cudaMemsetAsync(exp32, 0, sizeof(int32_t) * (size_t)d.n_pairs, s));
     ev_record(c, EV_PREP);
-    ST_TRY(pass_run<float>(c, d, nullptr, d.n_pairs, pi, total_tab, hc, total_hc, out32, true));
+    ST_TRY(pass_run<float>(c, d, nullptr, d.n_pairs, pi, total_tab, hc, total_hc, out32, true, exp32));
     int32_t* rlist;
     ST_TRY(ws(c, B_RLIST, (size_t)d.n_pairs, &rlist));
     CUDA_TRY(cudaMemsetAsync(&scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
-    k_finalize_fp32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out32, d.n_pairs, d.pairs, d.hoff, c->bucket,
+    k_finalize_fp32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out32, exp32, d.n_pairs, d.pairs, d.hoff, c->bucket,
                                                                   dev_out, dev_status, rlist,
                                                                   &scal->n_rescue, dev_status != nullptr);
     LAUNCHED(c);

@@ -161,6 +161,7 @@ struct WfArgs2 {
   int64_t chunk_blocks;
   unsigned int* item_counter;
   T* out;
+  int32_t* exp_out;  // FP32 pass: per output slot, the power of 2 the ring rescale applied
   int ring_len;  // slots, >= P + 4
 };
 
@@ -240,8 +241,12 @@ __device__ __forceinline__ void sts16(uint32_t a, const uint4 v) {
 
 // Steps per pass: every virtual lane sweeps its ncols columns plus the G-step stagger of
 // its switch group; P >= 72 keeps the ring slot of a column written (virtual lane 63)
-// before it is read (virtual lane 0 of the next pass).
+// before it is read (virtual lane 0 of the next pass). Long rows (ncols >= WF_RESCALE_COLS)
+// get 64 more steps, so that virtual lane 63 has finished its whole row when virtual lane
+// 0 of the next pass starts: the ring rescale then sees the full ring row.
+constexpr int WF_RESCALE_COLS = 768;
 __host__ __device__ inline int wf_pass_len(int ncols) {
+  if (ncols >= WF_RESCALE_COLS) return ncols + WF_G + 64;
   return (ncols + WF_G > WF_MIN_P) ? ncols + WF_G : WF_MIN_P;
 }
 // Haplotype code regions: 4 shifted copies per haplotype so that every lane reads its
@@ -292,8 +297,9 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
 }
 
-// One warp streams through blocks [s, s+nblk) of one bin (ncols columns each).
-template <typename T>
+// One warp streams through blocks [s, s+nblk) of one bin (ncols columns each). kLong: the
+// launch of the long-row bins (the only one with the ring rescale compiled in).
+template <typename T, bool kLong>
 __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s, uint32_t xbuf_s,
                                           int lane, int64_t s, int nblk, int ncols, bool trace = false) {
   using V = typename WfT<T>::V;
@@ -337,6 +343,34 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 #ifdef PHMM_DBG_TRACE
   int tstep = 0;
 #endif
+
+  // Ring rescale (FP32 pass, long rows only): when a pair continues from
+  // virtual lane 63 of one pass into virtual lane 0 of the next, its ring row (the row
+  // above virtual lane 0, complete by then: wf_pass_len) is multiplied in place by 2^sh,
+  // sh chosen from the row's max, so long reads stay inside the FP32 range; sh is added
+  // to the pair's exponent slot. Costs nothing in the hot loop but one sample per 4 steps.
+#ifndef PHMM_RING_RESCALE
+#define PHMM_RING_RESCALE 1
+#endif
+  const bool rescale = kLong && PHMM_RING_RESCALE && sizeof(T) == 4 && ncols >= WF_RESCALE_COLS;  // uniform
+  T rmax = 0;  // lane 31: max of M, I, D of virtual lane 63's last row, sampled every 4 columns
+  // slots [0, ncols] *= 2^sh, saturating at 2^110 (returns true if any value saturated: the
+  // sampled max missed a peak, the pair then goes to the FP64 rescue)
+  auto ring_scale = [&](int sh) -> bool {
+    const T f = (T)__int_as_float((127 + sh) << 23);
+    const T cap = (T)__int_as_float((127 + 110) << 23);
+    bool sat = false;
+    __syncwarp();
+    for (int k = lane; k <= ncols; k += 32) {
+      T a, b, c;
+      ring_get3(ring_s + RS * (uint32_t)k, a, b, c);
+      a *= f; b *= f; c *= f;
+      sat |= (a > cap) | (b > cap) | (c > cap);
+      ring_put3(ring_s + RS * (uint32_t)k, fminf(a, cap), fminf(b, cap), fminf(c, cap));
+    }
+    __syncwarp();
+    return __any_sync(0xffffffffu, sat);
+  };
 
   auto step = [&](const int r) {
     if (is31) ring_get3(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
@@ -396,12 +430,33 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     wA_nx2 = __ldg(pA); wB_nx2 = __ldg(pB);
     ++pA; ++pB;
     step(0); step(1); step(2); step(3);
+    if (rescale && is31) rmax = fmaxf(fmaxf(rmax, hi(L.D[K - 1])), fmaxf(hi(L.M[K - 1]), hi(L.I[K - 1])));
   };
 
   for (int q = 0; q <= npass; ++q) {
 #pragma unroll 1
     for (int e = 0; e < NGRP; ++e) {
-      if (e == 0) c0 = -1;                      // virtual lane 0 starts its pass: column -1 next
+      if (e == 0) {
+        c0 = -1;  // virtual lane 0 starts its pass: column -1 next
+        if (rescale) {
+          // lane 0's block of this pass continues the pair of virtual lane 63's last block?
+          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST);
+          const int cont0 = __shfl_sync(0xffffffffu, (int)cont, 0);
+          const float rm = __shfl_sync(0xffffffffu, (float)rmax, 31);
+          int sh = 0;
+          if (cont0 && rm > 0.f && rm <= 3.0e38f) {
+            const int E = ilogbf(rm);
+            // rescale a row that decayed below 2^64 back to 2^80 (below 2^-90 precision may
+            // already be lost: leave it, the pair's sum then fails the 1e-28 test and goes
+            // to the FP64 rescue)
+            if (E >= -90 && E < 64) sh = min(80 - E, 126);
+          }
+          if (sh != 0) {
+            const bool sat = ring_scale(sh);
+            if (is0 && A.exp_out) A.exp_out[dnA.out_idx] += sat ? -(1 << 24) : sh;
+          }
+        }
+      }
       if (e == NGRP - 1) c31B = -1 - (G - 1);  // virtual lane 63
       if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
         const int bA = q * 64 + 2 * lane, bB = bA + 1;
@@ -422,6 +477,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
           ring_get3(ring_s, a, bb, c);
           upM = set_half<0>(upM, a); upI = set_half<0>(upI, bb); upD = set_half<0>(upD, c);
         }
+        if (is31 && grp == NGRP - 1) rmax = 0;  // virtual lane 63 starts a new block
       }
       const int ngroups = (e < NGRP - 1) ? G / 4 : (q < npass ? (P - (NGRP - 1) * G) / 4 : 0);
 #pragma unroll 1
@@ -432,7 +488,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 
 // The kernels are defined in wf.cu (their own translation unit, compiled with
 // -Xptxas -O1: ptxas -O2/-O3 mis-schedules the FP32 kernel -- results silently differ
-// from the -O0/-O1 builds and from the CPU model of the schedule; DESIGN.md §4.6).
+// from the -O0/-O1 builds and from the CPU model of the schedule; DESIGN.md §4.7).
 // phmm_lib.cu reaches them through these host functions.
 // shared memory of one warp: its prior tables and its ring
 template <typename T> __host__ __device__ size_t wf_warp_smem(int ring_len) {
@@ -440,15 +496,16 @@ template <typename T> __host__ __device__ size_t wf_warp_smem(int ring_len) {
   return (size_t)2 * WF_NCODE * WF_KC * 32 * 16 +
          (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) * ring_slot_bytes<T>();
 }
-template <typename T> cudaError_t wf_occupancy(int warps, size_t smem, int* blocks_per_sm);
+template <typename T> cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm);
 template <typename T>
-cudaError_t wf_launch(unsigned grid, int warps, size_t smem, cudaStream_t stream, const WfArgs2<T>& args);
+cudaError_t wf_launch(bool long_rows, unsigned grid, int warps, size_t smem, cudaStream_t stream,
+                      const WfArgs2<T>& args);
 
 #ifdef PHMM_DEFINE_WF
 #ifndef PHMM_F32_MINB
 #define PHMM_F32_MINB 2  // CTAs (of 4 warps) per SM the register budget must allow (255 regs)
 #endif
-template <typename T>
+template <typename T, bool kLong>
 __global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfArgs2<T> A) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
@@ -492,7 +549,7 @@ __global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfAr
     s = advance(s);
     e = (e >= b1) ? b1 : advance(e);
     if (e <= s) continue;
-    wf_stream<T>(A, ptab_s, ring_s, xbuf_s, lane, s, (int)(e - s), bin * A.bucket, it == 0);
+    wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, lane, s, (int)(e - s), bin * A.bucket, it == 0);
     __syncwarp();
   }
 }

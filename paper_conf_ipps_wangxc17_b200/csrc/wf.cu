@@ -1,5 +1,5 @@
 // wf.cu -- translation unit of the wavefront kernels (k_wavefront<float>, <double>).
-// Built with -Xptxas -O1 (see wavefront.cuh / DESIGN.md §4.6); everything else in
+// Built with -Xptxas -O1 (see wavefront.cuh / DESIGN.md §4.7); everything else in
 // libphmm is built at -O3.
 #define PHMM_DEFINE_WF
 #include "wavefront.cuh"
@@ -7,24 +7,33 @@
 namespace phmm {
 
 template <typename T>
-cudaError_t wf_occupancy(int warps, size_t smem, int* blocks_per_sm) {
-  cudaError_t e = cudaFuncSetAttribute(k_wavefront<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_wavefront<T>, warps * 32, smem);
+static void* wf_kernel(bool long_rows) {
+  return long_rows ? reinterpret_cast<void*>(k_wavefront<T, true>) : reinterpret_cast<void*>(k_wavefront<T, false>);
 }
 
 template <typename T>
-cudaError_t wf_launch(unsigned grid, int warps, size_t smem, cudaStream_t stream, const WfArgs2<T>& args) {
-  cudaError_t e = cudaFuncSetAttribute(k_wavefront<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm) {
+  const void* f = wf_kernel<T>(long_rows);
+  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  k_wavefront<T><<<grid, warps * 32, smem, stream>>>(args);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, f, warps * 32, smem);
+}
+
+template <typename T>
+cudaError_t wf_launch(bool long_rows, unsigned grid, int warps, size_t smem, cudaStream_t stream,
+                      const WfArgs2<T>& args) {
+  const void* f = wf_kernel<T>(long_rows);
+  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  if (long_rows) k_wavefront<T, true><<<grid, warps * 32, smem, stream>>>(args);
+  else k_wavefront<T, false><<<grid, warps * 32, smem, stream>>>(args);
   return cudaGetLastError();
 }
 
-template cudaError_t wf_occupancy<float>(int, size_t, int*);
-template cudaError_t wf_occupancy<double>(int, size_t, int*);
-template cudaError_t wf_launch<float>(unsigned, int, size_t, cudaStream_t, const WfArgs2<float>&);
-template cudaError_t wf_launch<double>(unsigned, int, size_t, cudaStream_t, const WfArgs2<double>&);
+template cudaError_t wf_occupancy<float>(bool, int, size_t, int*);
+template cudaError_t wf_occupancy<double>(bool, int, size_t, int*);
+template cudaError_t wf_launch<float>(bool, unsigned, int, size_t, cudaStream_t, const WfArgs2<float>&);
+template cudaError_t wf_launch<double>(bool, unsigned, int, size_t, cudaStream_t, const WfArgs2<double>&);
 
 }  // namespace phmm
 

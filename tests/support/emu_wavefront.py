@@ -19,6 +19,13 @@ The GPU kernel's per-step state was compared against this model with a trace bui
 import numpy as np
 
 G, PADC, MINP = 8, 5, 72
+RESCALE_COLS = 768  # long rows: passes 64 steps longer, ring rescale on
+
+
+def pass_len(ncols):
+    if ncols >= RESCALE_COLS:
+        return ncols + G + 64
+    return max(ncols + G, MINP)
 E = np.float32
 
 
@@ -99,8 +106,8 @@ def hap_code_row(hap, ncols, P):
 TRACE = []
 
 
-def run_stream(blocks, ncols, K):
-    P = max(ncols + G, MINP)
+def run_stream(blocks, ncols, K, rescale=True):
+    P = pass_len(ncols)
     nblk = len(blocks)
     npass = (nblk + 63) // 64
     d0 = E(2.0 ** 120) / E(ncols)
@@ -118,6 +125,7 @@ def run_stream(blocks, ncols, K):
     out = [-1] * V
     ring = np.zeros((P + 8, 3), E)
     res = {}
+    exps = {}
 
     def code_of(v):
         c = col[v]
@@ -154,8 +162,32 @@ def run_stream(blocks, ncols, K):
         TRACE.append(np.stack([M[:, K - 1], I[:, K - 1], D[:, K - 1]], 1).copy())
         col[:] += 1
 
+    rmax = [0.0]
+    rescale = ncols >= RESCALE_COLS
+
+    def ring_scale(sh):
+        # saturating at 2^110: a peak the sampled max missed sends the pair to the FP64 rescue
+        x = ring[0:ncols + 1].astype(np.float64) * 2.0 ** sh
+        ring[0:ncols + 1] = np.minimum(x, 2.0 ** 110).astype(E)
+        return bool(np.any(x > 2.0 ** 110))
+
     for q in range(npass + 1):
         for e in range(8):
+            if rescale and e == 0:
+                # ring rescale: lane 0's block continues the pair of lane 63's
+                b = q * 64
+                cont = q < npass and b < nblk and not blocks[b]["first"]
+                sh = 0
+                if cont and 0 < rmax[0] <= 3.0e38:
+                    Ex = int(np.floor(np.log2(rmax[0])))
+                    if -90 <= Ex < 64:
+                        sh = min(80 - Ex, 126)
+                if sh:
+                    pr_ = blocks[b]["pair"]
+                    sat = ring_scale(sh)
+                    exps[pr_] = exps.get(pr_, 0) + (-(1 << 24) if sat else sh)
+            if e == 7:
+                rmax[0] = 0.0
             for v in range(8 * e, 8 * e + 8):
                 gi = v % G
                 b = q * 64 + v
@@ -182,9 +214,11 @@ def run_stream(blocks, ncols, K):
                 if v == 0:
                     up[0] = ring[0]
             nsteps = G if e < 7 else (P - 7 * G if q < npass else 0)
-            for _ in range(nsteps):
+            for k in range(nsteps):
                 step()
-    return res
+                if rescale and k % 4 == 3:
+                    rmax[0] = max(rmax[0], float(M[63, K - 1]), float(I[63, K - 1]), float(D[63, K - 1]))
+    return res, exps
 
 
 def run_batch(batch, order=None, bucket=4, K=8):
@@ -196,9 +230,9 @@ def run_batch(batch, order=None, bucket=4, K=8):
         r, h = pairs[p]
         n = int(batch.hap_offsets[h + 1] - batch.hap_offsets[h])
         bins.setdefault(ncols_of(n, bucket), []).append(p)
-    out = {}
+    out, exps = {}, {}
     for nc, plist in bins.items():
-        P = max(nc + G, MINP)
+        P = pass_len(nc)
         blocks = []
         for p in plist:
             r, h = pairs[p]
@@ -207,13 +241,20 @@ def run_batch(batch, order=None, bucket=4, K=8):
                                     batch.del_quals[s:e], batch.gcp_quals[s:e], K)
             codes = hap_code_row(batch.hap(h), nc, P)
             for j in range(nb):
-                blocks.append(dict(rows=rows[K * j:K * j + K], codes=codes, pair=p, last=(j == nb - 1),
+                blocks.append(dict(rows=rows[K * j:K * j + K], codes=codes, pair=p, last=(j == nb - 1), first=(j == 0),
                                    rrow=(f % K) if f // K == j else 15))
-        out.update(run_stream(blocks, nc, K))
+        r_, x_ = run_stream(blocks, nc, K)
+        out.update(r_)
+        exps.update(x_)
     res = np.zeros(len(pairs))
     for p in range(len(pairs)):
         r, h = pairs[p]
         n = int(batch.hap_offsets[h + 1] - batch.hap_offsets[h])
         s = out[p]
-        res[p] = (np.log10(s) if s > 0 else -np.inf) - 120 * np.log10(2) + np.log10(ncols_of(n, bucket) / n)
+        x = exps.get(p, 0)
+        if x < -(1 << 23):  # saturated by the ring rescale: the FP64 rescue's job
+            res[p] = np.nan
+            continue
+        res[p] = (np.log10(s) if s > 0 else -np.inf) - (120 + x) * np.log10(2) + \
+            np.log10(ncols_of(n, bucket) / n)
     return res

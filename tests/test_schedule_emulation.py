@@ -31,3 +31,15 @@ def test_emulated_schedule_is_order_independent():
     perm = list(np.random.default_rng(1).permutation(b.n_pairs))
     c = emu.run_batch(b, order=perm)
     assert np.array_equal(a, c)
+
+
+def test_emulated_ring_rescale_long_rows():
+    """Long rows (ncols >= 768): the ring rescale carries pairs far below
+    the FP32 range (log10 P down to about -100) through the FP32 schedule."""
+    b = synth.config_batch("C4", n_regions=1).subset(range(10))
+    ref = oracle.batch_log10(b)
+    got = emu.run_batch(b)
+    assert np.min(ref) < -70
+    ok = np.isfinite(got)
+    assert ok.sum() >= 8
+    assert np.max(np.abs(got[ok] - ref[ok])) < 1e-3

@@ -1,5 +1,6 @@
 #!/bin/bash
-# One GPU round: smoke, full bench line, launch list (ncu timing pass), one ncu --set full of the FP32 kernel.
+# One GPU round: smoke, full bench line, launch list (ncu timing pass), ncu --set full of the
+# FP32 and FP64 wavefront kernels (C2), shared-memory bank conflicts on the striped C4 path.
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
 python bench.py --steps 10 --warmup 3 > gpurun_out/bench.json 2> gpurun_out/bench.err; tail -2 gpurun_out/bench.err; cat gpurun_out/bench.json
@@ -8,3 +9,14 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
 ncu --set full --clock-control none --import-source on --kernel-name-base mangled -k regex:k_wavefrontIf -s 1 -c 1 -o gpurun_out/prof_wf32 \
     python bench.py --steps 1 --warmup 1 --profile-steps --no-e2e --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
 tail -1 gpurun_out/ncu_full.log
+ncu --set full --clock-control none --import-source on --kernel-name-base mangled -k regex:k_wavefrontId -s 1 -c 1 -o gpurun_out/prof_wf64 \
+    python bench.py --steps 1 --warmup 1 --profile-steps --no-e2e --no-cpu-baseline > gpurun_out/prof_wf64.log 2>&1
+tail -1 gpurun_out/prof_wf64.log
+ncu --clock-control none --kernel-name-base mangled -k regex:k_wavefrontIf -c 1 --csv --metrics \
+l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum,l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_st.sum,\
+l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum,l1tex__data_pipe_lsu_wavefronts_mem_shared_op_st.sum,\
+smsp__inst_executed_op_shared_ld.sum,smsp__inst_executed_op_shared_st.sum,smsp__inst_executed_shfl.sum,\
+smsp__issue_active.avg.pct_of_peak_sustained_active,sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active,\
+sm__warps_active.avg.pct_of_peak_sustained_active,launch__registers_per_thread,gpu__time_duration.sum \
+  python bench.py --workload C4 --regions 32 --steps 1 --warmup 1 --profile-steps --no-e2e --no-cpu-baseline \
+  > gpurun_out/ncu_c4_banks.csv 2> gpurun_out/ncu_c4_banks.err
