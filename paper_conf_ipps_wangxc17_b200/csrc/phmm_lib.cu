@@ -363,7 +363,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     Launch lb{bin_cut, kMaxBins + 1, 0, p_max + 4, 0};
     int best = 0;
     for (int w = WF_WARPS; w >= 1; w >>= 1) {
-      const size_t sm = wf_warp_smem<T>(lb.ring_len) * w;
+      const size_t sm = wf_warp_smem<T, true>(lb.ring_len) * w;
       if (sm > (size_t)c->smem_optin) continue;
       int b = 0;
       CUDA_TRY(wf_occupancy<T>(true, w, sm, &b));
@@ -427,8 +427,8 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     A.bin_hi = L[i].bin_hi;
     A.ring_len = L[i].ring_len;
     A.item_counter = &scal->item_counter[i];
-    CUDA_TRY(wf_launch<T>(i == 1, (unsigned)(c->nsm * L[i].bps), L[i].warps,
-                          wf_warp_smem<T>(L[i].ring_len) * L[i].warps, s, A));
+    const size_t smem = (i == 1 ? wf_warp_smem<T, true>(L[i].ring_len) : wf_warp_smem<T>(L[i].ring_len)) * L[i].warps;
+    CUDA_TRY(wf_launch<T>(i == 1, (unsigned)(c->nsm * L[i].bps), L[i].warps, smem, s, A));
     ++c->launches;
   }
   if (timed) ev_record(c, EV_WF1);

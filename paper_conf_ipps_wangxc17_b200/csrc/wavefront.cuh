@@ -224,7 +224,41 @@ __device__ __forceinline__ void ring_get3(uint32_t a, double& x, double& y, doub
   asm volatile("ld.shared.v2.f64 {%0, %1}, [%3];\n\tld.shared.f64 %2, [%3+16];"
                : "=d"(x), "=d"(y), "=d"(z) : "r"(a) : "memory");
 }
-template <typename T> __host__ __device__ constexpr uint32_t ring_slot_bytes() { return sizeof(T) == 4 ? 16u : 32u; }
+// ring slot: 16 / 32 bytes (one vector load); packed 24 bytes (three scalar loads) in the
+// FP64 long-row kernel, where the ring limits occupancy (C4 rescue: 3 -> 4 warps per SM;
+// packing the FP32 long-row ring measured slower)
+template <typename T, bool kLong = false> __host__ __device__ constexpr bool ring_packed() {
+  return kLong && sizeof(T) == 8;
+}
+template <typename T, bool kLong = false> __host__ __device__ constexpr uint32_t ring_slot_bytes() {
+  return ring_packed<T, kLong>() ? 3u * (uint32_t)sizeof(T) : (sizeof(T) == 4 ? 16u : 32u);
+}
+template <typename T>
+__device__ __forceinline__ void ring_get3p(uint32_t a, T& x, T& y, T& z) {
+  if constexpr (sizeof(T) == 4)
+    asm volatile("ld.shared.f32 %0, [%3];\n\tld.shared.f32 %1, [%3+4];\n\tld.shared.f32 %2, [%3+8];"
+                 : "=f"(x), "=f"(y), "=f"(z) : "r"(a) : "memory");
+  else
+    asm volatile("ld.shared.f64 %0, [%3];\n\tld.shared.f64 %1, [%3+8];\n\tld.shared.f64 %2, [%3+16];"
+                 : "=d"(x), "=d"(y), "=d"(z) : "r"(a) : "memory");
+}
+template <typename T>
+__device__ __forceinline__ void ring_put3p(uint32_t a, T x, T y, T z) {
+  if constexpr (sizeof(T) == 4)
+    asm volatile("st.shared.f32 [%0], %1;\n\tst.shared.f32 [%0+4], %2;\n\tst.shared.f32 [%0+8], %3;"
+                 :: "r"(a), "f"(x), "f"(y), "f"(z) : "memory");
+  else
+    asm volatile("st.shared.f64 [%0], %1;\n\tst.shared.f64 [%0+8], %2;\n\tst.shared.f64 [%0+16], %3;"
+                 :: "r"(a), "d"(x), "d"(y), "d"(z) : "memory");
+}
+template <bool kPacked, typename T>
+__device__ __forceinline__ void rget(uint32_t a, T& x, T& y, T& z) {
+  if constexpr (kPacked) ring_get3p<T>(a, x, y, z); else ring_get3(a, x, y, z);
+}
+template <bool kPacked, typename T>
+__device__ __forceinline__ void rput(uint32_t a, T x, T y, T z) {
+  if constexpr (kPacked) ring_put3p<T>(a, x, y, z); else ring_put3(a, x, y, z);
+}
 
 // 16-byte shared load reinterpreted as 4 floats or 2 doubles
 __device__ __forceinline__ void lds16(uint32_t a, float* v) {
@@ -297,6 +331,27 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
 }
 
+// Ring slots [0, ncols] *= 2^sh, saturating at 2^110; true if any value saturated (the
+// sampled max missed a peak: the pair then goes to the FP64 rescue). Not inlined: it runs
+// once per rescaled pass and must not perturb the register allocation of the hot loop.
+template <typename T, bool kPacked>
+__device__ __noinline__ bool wf_ring_scale(uint32_t ring_s, int ncols, int lane, int sh) {
+  constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
+  const T f = (T)__int_as_float((127 + sh) << 23);
+  const T cap = (T)__int_as_float((127 + 110) << 23);
+  bool sat = false;
+  __syncwarp();
+  for (int k = lane; k <= ncols; k += 32) {
+    T a, b, c;
+    rget<kPacked>(ring_s + RS * (uint32_t)k, a, b, c);
+    a *= f; b *= f; c *= f;
+    sat |= (a > cap) | (b > cap) | (c > cap);
+    rput<kPacked>(ring_s + RS * (uint32_t)k, fminf(a, cap), fminf(b, cap), fminf(c, cap));
+  }
+  __syncwarp();
+  return __any_sync(0xffffffffu, sat);
+}
+
 // One warp streams through blocks [s, s+nblk) of one bin (ncols columns each). kLong: the
 // launch of the long-row bins (the only one with the ring rescale compiled in).
 template <typename T, bool kLong>
@@ -308,7 +363,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   constexpr int G = WF_G;            // virtual lanes per switch group
   constexpr int NGRP = 64 / G;       // switch events per pass
   constexpr int LPG = G / 2;         // physical lanes per group
-  constexpr uint32_t RS = ring_slot_bytes<T>();
+  constexpr uint32_t RS = ring_slot_bytes<T, kLong>();
   const int grp = lane / LPG;
   const int giA = 2 * (lane % LPG), giB = giA + 1;  // position of each half inside its group
   const T d0 = (T)ldexp(1.0, WfT<T>::kScaleExp) / (T)ncols;  // virtual row 0
@@ -354,26 +409,9 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 #endif
   const bool rescale = kLong && PHMM_RING_RESCALE && sizeof(T) == 4 && ncols >= WF_RESCALE_COLS;  // uniform
   T rmax = 0;  // lane 31: max of M, I, D of virtual lane 63's last row, sampled every 4 columns
-  // slots [0, ncols] *= 2^sh, saturating at 2^110 (returns true if any value saturated: the
-  // sampled max missed a peak, the pair then goes to the FP64 rescue)
-  auto ring_scale = [&](int sh) -> bool {
-    const T f = (T)__int_as_float((127 + sh) << 23);
-    const T cap = (T)__int_as_float((127 + 110) << 23);
-    bool sat = false;
-    __syncwarp();
-    for (int k = lane; k <= ncols; k += 32) {
-      T a, b, c;
-      ring_get3(ring_s + RS * (uint32_t)k, a, b, c);
-      a *= f; b *= f; c *= f;
-      sat |= (a > cap) | (b > cap) | (c > cap);
-      ring_put3(ring_s + RS * (uint32_t)k, fminf(a, cap), fminf(b, cap), fminf(c, cap));
-    }
-    __syncwarp();
-    return __any_sync(0xffffffffu, sat);
-  };
 
   auto step = [&](const int r) {
-    if (is31) ring_get3(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
+    if (is31) rget<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
     // code byte r (= code*WF_CB) placed in byte 1 -> the code's rows in the table
     const uint32_t oA = __byte_perm(wA, 0, 0x4404 + (r << 4)), oB = __byte_perm(wB, 0, 0x4404 + (r << 4));
     T prA[K], prB[K];
@@ -391,16 +429,16 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     const T sI = is31 ? rvI : i3b;
     const T sD = is31 ? rvD : d3b;
     if (is31 && (unsigned)(c31B + 1) <= (unsigned)ncols)  // -1 <= c31B < ncols
-      ring_put3(ring_s + RS * (uint32_t)(c31B + 1), m3b, i3b, d3b);
+      rput<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c31B + 1), m3b, i3b, d3b);
     dgM = upM; dgI = upI; dgD = upD;
     // next step: half A's row above = lane-1's half B; half B's row above = this lane's half A
 #if PHMM_XCHG_SMEM
     // design A (Listing 2a, L20@44): write, synchronise, read through a
     // shared-memory line buffer (one slot per lane) instead of the shuffle
-    ring_put3(xbuf_s + RS * (uint32_t)lane, sM, sI, sD);
+    rput<ring_packed<T, kLong>()>(xbuf_s + RS * (uint32_t)lane, sM, sI, sD);
     __syncwarp();
     T xM, xI, xD;
-    ring_get3(xbuf_s + RS * (uint32_t)src, xM, xI, xD);
+    rget<ring_packed<T, kLong>()>(xbuf_s + RS * (uint32_t)src, xM, xI, xD);
     __syncwarp();
     upM = pk(xM, m3a);
     upI = pk(xI, i3a);
@@ -430,7 +468,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     wA_nx2 = __ldg(pA); wB_nx2 = __ldg(pB);
     ++pA; ++pB;
     step(0); step(1); step(2); step(3);
-    if (rescale && is31) rmax = fmaxf(fmaxf(rmax, hi(L.D[K - 1])), fmaxf(hi(L.M[K - 1]), hi(L.I[K - 1])));
+    if (kLong && is31) rmax = fmaxf(fmaxf(rmax, hi(L.D[K - 1])), fmaxf(hi(L.M[K - 1]), hi(L.I[K - 1])));
   };
 
   for (int q = 0; q <= npass; ++q) {
@@ -452,7 +490,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
             if (E >= -90 && E < 64) sh = min(80 - E, 126);
           }
           if (sh != 0) {
-            const bool sat = ring_scale(sh);
+            const bool sat = wf_ring_scale<T, ring_packed<T, kLong>()>(ring_s, ncols, lane, sh);
             if (is0 && A.exp_out) A.exp_out[dnA.out_idx] += sat ? -(1 << 24) : sh;
           }
         }
@@ -474,7 +512,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
         if (bB + 64 < nblk) dnB = A.blk[s + bB + 64];
         if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
           T a, bb, c;
-          ring_get3(ring_s, a, bb, c);
+          rget<ring_packed<T, kLong>()>(ring_s, a, bb, c);
           upM = set_half<0>(upM, a); upI = set_half<0>(upI, bb); upD = set_half<0>(upD, c);
         }
         if (is31 && grp == NGRP - 1) rmax = 0;  // virtual lane 63 starts a new block
@@ -491,10 +529,12 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 // from the -O0/-O1 builds and from the CPU model of the schedule).
 // phmm_lib.cu reaches them through these host functions.
 // shared memory of one warp: its prior tables and its ring
-template <typename T> __host__ __device__ size_t wf_warp_smem(int ring_len) {
-  // prior tables, ring, and (design-A ablation only) the exchange line buffer
-  return (size_t)2 * WF_NCODE * WF_KC * 32 * 16 +
-         (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) * ring_slot_bytes<T>();
+template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_smem(int ring_len) {
+  // prior tables, ring, and (design-A ablation only) the exchange line buffer; a multiple of
+  // 16 bytes so that every warp's tables stay 16-byte aligned
+  const size_t b = (size_t)2 * WF_NCODE * WF_KC * 32 * 16 +
+                   (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) * ring_slot_bytes<T, kLong>();
+  return (b + 15) & ~(size_t)15;
 }
 template <typename T> cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm);
 template <typename T>
@@ -512,12 +552,12 @@ __global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfAr
   const int wib = threadIdx.x >> 5;
   // per warp: prior tables [2 halves][6 codes][WF_KC chunks][32 lanes] x 16 B, then the ring
   constexpr uint32_t kTabBytes = 2 * WF_NCODE * WF_KC * 32 * 16;
-  const uint32_t per_warp = (uint32_t)wf_warp_smem<T>(A.ring_len);
+  const uint32_t per_warp = (uint32_t)wf_warp_smem<T, kLong>(A.ring_len);
   unsigned char* base = smem_raw + (size_t)wib * per_warp;
   for (uint32_t i = 4 * lane; i < per_warp; i += 128) *reinterpret_cast<uint32_t*>(base + i) = 0u;
   __syncwarp();
   const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
-  const uint32_t xbuf_s = ring_s + (uint32_t)A.ring_len * ring_slot_bytes<T>();  // design A only
+  const uint32_t xbuf_s = ring_s + (uint32_t)A.ring_len * ring_slot_bytes<T, kLong>();  // design A only
   // work item it of the launch: chunk k of bin b (binary search in item_start)
   const unsigned long long it0 = A.item_start[A.bin_lo], it1 = A.item_start[A.bin_hi];
   while (true) {
