@@ -336,17 +336,24 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
 // once per rescaled pass and must not perturb the register allocation of the hot loop.
 template <typename T, bool kPacked>
 __device__ __noinline__ bool wf_ring_scale(uint32_t ring_s, int ncols, int lane, int sh) {
+  // the slots as a flat array of T (FP32: the 4th word of a 16-byte slot is padding and is
+  // scaled too): consecutive lanes on consecutive words, no bank conflicts
   constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
+  const int nw = (ncols + 1) * (int)(RS / sizeof(T));
   const T f = (T)__int_as_float((127 + sh) << 23);
   const T cap = (T)__int_as_float((127 + 110) << 23);
   bool sat = false;
   __syncwarp();
-  for (int k = lane; k <= ncols; k += 32) {
-    T a, b, c;
-    rget<kPacked>(ring_s + RS * (uint32_t)k, a, b, c);
-    a *= f; b *= f; c *= f;
-    sat |= (a > cap) | (b > cap) | (c > cap);
-    rput<kPacked>(ring_s + RS * (uint32_t)k, fminf(a, cap), fminf(b, cap), fminf(c, cap));
+  for (int k = lane; k < nw; k += 32) {
+    const uint32_t a = ring_s + (uint32_t)(k * (int)sizeof(T));
+    T x;
+    if constexpr (sizeof(T) == 4) asm volatile("ld.shared.f32 %0, [%1];" : "=f"(x) : "r"(a) : "memory");
+    else asm volatile("ld.shared.f64 %0, [%1];" : "=d"(x) : "r"(a) : "memory");
+    x *= f;
+    sat |= x > cap;
+    x = fmin(x, cap);
+    if constexpr (sizeof(T) == 4) asm volatile("st.shared.f32 [%0], %1;" :: "r"(a), "f"(x) : "memory");
+    else asm volatile("st.shared.f64 [%0], %1;" :: "r"(a), "d"(x) : "memory");
   }
   __syncwarp();
   return __any_sync(0xffffffffu, sat);
