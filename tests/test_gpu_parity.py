@@ -227,6 +227,32 @@ def test_full_c2_sampled(ctx32):
     assert 0 < np.sum(st == 1) < b.n_pairs // 10
 
 
+@pytest.mark.parametrize("cfg,regions", [("C4", 256), ("C5", 8192), ("C3", 4096)])
+def test_bench_configs_sampled(ctx32, cfg, regions):
+    """The other bench workloads at the size bench.py times them (C4: 16,384 pairs of
+    1,000 x 1,500 with the ring rescale; C5-shaped shard: 2^21 mixed pairs; C3: ~1e6 mixed
+    pairs): a seeded sample of pairs plus rescued and ring-rescaled pairs against the oracle."""
+    import torch
+
+    b = synth.config_batch(cfg, n_regions=regions)
+    db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+    out, st = ctx32.compute_batch_dev(db)
+    torch.cuda.synchronize()
+    out = out.cpu().numpy()
+    st = st.cpu().numpy()
+    rng = np.random.default_rng(7)
+    cells = b.pair_cells()
+    k = max(40, int(2e9 / cells.mean()) // 10)  # ~2e8 oracle cells
+    sample = np.unique(np.concatenate([rng.choice(b.n_pairs, min(k, b.n_pairs), replace=False),
+                                       rng.permutation(np.nonzero(st != 0)[0])[:k // 4]]))
+    ref = oracle.batch_log10(b, pair_idx=sample)
+    _check(out[sample], ref, "fp32")
+    if cfg == "C4":
+        # pairs far below the FP32 range come back from the FP32 pass (ring rescale)
+        fp32_low = (st[sample] == 0) & (ref < -70)
+        assert fp32_low.sum() > 0
+
+
 def _long_short_mix(seed, n_long, n_short, long_range=(4000, 4094)):
     """Haplotypes up to the maximum length (4094) mixed with short ones: the long
     bins run in the second, reduced-occupancy wavefront launch."""
