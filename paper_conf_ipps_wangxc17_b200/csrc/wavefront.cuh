@@ -334,8 +334,27 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
 // Ring slots [0, ncols] *= 2^sh, saturating at 2^110; true if any value saturated (the
 // sampled max missed a peak: the pair then goes to the FP64 rescue). Not inlined: it runs
 // once per rescaled pass and must not perturb the register allocation of the hot loop.
+// Max of the ring row (slots [0, ncols], every value incl. the FP32 slot padding, which is
+// 0 or a scaled copy of real values), reduced over the warp.
 template <typename T, bool kPacked>
-__device__ __noinline__ bool wf_ring_scale(uint32_t ring_s, int ncols, int lane, int sh) {
+__device__ __forceinline__ T wf_ring_max(uint32_t ring_s, int ncols, int lane) {
+  constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
+  const int nw = (ncols + 1) * (int)(RS / sizeof(T));
+  T m = 0;
+  __syncwarp();
+  for (int k = lane; k < nw; k += 32) {
+    const uint32_t a = ring_s + (uint32_t)(k * (int)sizeof(T));
+    T x;
+    if constexpr (sizeof(T) == 4) asm volatile("ld.shared.f32 %0, [%1];" : "=f"(x) : "r"(a) : "memory");
+    else asm volatile("ld.shared.f64 %0, [%1];" : "=d"(x) : "r"(a) : "memory");
+    m = fmax(m, x);
+  }
+  for (int o = 16; o > 0; o >>= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+  return m;
+}
+
+template <typename T, bool kPacked>
+__device__ __forceinline__ bool wf_ring_scale(uint32_t ring_s, int ncols, int lane, int sh) {
   // the slots as a flat array of T (FP32: the 4th word of a 16-byte slot is padding and is
   // scaled too): consecutive lanes on consecutive words, no bank conflicts
   constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
@@ -357,6 +376,23 @@ __device__ __noinline__ bool wf_ring_scale(uint32_t ring_s, int ncols, int lane,
   }
   __syncwarp();
   return __any_sync(0xffffffffu, sat);
+}
+
+// The ring rescale decision of one pass, all lanes: if lane 0's block
+// continues the pair of the ring row (`cont` of lane 0) and the row's max has decayed below
+// 2^64 (but not below 2^-90), scale the row to 2^80 and add the power of 2 to the pair's
+// exponent slot (lane 0; a saturated row marks the pair for the FP64 rescue). Not inlined,
+// so that it leaves the hot loop's register allocation alone.
+template <typename T, bool kPacked>
+__device__ __noinline__ void wf_ring_rescale(uint32_t ring_s, int ncols, int lane, bool cont, int32_t* exp_slot) {
+  if (!__shfl_sync(0xffffffffu, (int)cont, 0)) return;
+  const float rm = (float)wf_ring_max<T, kPacked>(ring_s, ncols, lane);
+  if (!(rm > 0.f && rm <= 3.0e38f)) return;
+  const int E = ilogbf(rm);
+  if (E < -90 || E >= 64) return;
+  const int sh = min(80 - E, 126);
+  const bool sat = wf_ring_scale<T, kPacked>(ring_s, ncols, lane, sh);
+  if (lane == 0 && exp_slot) *exp_slot += sat ? -(1 << 24) : sh;
 }
 
 // One warp streams through blocks [s, s+nblk) of one bin (ncols columns each). kLong: the
@@ -410,12 +446,12 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   // virtual lane 63 of one pass into virtual lane 0 of the next, its ring row (the row
   // above virtual lane 0, complete by then: wf_pass_len) is multiplied in place by 2^sh,
   // sh chosen from the row's max, so long reads stay inside the FP32 range; sh is added
-  // to the pair's exponent slot. Costs nothing in the hot loop but one sample per 4 steps.
+  // to the pair's exponent slot. Costs nothing in the hot loop: the row max is read from the
+  // ring itself once per pass.
 #ifndef PHMM_RING_RESCALE
 #define PHMM_RING_RESCALE 1
 #endif
-  const bool rescale = kLong && PHMM_RING_RESCALE && sizeof(T) == 4 && ncols >= WF_RESCALE_COLS;  // uniform
-  T rmax = 0;  // lane 31: max of M, I, D of virtual lane 63's last row, sampled every 4 columns
+  constexpr bool rescale = kLong && PHMM_RING_RESCALE && sizeof(T) == 4;  // long-row launch: ncols >= WF_RESCALE_COLS
 
   auto step = [&](const int r) {
     if (is31) rget<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
@@ -475,7 +511,6 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     wA_nx2 = __ldg(pA); wB_nx2 = __ldg(pB);
     ++pA; ++pB;
     step(0); step(1); step(2); step(3);
-    if (kLong && is31) rmax = fmaxf(fmaxf(rmax, hi(L.D[K - 1])), fmaxf(hi(L.M[K - 1]), hi(L.I[K - 1])));
   };
 
   for (int q = 0; q <= npass; ++q) {
@@ -483,23 +518,12 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     for (int e = 0; e < NGRP; ++e) {
       if (e == 0) {
         c0 = -1;  // virtual lane 0 starts its pass: column -1 next
-        if (rescale) {
+        if constexpr (rescale) {
           // lane 0's block of this pass continues the pair of virtual lane 63's last block?
-          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST);
-          const int cont0 = __shfl_sync(0xffffffffu, (int)cont, 0);
-          const float rm = __shfl_sync(0xffffffffu, (float)rmax, 31);
-          int sh = 0;
-          if (cont0 && rm > 0.f && rm <= 3.0e38f) {
-            const int E = ilogbf(rm);
-            // rescale a row that decayed below 2^64 back to 2^80 (below 2^-90 precision may
-            // already be lost: leave it, the pair's sum then fails the 1e-28 test and goes
-            // to the FP64 rescue)
-            if (E >= -90 && E < 64) sh = min(80 - E, 126);
-          }
-          if (sh != 0) {
-            const bool sat = wf_ring_scale<T, ring_packed<T, kLong>()>(ring_s, ncols, lane, sh);
-            if (is0 && A.exp_out) A.exp_out[dnA.out_idx] += sat ? -(1 << 24) : sh;
-          }
+          // (rows shorter than WF_RESCALE_COLS have no complete ring row at the pass start)
+          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && ncols >= WF_RESCALE_COLS;
+          wf_ring_rescale<T, ring_packed<T, kLong>()>(ring_s, ncols, lane, cont,
+                                                      A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
         }
       }
       if (e == NGRP - 1) c31B = -1 - (G - 1);  // virtual lane 63
@@ -522,7 +546,6 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
           rget<ring_packed<T, kLong>()>(ring_s, a, bb, c);
           upM = set_half<0>(upM, a); upI = set_half<0>(upI, bb); upD = set_half<0>(upD, c);
         }
-        if (is31 && grp == NGRP - 1) rmax = 0;  // virtual lane 63 starts a new block
       }
       const int ngroups = (e < NGRP - 1) ? G / 4 : (q < npass ? (P - (NGRP - 1) * G) / 4 : 0);
 #pragma unroll 1

@@ -162,7 +162,6 @@ def run_stream(blocks, ncols, K, rescale=True):
         TRACE.append(np.stack([M[:, K - 1], I[:, K - 1], D[:, K - 1]], 1).copy())
         col[:] += 1
 
-    rmax = [0.0]
     rescale = ncols >= RESCALE_COLS
 
     def ring_scale(sh):
@@ -178,16 +177,15 @@ def run_stream(blocks, ncols, K, rescale=True):
                 b = q * 64
                 cont = q < npass and b < nblk and not blocks[b]["first"]
                 sh = 0
-                if cont and 0 < rmax[0] <= 3.0e38:
-                    Ex = int(np.floor(np.log2(rmax[0])))
+                rm = float(np.max(ring[0:ncols + 1])) if cont else 0.0  # the whole ring row
+                if cont and 0 < rm <= 3.0e38:
+                    Ex = int(np.floor(np.log2(rm)))
                     if -90 <= Ex < 64:
                         sh = min(80 - Ex, 126)
                 if sh:
                     pr_ = blocks[b]["pair"]
                     sat = ring_scale(sh)
                     exps[pr_] = exps.get(pr_, 0) + (-(1 << 24) if sat else sh)
-            if e == 7:
-                rmax[0] = 0.0
             for v in range(8 * e, 8 * e + 8):
                 gi = v % G
                 b = q * 64 + v
@@ -216,8 +214,6 @@ def run_stream(blocks, ncols, K, rescale=True):
             nsteps = G if e < 7 else (P - 7 * G if q < npass else 0)
             for k in range(nsteps):
                 step()
-                if rescale and k % 4 == 3:
-                    rmax[0] = max(rmax[0], float(M[63, K - 1]), float(I[63, K - 1]), float(D[63, K - 1]))
     return res, exps
 
 
