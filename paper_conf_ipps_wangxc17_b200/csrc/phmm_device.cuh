@@ -197,30 +197,67 @@ __global__ void k_rescue_items(const int32_t* __restrict__ pairs, const int32_t*
 }
 
 // exclusive scan of bins + work items (single block; nbins <= kMaxBins)
-__global__ void k_scan_bins(const unsigned long long* __restrict__ bin_blocks, int nbins, int64_t chunk,
-                            unsigned long long* __restrict__ bin_start, unsigned long long* __restrict__ item_start) {
-  __shared__ unsigned long long sb[1024], si[1024];
-  // serial-by-tile scan: nbins is a few thousand at most
-  unsigned long long carry_b = 0, carry_i = 0;
+// Work items of each bin (the length-binned scheduler). A launch runs the
+// bins [0, cut) or [cut, nbins); in launch order, its blocks before the last 1/tail_div of
+// the launch's blocks are cut into items of `chunk` blocks, the rest into items of `chunk_s`
+// blocks, so the last items of a launch are short and its warps finish together (guided
+// self-scheduling). tail_div = 0: all items full-size. bin_nbig[b] = full-size items of bin b.
+__device__ __forceinline__ unsigned long long block_scan_1024(unsigned long long v, unsigned long long* sh,
+                                                              unsigned long long* total) {
+  sh[threadIdx.x] = v;
+  __syncthreads();
+  for (int off = 1; off < 1024; off <<= 1) {
+    const unsigned long long a = (threadIdx.x >= off) ? sh[threadIdx.x - off] : 0ull;
+    __syncthreads();
+    sh[threadIdx.x] += a;
+    __syncthreads();
+  }
+  const unsigned long long incl = sh[threadIdx.x];
+  *total = sh[1023];
+  __syncthreads();
+  return incl - v;  // exclusive
+}
+
+__global__ void __launch_bounds__(1024) k_scan_bins(const unsigned long long* __restrict__ bin_blocks, int nbins,
+                                                    int cut, int64_t chunk, int64_t chunk_s, int tail_div,
+                                                    unsigned long long* __restrict__ bin_start,
+                                                    unsigned long long* __restrict__ item_start,
+                                                    unsigned long long* __restrict__ bin_nbig) {
+  __shared__ unsigned long long sh[1024];
+  // pass 1: first block of every bin (serial-by-tile scan: nbins is a few thousand at most)
+  unsigned long long carry = 0, tot;
   for (int base = 0; base < nbins; base += 1024) {
     const int i = base + threadIdx.x;
     const unsigned long long vb = (i < nbins) ? bin_blocks[i] : 0ull;
-    const unsigned long long vi = (i < nbins) ? (vb + chunk - 1) / chunk : 0ull;
-    sb[threadIdx.x] = vb; si[threadIdx.x] = vi;
-    __syncthreads();
-    for (int off = 1; off < 1024; off <<= 1) {
-      unsigned long long ab = 0, ai = 0;
-      if (threadIdx.x >= off) { ab = sb[threadIdx.x - off]; ai = si[threadIdx.x - off]; }
-      __syncthreads();
-      sb[threadIdx.x] += ab; si[threadIdx.x] += ai;
-      __syncthreads();
-    }
-    if (i < nbins) { bin_start[i] = carry_b + sb[threadIdx.x] - vb; item_start[i] = carry_i + si[threadIdx.x] - vi; }
-    const unsigned long long tb = sb[1023], ti = si[1023];
-    __syncthreads();
-    carry_b += tb; carry_i += ti;
+    const unsigned long long ex = block_scan_1024(vb, sh, &tot);
+    if (i < nbins) bin_start[i] = carry + ex;
+    carry += tot;
   }
-  if (threadIdx.x == 0) { bin_start[nbins] = carry_b; item_start[nbins] = carry_i; }
+  if (threadIdx.x == 0) bin_start[nbins] = carry;
+  __syncthreads();
+  const int c = cut < 0 ? 0 : (cut > nbins ? nbins : cut);
+  const unsigned long long L0 = bin_start[c], L1 = carry - L0;  // blocks of the two launches
+  const unsigned long long thr0 = tail_div > 0 ? L0 - L0 / tail_div : L0;
+  const unsigned long long thr1 = L0 + (tail_div > 0 ? L1 - L1 / tail_div : L1);
+  // pass 2: items per bin
+  carry = 0;
+  for (int base = 0; base < nbins; base += 1024) {
+    const int i = base + threadIdx.x;
+    unsigned long long vi = 0;
+    if (i < nbins) {
+      const unsigned long long vb = bin_blocks[i], s0 = bin_start[i];
+      const unsigned long long thr = (i < c) ? thr0 : thr1;
+      const unsigned long long big = thr <= s0 ? 0ull : (thr - s0 < vb ? thr - s0 : vb);
+      const unsigned long long nbig = (big == vb) ? (vb + chunk - 1) / chunk : big / chunk;
+      const unsigned long long used = nbig * chunk < vb ? nbig * chunk : vb;
+      vi = nbig + (vb - used + chunk_s - 1) / chunk_s;
+      bin_nbig[i] = nbig;
+    }
+    const unsigned long long ex = block_scan_1024(vi, sh, &tot);
+    if (i < nbins) item_start[i] = carry + ex;
+    carry += tot;
+  }
+  if (threadIdx.x == 0) item_start[nbins] = carry;
 }
 
 }  // namespace phmm

@@ -215,7 +215,7 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   const int nb1 = kMaxBins + 2;
-  unsigned long long* bins;  // [blocks | pairs | - | start | item_start], nb1 each
+  unsigned long long* bins;  // [blocks | pairs | nbig | start | item_start], nb1 each
   ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
   int32_t *pair_bin, *pair_nb;
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
@@ -314,7 +314,8 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   const int nb1 = kMaxBins + 2;
   unsigned long long* bins;
   ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
-  unsigned long long *bin_blocks = bins, *bin_start = bins + 3 * nb1, *item_start = bins + 4 * nb1;
+  unsigned long long *bin_blocks = bins, *bin_nbig = bins + 2 * nb1, *bin_start = bins + 3 * nb1,
+                     *item_start = bins + 4 * nb1;
   int32_t *pair_bin, *pair_nb, *item_read = nullptr, *pair_item = nullptr;
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
   ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
@@ -377,10 +378,17 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   // work items: ~4 per warp for load balance; a small pass (e.g. the FP64 rescue list)
   // gets one item per warp instead of fewer, larger items that leave warps idle
   int64_t chunk = (int64_t)(pi.total_blocks / (unsigned long long)(nwarps * 4));
-  if (chunk < 512) chunk = std::max<int64_t>(64, ((int64_t)pi.total_blocks + nwarps - 1) / nwarps);
+  int tail_div = WF_TAIL_DIV;
+  if (chunk < 512) {
+    chunk = std::max<int64_t>(64, ((int64_t)pi.total_blocks + nwarps - 1) / nwarps);
+    tail_div = 0;  // one item per warp already
+  }
   if (chunk > 65536) chunk = 65536;
+  // the last 1/WF_TAIL_DIV of each launch's blocks in short items (guided self-scheduling)
+  const int64_t chunk_s = std::max<int64_t>(64, chunk / WF_TAIL_SPLIT);
   const int nbins = kMaxBins + 1;
-  k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, chunk, bin_start, item_start);
+  k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, nl > 1 ? L[1].bin_lo : nbins, chunk, chunk_s, tail_div,
+                                 bin_start, item_start, bin_nbig);
   LAUNCHED(c);
   // stable sort of the pass's pairs by bin, then contiguous block ranges by an exclusive scan
   uint32_t* keys;
@@ -418,6 +426,8 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   A.item_start = item_start;
   A.bucket = c->bucket;
   A.chunk_blocks = chunk;
+  A.chunk_small = chunk_s;
+  A.bin_nbig = bin_nbig;
   A.out = out;
   A.exp_out = exp_out;
   CUDA_TRY(cudaMemsetAsync(scal->item_counter, 0, sizeof(scal->item_counter), s));

@@ -44,7 +44,16 @@ __device__ int g_trace_steps;
 #endif
 
 #ifndef PHMM_F32_K
-#define PHMM_F32_K 8
+#define PHMM_F32_K 8  // rows per half in the FP32 pass (8 or 4)
+#endif
+#ifndef PHMM_F32_MINB
+#define PHMM_F32_MINB 2  // CTAs (of 4 warps) per SM the FP32 kernel's register budget must allow (2: 255 regs)
+#endif
+#ifndef PHMM_F64_K
+#define PHMM_F64_K 4  // rows per half in the FP64 rescue pass (4 or 2)
+#endif
+#ifndef PHMM_F64_MINB
+#define PHMM_F64_MINB 2
 #endif
 #ifndef PHMM_XCHG_SMEM
 #define PHMM_XCHG_SMEM 0  // 1: design-A ablation build (row exchange through shared memory)
@@ -57,12 +66,22 @@ constexpr int WF_PAD = 5;
 #define PHMM_WF_WARPS 4
 #endif
 constexpr int WF_WARPS = PHMM_WF_WARPS;  // warps per CTA
+#ifndef PHMM_TAIL_DIV
+#define PHMM_TAIL_DIV 8
+#endif
+#ifndef PHMM_TAIL_SPLIT
+#define PHMM_TAIL_SPLIT 4
+#endif
+constexpr int WF_TAIL_SPLIT = PHMM_TAIL_SPLIT;  // short items are 1/WF_TAIL_SPLIT of a full-size item
+constexpr int WF_TAIL_DIV = PHMM_TAIL_DIV;  // last 1/WF_TAIL_DIV of a launch's blocks in short work items (0: none)
 constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
 constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
-constexpr int WF_KC = 2;          // 16-byte chunks per row set (FP32 K=8 and FP64 K=4 alike)
+constexpr int WF_KC32 = PHMM_F32_K / 4;  // 16-byte chunks per row set of the FP32 pass (K floats)
+constexpr int WF_KC64 = PHMM_F64_K / 2;  // ... of the FP64 pass (K doubles)
 // code byte in the haplotype code arrays = code * WF_CB; moved into bits 8..15 it is
-// code * WF_KC * 512 bytes = the stride of one code's rows in a lane's prior table
-constexpr int WF_CB = 2 * WF_KC;
+// code * WF_KC32 * 512 bytes = the stride of one code's rows in a lane's FP32 prior table
+// (the FP64 pass, which reads the same code arrays, scales it by WF_KC64 / WF_KC32)
+constexpr int WF_CB = 2 * WF_KC32;
 
 // BlkDesc.flags: bit0 last, bit1 first, bits 8-11 R row (15 = none)
 constexpr uint16_t WF_RROW_SHIFT = 8;
@@ -76,14 +95,19 @@ template <typename T> struct WfT;
 template <> struct WfT<float> {
   using V = v2f;
   static constexpr int K = PHMM_F32_K;
+  static constexpr int KC = WF_KC32;
+  static constexpr int MINB = PHMM_F32_MINB;  // CTAs per SM the register budget must allow
   static constexpr int kScaleExp = 120;
 };
 template <> struct WfT<double> {
   using V = v2d;
-  static constexpr int K = 4;
+  static constexpr int K = PHMM_F64_K;
+  static constexpr int KC = WF_KC64;
+  static constexpr int MINB = PHMM_F64_MINB;
   static constexpr int kScaleExp = 1020;
 };
-static_assert(WfT<float>::K * 4 == WF_KC * 16 && WfT<double>::K * 8 == WF_KC * 16, "chunk layout");
+static_assert(WfT<float>::K * 4 == WF_KC32 * 16 && WfT<double>::K * 8 == WF_KC64 * 16, "chunk layout");
+static_assert(WF_KC64 % WF_KC32 == 0 || WF_KC32 % WF_KC64 == 0, "code stride");
 
 __device__ __forceinline__ v2f pk(float lo, float hi) {
   v2f r;
@@ -146,7 +170,7 @@ struct alignas(16) TBlock {
   T coef[WF_NCOEF][WfT<T>::K];  // u, w, ep', mu
   T prior[5][WfT<T>::K];        // T(row, code) for code = A, C, G, T, N
 };
-static_assert(sizeof(TBlock<float>) == 9 * WF_KC * 16 && sizeof(TBlock<double>) == 9 * WF_KC * 16, "TBlock");
+static_assert(sizeof(TBlock<float>) == 9 * WF_KC32 * 16 && sizeof(TBlock<double>) == 9 * WF_KC64 * 16, "TBlock");
 
 template <typename T>
 struct WfArgs2 {
@@ -158,7 +182,9 @@ struct WfArgs2 {
   const unsigned long long* item_start;  // [nbins+1] first work item of each bin
   int bin_lo, bin_hi;                    // this launch runs the work items of bins [bin_lo, bin_hi)
   int bucket;
-  int64_t chunk_blocks;
+  int64_t chunk_blocks;                  // blocks per full-size work item
+  int64_t chunk_small;                   // blocks per short work item (the tail of each bin)
+  const unsigned long long* bin_nbig;    // [nbins] full-size items of each bin
   unsigned int* item_counter;
   T* out;
   int32_t* exp_out;  // FP32 pass: per output slot, the power of 2 the ring rescale applied
@@ -298,12 +324,13 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   constexpr int PER = 16 / sizeof(T);  // values per 16-byte chunk
   if (have) {
     const uint4* __restrict__ s4 = reinterpret_cast<const uint4*>(A.tab + d.tab_blk);
-    union { uint4 u[WF_NCOEF * WF_KC]; T v[WF_NCOEF][K]; } cw;
+    constexpr int KC = WfT<T>::KC;
+    union { uint4 u[WF_NCOEF * KC]; T v[WF_NCOEF][K]; } cw;
 #pragma unroll
-    for (int k = 0; k < WF_NCOEF * WF_KC; ++k) cw.u[k] = __ldg(s4 + k);
+    for (int k = 0; k < WF_NCOEF * KC; ++k) cw.u[k] = __ldg(s4 + k);
 #pragma unroll
-    for (int k = 0; k < 5 * WF_KC; ++k)  // prior[code][chunk]
-      sts16(tab_s + 512u * k, __ldg(s4 + WF_NCOEF * WF_KC + k));
+    for (int k = 0; k < 5 * KC; ++k)  // prior[code][chunk]
+      sts16(tab_s + 512u * k, __ldg(s4 + WF_NCOEF * KC + k));
     const int rrow = (d.flags >> WF_RROW_SHIFT) & 15;
 #pragma unroll
     for (int u = 0; u < K; ++u) {
@@ -427,7 +454,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   int outA = -1, outB = -1;
   V upM = vzero<V>(), upI = vzero<V>(), upD = vzero<V>(), dgM = vzero<V>(), dgI = vzero<V>(), dgD = vzero<V>();
   const uint32_t tabA_s = ptab_s + 16u * lane;                              // [code][chunk][lane] 16 B
-  const uint32_t tabB_s = ptab_s + 16u * (WF_NCODE * WF_KC * 32 + lane);   // half B
+  const uint32_t tabB_s = ptab_s + 16u * (WF_NCODE * WfT<T>::KC * 32 + lane);   // half B
   const int src = (lane + 31) & 31;
   const bool is0 = lane == 0, is31 = lane == 31;
   int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
@@ -456,10 +483,17 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   auto step = [&](const int r) {
     if (is31) rget<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
     // code byte r (= code*WF_CB) placed in byte 1 -> the code's rows in the table
-    const uint32_t oA = __byte_perm(wA, 0, 0x4404 + (r << 4)), oB = __byte_perm(wB, 0, 0x4404 + (r << 4));
+    // code stride of this pass's table relative to the code byte's (powers of 2)
+    constexpr int kKC = WfT<T>::KC;
+    auto cs = [](uint32_t o) -> uint32_t {
+      if constexpr (kKC == WF_KC32) return o;
+      else if constexpr (kKC > WF_KC32) return o * (uint32_t)(kKC / WF_KC32);
+      else return o / (uint32_t)(WF_KC32 / kKC);
+    };
+    const uint32_t oA = cs(__byte_perm(wA, 0, 0x4404 + (r << 4))), oB = cs(__byte_perm(wB, 0, 0x4404 + (r << 4)));
     T prA[K], prB[K];
 #pragma unroll
-    for (int ch = 0; ch < WF_KC; ++ch) {
+    for (int ch = 0; ch < WfT<T>::KC; ++ch) {
       lds16(tabA_s + oA + 512u * ch, prA + PER * ch);
       lds16(tabB_s + oB + 512u * ch, prB + PER * ch);
     }
@@ -562,7 +596,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_smem(int ring_len) {
   // prior tables, ring, and (design-A ablation only) the exchange line buffer; a multiple of
   // 16 bytes so that every warp's tables stay 16-byte aligned
-  const size_t b = (size_t)2 * WF_NCODE * WF_KC * 32 * 16 +
+  const size_t b = (size_t)2 * WF_NCODE * WfT<T>::KC * 32 * 16 +
                    (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) * ring_slot_bytes<T, kLong>();
   return (b + 15) & ~(size_t)15;
 }
@@ -572,16 +606,13 @@ cudaError_t wf_launch(bool long_rows, unsigned grid, int warps, size_t smem, cud
                       const WfArgs2<T>& args);
 
 #ifdef PHMM_DEFINE_WF
-#ifndef PHMM_F32_MINB
-#define PHMM_F32_MINB 2  // CTAs (of 4 warps) per SM the register budget must allow (255 regs)
-#endif
 template <typename T, bool kLong>
-__global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfArgs2<T> A) {
+__global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArgs2<T> A) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   const int lane = threadIdx.x & 31;
   const int wib = threadIdx.x >> 5;
-  // per warp: prior tables [2 halves][6 codes][WF_KC chunks][32 lanes] x 16 B, then the ring
-  constexpr uint32_t kTabBytes = 2 * WF_NCODE * WF_KC * 32 * 16;
+  // per warp: prior tables [2 halves][6 codes][KC chunks][32 lanes] x 16 B, then the ring
+  constexpr uint32_t kTabBytes = 2 * WF_NCODE * WfT<T>::KC * 32 * 16;
   const uint32_t per_warp = (uint32_t)wf_warp_smem<T, kLong>(A.ring_len);
   unsigned char* base = smem_raw + (size_t)wib * per_warp;
   for (uint32_t i = 4 * lane; i < per_warp; i += 128) *reinterpret_cast<uint32_t*>(base + i) = 0u;
@@ -603,8 +634,15 @@ __global__ void __launch_bounds__(WF_WARPS * 32, PHMM_F32_MINB) k_wavefront(WfAr
     const int bin = lo_;
     const int64_t b0 = (int64_t)A.bin_start[bin], b1 = (int64_t)A.bin_start[bin + 1];
     const int64_t k = (int64_t)(it - A.item_start[bin]);
-    int64_t s = b0 + k * A.chunk_blocks;
-    int64_t e = s + A.chunk_blocks;
+    const int64_t nbig = (int64_t)A.bin_nbig[bin];
+    int64_t s, e;
+    if (k < nbig) {
+      s = b0 + k * A.chunk_blocks;
+      e = s + A.chunk_blocks;
+    } else {
+      s = b0 + nbig * A.chunk_blocks + (k - nbig) * A.chunk_small;
+      e = s + A.chunk_small;
+    }
     if (e > b1) e = b1;
     auto advance = [&](int64_t x) -> int64_t {
       while (x < b1) {
