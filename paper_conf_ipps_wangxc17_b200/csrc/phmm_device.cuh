@@ -219,10 +219,11 @@ __device__ __forceinline__ unsigned long long block_scan_1024(unsigned long long
 }
 
 __global__ void __launch_bounds__(1024) k_scan_bins(const unsigned long long* __restrict__ bin_blocks, int nbins,
-                                                    int cut, int64_t chunk, int64_t chunk_s, int tail_div,
+                                                    int cut, int64_t chunk, int64_t chunk_s, int tail_div, int lpt,
                                                     unsigned long long* __restrict__ bin_start,
                                                     unsigned long long* __restrict__ item_start,
-                                                    unsigned long long* __restrict__ bin_nbig) {
+                                                    unsigned long long* __restrict__ bin_nbig,
+                                                    unsigned long long* __restrict__ launch_items) {
   __shared__ unsigned long long sh[1024];
   // pass 1: first block of every bin (serial-by-tile scan: nbins is a few thousand at most)
   unsigned long long carry = 0, tot;
@@ -236,18 +237,22 @@ __global__ void __launch_bounds__(1024) k_scan_bins(const unsigned long long* __
   if (threadIdx.x == 0) bin_start[nbins] = carry;
   __syncthreads();
   const int c = cut < 0 ? 0 : (cut > nbins ? nbins : cut);
-  const unsigned long long L0 = bin_start[c], L1 = carry - L0;  // blocks of the two launches
+  const unsigned long long B0 = bin_start[c], Ball = carry;
+  const unsigned long long L0 = B0, L1 = Ball - B0;  // blocks of the two launches
   const unsigned long long thr0 = tail_div > 0 ? L0 - L0 / tail_div : L0;
-  const unsigned long long thr1 = L0 + (tail_div > 0 ? L1 - L1 / tail_div : L1);
-  // pass 2: items per bin
+  const unsigned long long thr1 = tail_div > 0 ? L1 - L1 / tail_div : L1;
+  // pass 2: items per bin (item_start: exclusive prefix in bin order for now)
   carry = 0;
   for (int base = 0; base < nbins; base += 1024) {
     const int i = base + threadIdx.x;
     unsigned long long vi = 0;
     if (i < nbins) {
-      const unsigned long long vb = bin_blocks[i], s0 = bin_start[i];
-      const unsigned long long thr = (i < c) ? thr0 : thr1;
-      const unsigned long long big = thr <= s0 ? 0ull : (thr - s0 < vb ? thr - s0 : vb);
+      const unsigned long long vb = bin_blocks[i];
+      const bool l0 = i < c;
+      // position of the bin's first block in its launch's order (ascending or, lpt, descending bins)
+      const unsigned long long pos = lpt ? (l0 ? B0 : Ball) - bin_start[i + 1] : bin_start[i] - (l0 ? 0ull : B0);
+      const unsigned long long thr = l0 ? thr0 : thr1;
+      const unsigned long long big = thr <= pos ? 0ull : (thr - pos < vb ? thr - pos : vb);
       const unsigned long long nbig = (big == vb) ? (vb + chunk - 1) / chunk : big / chunk;
       const unsigned long long used = nbig * chunk < vb ? nbig * chunk : vb;
       vi = nbig + (vb - used + chunk_s - 1) / chunk_s;
@@ -258,6 +263,27 @@ __global__ void __launch_bounds__(1024) k_scan_bins(const unsigned long long* __
     carry += tot;
   }
   if (threadIdx.x == 0) item_start[nbins] = carry;
+  __syncthreads();
+  const unsigned long long I0 = item_start[c], Iall = carry;
+  if (threadIdx.x == 0) {
+    launch_items[0] = 0; launch_items[1] = I0; launch_items[2] = I0; launch_items[3] = Iall;
+  }
+  if (lpt) {  // descending bins inside each launch: item_start[i] = launch base + items of the bins above i
+    constexpr int kPer = (kMaxBins + 1 + 1023) / 1024;
+    unsigned long long v[kPer];
+#pragma unroll
+    for (int r = 0; r < kPer; ++r) {  // read every old value before any is overwritten
+      const int i = threadIdx.x + 1024 * r;
+      const unsigned long long nxt = (i + 1 < nbins) ? item_start[i + 1] : Iall;
+      v[r] = (i < c) ? I0 - nxt : I0 + (Iall - nxt);
+    }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < kPer; ++r) {
+      const int i = threadIdx.x + 1024 * r;
+      if (i < nbins) item_start[i] = v[r];
+    }
+  }
 }
 
 }  // namespace phmm

@@ -215,8 +215,8 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   const int nb1 = kMaxBins + 2;
-  unsigned long long* bins;  // [blocks | pairs | nbig | start | item_start], nb1 each
-  ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
+  unsigned long long* bins;  // [blocks | pairs | nbig | start | item_start | launch items], nb1 each
+  ST_TRY(ws(c, B_BINS, (size_t)6 * nb1, &bins));
   int32_t *pair_bin, *pair_nb;
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
   ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
@@ -313,9 +313,9 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   const int nb1 = kMaxBins + 2;
   unsigned long long* bins;
-  ST_TRY(ws(c, B_BINS, (size_t)5 * nb1, &bins));
+  ST_TRY(ws(c, B_BINS, (size_t)6 * nb1, &bins));
   unsigned long long *bin_blocks = bins, *bin_nbig = bins + 2 * nb1, *bin_start = bins + 3 * nb1,
-                     *item_start = bins + 4 * nb1;
+                     *item_start = bins + 4 * nb1, *launch_items = bins + 5 * nb1;
   int32_t *pair_bin, *pair_nb, *item_read = nullptr, *pair_item = nullptr;
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
   ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
@@ -388,7 +388,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   const int64_t chunk_s = std::max<int64_t>(64, chunk / WF_TAIL_SPLIT);
   const int nbins = kMaxBins + 1;
   k_scan_bins<<<1, 1024, 0, s>>>(bin_blocks, nbins, nl > 1 ? L[1].bin_lo : nbins, chunk, chunk_s, tail_div,
-                                 bin_start, item_start, bin_nbig);
+                                 WF_LPT, bin_start, item_start, bin_nbig, launch_items);
   LAUNCHED(c);
   // stable sort of the pass's pairs by bin, then contiguous block ranges by an exclusive scan
   uint32_t* keys;
@@ -428,6 +428,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   A.chunk_blocks = chunk;
   A.chunk_small = chunk_s;
   A.bin_nbig = bin_nbig;
+  A.lpt = WF_LPT;
   A.out = out;
   A.exp_out = exp_out;
   CUDA_TRY(cudaMemsetAsync(scal->item_counter, 0, sizeof(scal->item_counter), s));
@@ -437,6 +438,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     A.bin_hi = L[i].bin_hi;
     A.ring_len = L[i].ring_len;
     A.item_counter = &scal->item_counter[i];
+    A.launch_items = launch_items + 2 * i;
     const size_t smem = (i == 1 ? wf_warp_smem<T, true>(L[i].ring_len) : wf_warp_smem<T>(L[i].ring_len)) * L[i].warps;
     CUDA_TRY(wf_launch<T>(i == 1, (unsigned)(c->nsm * L[i].bps), L[i].warps, smem, s, A));
     ++c->launches;

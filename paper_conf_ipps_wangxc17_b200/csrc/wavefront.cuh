@@ -70,9 +70,13 @@ constexpr int WF_WARPS = PHMM_WF_WARPS;  // warps per CTA
 #define PHMM_TAIL_DIV 8
 #endif
 #ifndef PHMM_TAIL_SPLIT
-#define PHMM_TAIL_SPLIT 4
+#define PHMM_TAIL_SPLIT 8
 #endif
 constexpr int WF_TAIL_SPLIT = PHMM_TAIL_SPLIT;  // short items are 1/WF_TAIL_SPLIT of a full-size item
+#ifndef PHMM_LPT
+#define PHMM_LPT 1
+#endif
+constexpr int WF_LPT = PHMM_LPT;  // 1: longest-row bins first inside a launch
 constexpr int WF_TAIL_DIV = PHMM_TAIL_DIV;  // last 1/WF_TAIL_DIV of a launch's blocks in short work items (0: none)
 constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
 constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
@@ -185,6 +189,8 @@ struct WfArgs2 {
   int64_t chunk_blocks;                  // blocks per full-size work item
   int64_t chunk_small;                   // blocks per short work item (the tail of each bin)
   const unsigned long long* bin_nbig;    // [nbins] full-size items of each bin
+  const unsigned long long* launch_items;  // [2]: this launch's work items are [launch_items[0], launch_items[1])
+  int lpt;                               // 1: bins in descending order inside a launch (longest rows first)
   unsigned int* item_counter;
   T* out;
   int32_t* exp_out;  // FP32 pass: per output slot, the power of 2 the ring rescale applied
@@ -620,16 +626,23 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
   const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
   const uint32_t xbuf_s = ring_s + (uint32_t)A.ring_len * ring_slot_bytes<T, kLong>();  // design A only
   // work item it of the launch: chunk k of bin b (binary search in item_start)
-  const unsigned long long it0 = A.item_start[A.bin_lo], it1 = A.item_start[A.bin_hi];
+  const unsigned long long it0 = A.launch_items[0], it1 = A.launch_items[1];
   while (true) {
     unsigned long long it = 0;
     if (lane == 0) it = it0 + atomicAdd(A.item_counter, 1u);
     it = __shfl_sync(0xffffffffu, it, 0);
     if (it >= it1) break;
     int lo_ = A.bin_lo, hi_ = A.bin_hi - 1;
-    while (lo_ < hi_) {
-      const int mid = (lo_ + hi_ + 1) >> 1;
-      if (A.item_start[mid] <= it) lo_ = mid; else hi_ = mid - 1;
+    if (A.lpt) {  // item_start descending in the bin index: the smallest bin with item_start <= it
+      while (lo_ < hi_) {
+        const int mid = (lo_ + hi_) >> 1;
+        if (A.item_start[mid] <= it) hi_ = mid; else lo_ = mid + 1;
+      }
+    } else {      // ascending: the largest bin with item_start <= it
+      while (lo_ < hi_) {
+        const int mid = (lo_ + hi_ + 1) >> 1;
+        if (A.item_start[mid] <= it) lo_ = mid; else hi_ = mid - 1;
+      }
     }
     const int bin = lo_;
     const int64_t b0 = (int64_t)A.bin_start[bin], b1 = (int64_t)A.bin_start[bin + 1];
