@@ -141,18 +141,19 @@ __device__ __forceinline__ double start_mass_correction(const int32_t* __restric
   return log10((double)ncols_of(n, bucket) / (double)n);
 }
 
+// rescue_list gets p + rbase (a chunk of a larger batch lists its pairs by their batch index).
 __global__ void k_finalize_fp32(const float* __restrict__ s32, const int32_t* __restrict__ exp32, int64_t n_pairs,
                                 const int32_t* __restrict__ pairs,
                                 const int64_t* __restrict__ hoff, int bucket, double* __restrict__ out,
                                 uint8_t* __restrict__ status, int32_t* __restrict__ rescue_list,
-                                int64_t* __restrict__ n_rescue, int write_status) {
+                                int64_t* __restrict__ n_rescue, int write_status, int64_t rbase) {
   const double off = 120.0 * 0.30102999566398119521;
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n_pairs; p += (int64_t)gridDim.x * blockDim.x) {
     const float s = s32[p];
     // NaN-safe: also catches s < 1e-28; exp32 < 0 by 2^23: the ring rescale saturated
     if (!(s >= 1e-28f) || !isfinite(s) || exp32[p] < -(1 << 23)) {
       const unsigned long long k = atomicAdd(reinterpret_cast<unsigned long long*>(n_rescue), 1ull);
-      rescue_list[k] = (int32_t)p;
+      rescue_list[k] = (int32_t)(p + rbase);
     } else {
       // the ring rescale multiplied the pair's later rows by 2^exp32[p]
       out[p] = log10((double)s) - (off + (double)exp32[p] * 0.30102999566398119521) +
@@ -183,6 +184,24 @@ __global__ void k_finalize_fp64(const double* __restrict__ s64, const int32_t* _
     if (st == 2) atomicAdd(n_underflow, 1ull);
     out[p] = v;
     if (write_status) status[p] = st;
+  }
+}
+
+// One chunk of a host batch (phmm_compute_batch's copy/compute pipeline): the chunk's
+// offsets relative to its first read / haplotype and its pairs relative to both, so that the
+// chunk is an ordinary batch over [rlo, rlo + nr) reads and [hlo, hlo + nh) haplotypes.
+__global__ void k_rebase_chunk(const int64_t* __restrict__ roff, int64_t rlo, int64_t nr, int64_t* __restrict__ roff_c,
+                               const int64_t* __restrict__ hoff, int64_t hlo, int64_t nh, int64_t* __restrict__ hoff_c,
+                               const int32_t* __restrict__ pairs, int64_t p0, int64_t np, int32_t* __restrict__ pairs_c) {
+  const int64_t n = (nr + 1 > nh + 1 ? nr + 1 : nh + 1) > np ? (nr + 1 > nh + 1 ? nr + 1 : nh + 1) : np;
+  const int64_t r0 = roff[rlo], h0 = hoff[hlo];
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    if (i <= nr) roff_c[i] = roff[rlo + i] - r0;
+    if (i <= nh) hoff_c[i] = hoff[hlo + i] - h0;
+    if (i < np) {
+      pairs_c[2 * i] = pairs[2 * (p0 + i)] - (int32_t)rlo;
+      pairs_c[2 * i + 1] = pairs[2 * (p0 + i) + 1] - (int32_t)hlo;
+    }
   }
 }
 

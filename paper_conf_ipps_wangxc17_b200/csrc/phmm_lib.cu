@@ -34,7 +34,9 @@ enum BufId {
   B_SW_REF, B_SW_ROFF, B_SW_ALT, B_SW_AOFF, B_SW_TASKS, B_SW_RES, B_SW_OPS,  // SW host-variant staging
   B_SW_BTSZ, B_SW_BTOFF, B_SW_OPCAP, B_SW_OPOFF, B_SW_BT, B_SW_KEYS, B_SW_VALS, B_SW_OPTMP, B_SW_NOPS,
   B_SW_NOPOFF,
-  B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_EXP32, B_COUNT
+  B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_EXP32, B_GRING,
+  B_CH_ROFF, B_CH_HOFF, B_CH_PAIRS, B_CH_CNT,  // host-variant pipeline: one chunk's rebased offsets / pairs
+  B_COUNT
 };
 
 struct Buf {
@@ -56,6 +58,10 @@ struct Scalars {
 
 constexpr int kEvents = 10;
 constexpr int kThreads = 256;
+// host variant (phmm_compute_batch): the pairs are cut into up to kMaxChunks chunks of at least
+// kChunkMinPairs; chunk k+1's inputs are copied on a second stream while chunk k computes
+constexpr int kMaxChunks = 4;
+constexpr int64_t kChunkMinPairs = 65536;
 
 }  // namespace
 
@@ -73,6 +79,9 @@ struct phmm_ctx {
   int64_t* host_sizes = nullptr;  // pinned, 2 values
   int64_t sw_ops_cap = 0;         // last SW call: sum over tasks of M + N
   cudaEvent_t ev[kEvents] = {};
+  cudaStream_t copy_stream = nullptr;     // host variant: H2D of the next chunk
+  cudaEvent_t cev[kMaxChunks + 1] = {};   // chunk k's inputs on the device / the call's start
+  int max_chunks = 1;                     // PHMM_CHUNKS=n (<= kMaxChunks) turns the pipeline on (measured slower)
   phmm_stats st{};
   int launches = 0;
 };
@@ -361,7 +370,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   int nl = 0;
   L[nl++] = Launch{0, std::min(bin_cut, kMaxBins + 1), WF_WARPS, std::min(p_max + 4, ring_full), bps_full};
   if (bin_cut <= kMaxBins) {
-    Launch lb{bin_cut, kMaxBins + 1, 0, p_max + 4, 0};
+    Launch lb{bin_cut, kMaxBins + 1, 0, p_max + 8, 0};  // global ring: prefetch reads up to slot P + 4
     int best = 0;
     for (int w = WF_WARPS; w >= 1; w >>= 1) {
       const size_t sm = wf_warp_smem<T, true>(lb.ring_len) * w;
@@ -431,6 +440,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   A.lpt = WF_LPT;
   A.out = out;
   A.exp_out = exp_out;
+  A.gring = nullptr;
   CUDA_TRY(cudaMemsetAsync(scal->item_counter, 0, sizeof(scal->item_counter), s));
   if (timed) ev_record(c, EV_WF0);
   for (int i = 0; i < nl; ++i) {
@@ -440,10 +450,72 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     A.item_counter = &scal->item_counter[i];
     A.launch_items = launch_items + 2 * i;
     const size_t smem = (i == 1 ? wf_warp_smem<T, true>(L[i].ring_len) : wf_warp_smem<T>(L[i].ring_len)) * L[i].warps;
+    if (i == 1 && ring_global<true>()) {  // the long launch's rings: one per resident warp, zeroed
+      const size_t gb = (size_t)c->nsm * L[i].bps * L[i].warps * (size_t)L[i].ring_len * ring_slot_bytes<T, true>();
+      ST_TRY(ws(c, B_GRING, gb, &A.gring));
+      CUDA_TRY(cudaMemsetAsync(A.gring, 0, gb, s));
+    }
     CUDA_TRY(wf_launch<T>(i == 1, (unsigned)(c->nsm * L[i].bps), L[i].warps, smem, s, A));
     ++c->launches;
   }
   if (timed) ev_record(c, EV_WF1);
+  return PHMM_OK;
+}
+
+// The FP32 pass over a batch (all its pairs): per-read tables, binning, k_wavefront<float>,
+// k_finalize_fp32 into dev_out / dev_status; pairs below the FP32 range are appended to rlist
+// (as pair index + rbase) and counted in *n_rescue. Returns the haplotype code regions it built.
+phmm_status fp32_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status, int32_t* rlist,
+                      int64_t rbase, int64_t* n_rescue, PassInfo* pi, uint8_t** hc, int64_t* total_hc, bool timed) {
+  cudaStream_t s = c->stream;
+  int64_t total_tab = 0;
+  ST_TRY((pass_prepare<float>(c, d, nullptr, d.n_pairs, pi, &total_tab, total_hc)));
+  ST_TRY(build_hap_codes(c, d, *total_hc, pi->max_ncols, hc));
+  float* out32;
+  ST_TRY(ws(c, B_OUT32, (size_t)d.n_pairs, &out32));
+  int32_t* exp32;  // powers of 2 applied by the ring rescale of long pairs
+  ST_TRY(ws(c, B_EXP32, (size_t)d.n_pairs, &exp32));
+  CUDA_TRY(cudaMemsetAsync(exp32, 0, sizeof(int32_t) * (size_t)d.n_pairs, s));
+  if (timed) ev_record(c, EV_PREP);
+  ST_TRY(pass_run<float>(c, d, nullptr, d.n_pairs, *pi, total_tab, *hc, *total_hc, out32, timed, exp32));
+  k_finalize_fp32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out32, exp32, d.n_pairs, d.pairs, d.hoff, c->bucket,
+                                                                dev_out, dev_status, rlist, n_rescue,
+                                                                dev_status != nullptr, rbase);
+  LAUNCHED(c);
+  c->st.cells += (int64_t)pi->cells;
+  c->st.padded_cells += (int64_t)pi->padded_cells;
+  return PHMM_OK;
+}
+
+// FP64 rescue of the nr listed pairs of batch d on the same kernel design. hc: the haplotype
+// code regions of d (nullptr: build them here).
+phmm_status rescue_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status, const int32_t* rlist,
+                        int64_t nr, const uint8_t* hc, int64_t total_hc, bool timed) {
+  cudaStream_t s = c->stream;
+  Scalars* scal;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  PassInfo pr;
+  int64_t tab_r = 0;
+  if (hc) {
+    ST_TRY((pass_prepare<double>(c, d, rlist, nr, &pr, &tab_r)));
+  } else {
+    uint8_t* hc_b;
+    ST_TRY((pass_prepare<double>(c, d, rlist, nr, &pr, &tab_r, &total_hc)));
+    ST_TRY(build_hap_codes(c, d, total_hc, pr.max_ncols, &hc_b));
+    hc = hc_b;
+  }
+  double* out64;
+  ST_TRY(ws(c, B_OUT64, (size_t)nr, &out64));
+  ST_TRY((pass_run<double>(c, d, rlist, nr, pr, tab_r, hc, total_hc, out64, false)));
+  CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
+  k_finalize_fp64<<<grid_for(c, nr), kThreads, 0, s>>>(out64, rlist, nullptr, nr, d.pairs, d.hoff, c->bucket, dev_out,
+                                                       dev_status, dev_status != nullptr, 1, &scal->n_underflow);
+  LAUNCHED(c);
+  c->st.padded_cells += (int64_t)pr.padded_cells;
+  if (timed) ev_record(c, EV_RESC1);
+  CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
   return PHMM_OK;
 }
 
@@ -476,52 +548,21 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
+    c->st.cells = (int64_t)pi.cells;
+    c->st.padded_cells += (int64_t)pi.padded_cells;
   } else {
-    ST_TRY((pass_prepare<float>(c, d, nullptr, d.n_pairs, &pi, &total_tab, &total_hc)));
-    ST_TRY(build_hap_codes(c, d, total_hc, pi.max_ncols, &hc));
-    float* out32;
-    ST_TRY(ws(c, B_OUT32, (size_t)d.n_pairs, &out32));
-    int32_t* exp32;  // powers of 2 applied by the ring rescale of long pairs
-    ST_TRY(ws(c, B_EXP32, (size_t)d.n_pairs, &exp32));
-    CUDA_TRY(cudaMemsetAsync(exp32, 0, sizeof(int32_t) * (size_t)d.n_pairs, s));
-    ev_record(c, EV_PREP);
-    ST_TRY(pass_run<float>(c, d, nullptr, d.n_pairs, pi, total_tab, hc, total_hc, out32, true, exp32));
     int32_t* rlist;
     ST_TRY(ws(c, B_RLIST, (size_t)d.n_pairs, &rlist));
     CUDA_TRY(cudaMemsetAsync(&scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
-    k_finalize_fp32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out32, exp32, d.n_pairs, d.pairs, d.hoff, c->bucket,
-                                                                  dev_out, dev_status, rlist,
-                                                                  &scal->n_rescue, dev_status != nullptr);
-    LAUNCHED(c);
+    ST_TRY(fp32_pass(c, d, dev_out, dev_status, rlist, 0, &scal->n_rescue, &pi, &hc, &total_hc, true));
     ev_record(c, EV_RESC0);
     CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     const int64_t nr = c->host_scal->n_rescue;
     c->st.n_rescued = nr;
-    if (nr > 0) {
-      // FP64 rescue of the listed pairs on the same kernel design (same code regions)
-      PassInfo pr;
-      int64_t tab_r = 0;
-      ST_TRY((pass_prepare<double>(c, d, rlist, nr, &pr, &tab_r)));
-      double* out64;
-      ST_TRY(ws(c, B_OUT64, (size_t)nr, &out64));
-      ST_TRY((pass_run<double>(c, d, rlist, nr, pr, tab_r, hc, total_hc, out64, false)));
-      CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
-      k_finalize_fp64<<<grid_for(c, nr), kThreads, 0, s>>>(out64, rlist, nullptr, nr, d.pairs, d.hoff, c->bucket,
-                                                           dev_out, dev_status,
-                                                           dev_status != nullptr, 1, &scal->n_underflow);
-      LAUNCHED(c);
-      c->st.padded_cells += (int64_t)pr.padded_cells;
-    }
-    ev_record(c, EV_RESC1);
-    if (nr > 0) {
-      CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
-      CUDA_TRY(cudaStreamSynchronize(s));
-      c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
-    }
+    if (nr > 0) ST_TRY(rescue_pass(c, d, dev_out, dev_status, rlist, nr, hc, total_hc, true));
+    else ev_record(c, EV_RESC1);
   }
-  c->st.cells = (int64_t)pi.cells;
-  c->st.padded_cells += (int64_t)pi.padded_cells;
   return PHMM_OK;
 }
 
@@ -681,6 +722,133 @@ void finish_stats(phmm_ctx* c) {
   }
 }
 
+// ------------------------------------------------------------ host variant: copy/compute pipeline
+// phmm_compute_batch cuts the pairs into chunks; while chunk k computes on the context stream,
+// chunk k+1's inputs travel on the copy stream. Every read / haplotype is copied once: chunk k
+// copies the reads [rc0, rc1) not copied before (rc1 = one past the largest read index seen so
+// far, the last chunk takes the rest), and computes as an ordinary batch over the reads
+// [rlo, rhi) (rlo <= its smallest read index, and <= rc0 so that the chunks' read ranges
+// together cover -- and validate -- every read); same for haplotypes. The FP64 rescue runs once,
+// over the whole batch, after the last chunk; results travel back once, at the end, so an input
+// error found in a later chunk still leaves the caller's outputs untouched.
+struct ChunkPlan {
+  int64_t p0, p1, rlo, rhi, rc0, rc1, hlo, hhi, hc0, hc1;
+};
+
+phmm_status plan_chunk(const phmm_batch* b, int64_t p0, int64_t p1, int64_t rdone, int64_t hdone, bool last,
+                       ChunkPlan* cp) {
+  int64_t rmin = INT64_MAX, rmax = -1, hmin = INT64_MAX, hmax = -1;
+  const int32_t* pr = b->pairs;
+  for (int64_t p = p0; p < p1; ++p) {
+    const int64_t r = pr[2 * p], h = pr[2 * p + 1];
+    rmin = r < rmin ? r : rmin;
+    rmax = r > rmax ? r : rmax;
+    hmin = h < hmin ? h : hmin;
+    hmax = h > hmax ? h : hmax;
+  }
+  if (rmin < 0 || rmax >= b->n_reads || hmin < 0 || hmax >= b->n_haps) return PHMM_E_INDEX;
+  cp->p0 = p0;
+  cp->p1 = p1;
+  cp->rc0 = rdone;
+  cp->rc1 = last ? b->n_reads : std::max(rdone, rmax + 1);
+  cp->rlo = std::min(rmin, rdone);
+  cp->rhi = cp->rc1;
+  cp->hc0 = hdone;
+  cp->hc1 = last ? b->n_haps : std::max(hdone, hmax + 1);
+  cp->hlo = std::min(hmin, hdone);
+  cp->hhi = cp->hc1;
+  // the host offsets at the chunk's boundaries address the device copies: they must be ordered
+  // and in range (the device validates every offset inside the chunk's range)
+  auto ok = [](const int64_t* off, int64_t a, int64_t z, int64_t total) {
+    return off[a] >= 0 && off[a] <= off[z] && off[z] <= total;
+  };
+  if (!ok(b->read_offsets, cp->rlo, cp->rhi, b->total_read_bases) ||
+      !ok(b->read_offsets, cp->rc0, cp->rc1, b->total_read_bases) ||
+      !ok(b->hap_offsets, cp->hlo, cp->hhi, b->total_hap_bases) ||
+      !ok(b->hap_offsets, cp->hc0, cp->hc1, b->total_hap_bases))
+    return PHMM_E_INVALID_ARG;
+  return PHMM_OK;
+}
+
+phmm_status compute_host_chunked(phmm_ctx* c, const phmm_batch* b, int nchunks, uint8_t* rb, uint8_t* q, uint8_t* qi,
+                                 uint8_t* qd, uint8_t* qg, uint8_t* hap, int64_t* roff, int64_t* hoff, int32_t* pairs,
+                                 double* out, uint8_t* status) {
+  cudaStream_t s = c->stream, cs = c->copy_stream;
+  c->st = phmm_stats{};
+  c->st.n_pairs = b->n_pairs;
+  const int64_t np_max = (b->n_pairs + nchunks - 1) / nchunks;
+  int64_t *roff_c, *hoff_c, *cnt;
+  int32_t *pairs_c, *rlist;
+  ST_TRY(ws(c, B_CH_ROFF, (size_t)b->n_reads + 1, &roff_c));
+  ST_TRY(ws(c, B_CH_HOFF, (size_t)b->n_haps + 1, &hoff_c));
+  ST_TRY(ws(c, B_CH_PAIRS, (size_t)2 * np_max, &pairs_c));
+  ST_TRY(ws(c, B_CH_CNT, 2, &cnt));
+  ST_TRY(ws(c, B_RLIST, (size_t)b->n_pairs, &rlist));
+  const int64_t* ro = b->read_offsets;
+  const int64_t* ho = b->hap_offsets;
+  auto copy_chunk = [&](const ChunkPlan& P, int k) -> phmm_status {
+    if (k == 0) {  // all offsets with the first chunk (the rebase and the rescue read them)
+      CUDA_TRY(cudaMemcpyAsync(roff, ro, sizeof(int64_t) * (b->n_reads + 1), cudaMemcpyHostToDevice, cs));
+      CUDA_TRY(cudaMemcpyAsync(hoff, ho, sizeof(int64_t) * (b->n_haps + 1), cudaMemcpyHostToDevice, cs));
+    }
+    const int64_t a0 = ro[P.rc0], a1 = ro[P.rc1];
+    if (a1 > a0) {
+      const uint8_t* src[5] = {b->read_bases, b->base_quals, b->ins_quals, b->del_quals, b->gcp_quals};
+      uint8_t* dst[5] = {rb, q, qi, qd, qg};
+      for (int i = 0; i < 5; ++i)
+        CUDA_TRY(cudaMemcpyAsync(dst[i] + a0, src[i] + a0, (size_t)(a1 - a0), cudaMemcpyHostToDevice, cs));
+    }
+    const int64_t h0 = ho[P.hc0], h1 = ho[P.hc1];
+    if (h1 > h0) CUDA_TRY(cudaMemcpyAsync(hap + h0, b->hap_bases + h0, (size_t)(h1 - h0), cudaMemcpyHostToDevice, cs));
+    CUDA_TRY(cudaMemcpyAsync(pairs + 2 * P.p0, b->pairs + 2 * P.p0, sizeof(int32_t) * 2 * (P.p1 - P.p0),
+                             cudaMemcpyHostToDevice, cs));
+    CUDA_TRY(cudaEventRecord(c->cev[k], cs));
+    return PHMM_OK;
+  };
+  ChunkPlan plan[kMaxChunks];
+  auto bound = [&](int k) { return b->n_pairs * k / nchunks; };
+  ST_TRY(plan_chunk(b, bound(0), bound(1), 0, 0, nchunks == 1, &plan[0]));
+  // the copies start after whatever the caller queued on the context stream
+  CUDA_TRY(cudaEventRecord(c->cev[kMaxChunks], s));
+  CUDA_TRY(cudaStreamWaitEvent(cs, c->cev[kMaxChunks], 0));
+  ev_record(c, EV_START);
+  ST_TRY(copy_chunk(plan[0], 0));
+  CUDA_TRY(cudaMemsetAsync(cnt, 0, 2 * sizeof(int64_t), s));
+  for (int k = 0; k < nchunks; ++k) {
+    if (k + 1 < nchunks) {
+      ST_TRY(plan_chunk(b, bound(k + 1), bound(k + 2), plan[k].rc1, plan[k].hc1, k + 2 == nchunks, &plan[k + 1]));
+      ST_TRY(copy_chunk(plan[k + 1], k + 1));
+    }
+    const ChunkPlan& P = plan[k];
+    CUDA_TRY(cudaStreamWaitEvent(s, c->cev[k], 0));
+    const int64_t nr = P.rhi - P.rlo, nh = P.hhi - P.hlo, np = P.p1 - P.p0;
+    k_rebase_chunk<<<grid_for(c, std::max(std::max(nr, nh) + 1, np)), kThreads, 0, s>>>(
+        roff, P.rlo, nr, roff_c, hoff, P.hlo, nh, hoff_c, pairs, P.p0, np, pairs_c);
+    LAUNCHED(c);
+    const int64_t a0 = ro[P.rlo], h0 = ho[P.hlo];
+    DevBatch dk{rb + a0, q + a0, qi + a0, qd + a0, qg + a0, hap + h0, roff_c, hoff_c, pairs_c,
+                nr, nh, np, ro[P.rhi] - a0, ho[P.hhi] - h0};
+    ST_TRY(run_validate(c, dk));
+    PassInfo pi;
+    uint8_t* hc = nullptr;
+    int64_t total_hc = 0;
+    ST_TRY(fp32_pass(c, dk, out + P.p0, status ? status + P.p0 : nullptr, rlist, P.p0, cnt, &pi, &hc, &total_hc,
+                     false));
+  }
+  int64_t* hcnt = c->host_sizes;
+  CUDA_TRY(cudaMemcpyAsync(hcnt, cnt, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  const int64_t nres = hcnt[0];
+  c->st.n_rescued = nres;
+  if (nres > 0) {  // the FP64 rescue over the whole batch (its own haplotype code regions)
+    DevBatch dg{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs,
+                b->total_read_bases, b->total_hap_bases};
+    ST_TRY(rescue_pass(c, dg, out, status, rlist, nres, nullptr, 0, false));
+  }
+  ev_record(c, EV_D2H);
+  return PHMM_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -755,6 +923,13 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
   }
   for (int i = 0; i < kEvents; ++i)
     if (cudaEventCreate(&c->ev[i]) != cudaSuccess) return fail(PHMM_E_CUDA);
+  if (cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking) != cudaSuccess) {
+    c->copy_stream = nullptr;
+    return fail(PHMM_E_CUDA);
+  }
+  for (int i = 0; i <= kMaxChunks; ++i)
+    if (cudaEventCreateWithFlags(&c->cev[i], cudaEventDisableTiming) != cudaSuccess) return fail(PHMM_E_CUDA);
+  if (const char* e = std::getenv("PHMM_CHUNKS")) c->max_chunks = std::max(1, std::min(kMaxChunks, std::atoi(e)));
   *out = c;
   return PHMM_OK;
 }
@@ -767,6 +942,10 @@ void phmm_destroy(phmm_ctx* c) {
     if (c->buf[i].p) cudaFree(c->buf[i].p);
   for (int i = 0; i < kEvents; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  if (c->copy_stream) cudaStreamSynchronize(c->copy_stream);
+  for (int i = 0; i <= kMaxChunks; ++i)
+    if (c->cev[i]) cudaEventDestroy(c->cev[i]);
+  if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
   if (c->host_scal) cudaFreeHost(c->host_scal);
   if (c->host_sizes) cudaFreeHost(c->host_sizes);
   if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
@@ -845,6 +1024,26 @@ phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log
   ST_TRY(ws(c, B_PAIRS, (size_t)b->n_pairs * 2, &pairs));
   ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
   if (out_status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
+  int nchunks = (int)std::min<int64_t>(c->max_chunks, b->n_pairs / kChunkMinPairs);
+  if (c->prec != PHMM_PREC_FP32_RESCUE) nchunks = 1;
+  if (nchunks > 1) {
+    phmm_status st = compute_host_chunked(c, b, nchunks, rb, q, qi, qd, qg, hap, roff, hoff, pairs, out, status);
+    if (st != PHMM_OK) {
+      cudaStreamSynchronize(c->copy_stream);
+      cudaStreamSynchronize(s);
+      cudaGetLastError();
+      return st;
+    }
+    CUDA_TRY(cudaMemcpyAsync(out_log10, out, sizeof(double) * b->n_pairs, cudaMemcpyDeviceToHost, s));
+    if (out_status) CUDA_TRY(cudaMemcpyAsync(out_status, status, b->n_pairs, cudaMemcpyDeviceToHost, s));
+    ev_record(c, EV_END);
+    CUDA_TRY(cudaStreamSynchronize(s));
+    c->st.kernel_launches = c->launches;
+    c->st.ms_total = ev_ms(c, EV_START, EV_END);
+    c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
+    c->st.ms_h2d = c->st.ms_prep = c->st.ms_wavefront = c->st.ms_rescue = c->st.ms_finalize = -1.f;  // overlapped
+    return PHMM_OK;
+  }
   ev_record(c, EV_START);
   if (nr) {
     CUDA_TRY(cudaMemcpyAsync(rb, b->read_bases, nr, cudaMemcpyHostToDevice, s));
