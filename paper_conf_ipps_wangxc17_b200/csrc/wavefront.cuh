@@ -77,6 +77,9 @@ constexpr int WF_TAIL_SPLIT = PHMM_TAIL_SPLIT;  // short items are 1/WF_TAIL_SPL
 #define PHMM_LPT 1
 #endif
 constexpr int WF_LPT = PHMM_LPT;  // 1: longest-row bins first inside a launch
+#ifndef PHMM_DESC_SMEM
+#define PHMM_DESC_SMEM 0  // 1: next-pass block descriptors travel by cp.async into shared memory
+#endif
 #ifndef PHMM_CONCAT
 #define PHMM_CONCAT 0
 #endif
@@ -331,6 +334,9 @@ __device__ __forceinline__ void lds16(uint32_t a, float* v) {
 __device__ __forceinline__ void lds16(uint32_t a, double* v) {
   asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v[0]), "=d"(v[1]) : "r"(a) : "memory");
 }
+__device__ __forceinline__ void cp_async16(uint32_t a, const void* g) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(a), "l"(g) : "memory");
+}
 __device__ __forceinline__ void sts16(uint32_t a, const uint4 v) {
   asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" :: "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
                : "memory");
@@ -533,7 +539,8 @@ __device__ __forceinline__ unsigned long long wf_claim(const WfArgs2<T>& A, int 
 // kLong: the launch of the long-row bins (the only one with the ring rescale compiled in).
 template <typename T, bool kLong>
 __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s,
-                                                        uint64_t ring_g, uint32_t xbuf_s, uint32_t seg_s, int lane,
+                                                        uint64_t ring_g, uint32_t xbuf_s, uint32_t seg_s,
+                                                        uint32_t desc_s, int lane,
                                                         int64_t s, int nblk, int bin, bool trace = false) {
   const int ncols = bin * A.bucket;
   // segments of the concatenated stream, kept in shared memory (warp-uniform, read at switch
@@ -586,11 +593,35 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
   // global ring: lane 31 loads each slot 4 steps before its use (step r of a group loads the
   // slot of step r of the next group into rq*[r])
   T rqM[4] = {0, 0, 0, 0}, rqI[4] = {0, 0, 0, 0}, rqD[4] = {0, 0, 0, 0};
+#if PHMM_DESC_SMEM
+  // descriptors of the lane's next blocks, copied one pass ahead by cp.async into a per-lane
+  // shared-memory slot (no registers held across the hot loop)
+  const uint32_t dnA_s = desc_s + 32u * lane, dnB_s = dnA_s + 16u;
+  {
+    const uint4 none = make_uint4(0u, 0u, 0xffffffffu, 1u);  // tab 0, hap 0, out -1, n 1, flags 0
+    __syncwarp();
+    sts16(dnA_s, none);
+    sts16(dnB_s, none);
+    if (2 * lane < nblk) cp_async16(dnA_s, A.blk + s + 2 * lane);
+    if (2 * lane + 1 < nblk) cp_async16(dnB_s, A.blk + s + 2 * lane + 1);
+  }
+  auto ld_desc = [](uint32_t a) {
+    asm volatile("cp.async.wait_all;" ::: "memory");
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a)
+                 : "memory");
+    BlkDesc d;
+    d.tab_blk = v.x; d.hap_off = v.y; d.out_idx = (int32_t)v.z; d.n = (uint16_t)(v.w & 0xffffu);
+    d.flags = (uint16_t)(v.w >> 16);
+    return d;
+  };
+#else
   BlkDesc dnA, dnB;  // descriptors of the lane's next blocks (loaded one pass ahead)
   dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.n = 1; dnA.flags = 0;
   dnB = dnA;
   if (2 * lane < nblk) dnA = A.blk[s + 2 * lane];
   if (2 * lane + 1 < nblk) dnB = A.blk[s + 2 * lane + 1];
+#endif
   // append the next work item when the stream would end within this pass or the next (its
   // blocks then fill the passes whose descriptors are prefetched from here on)
   auto try_append = [&](int q) {
@@ -711,6 +742,9 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
         if constexpr (rescale) {
           // lane 0's block of this pass continues the pair of virtual lane 63's last block?
           // (rows shorter than WF_RESCALE_COLS have no complete ring row at the pass start)
+#if PHMM_DESC_SMEM
+          const BlkDesc dnA = ld_desc(dnA_s);
+#endif
           const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && ncols >= WF_RESCALE_COLS;
           wf_ring_rescale<T, ring_packed<T, kLong>(), kG>(kG ? ring_g : (uint64_t)ring_s, ncols, lane, cont,
                                                           A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
@@ -727,7 +761,11 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
       if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
         const int bA = q * 64 + 2 * lane, bB = bA + 1;
         const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
+#if PHMM_DESC_SMEM
+        const BlkDesc dA = ld_desc(dnA_s), dB = ld_desc(dnB_s);  // copied one pass ago (pass 0: before the loop)
+#else
         const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
+#endif
         if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S row: the last-row M+I sum (L20@2262)
         if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
         pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
@@ -736,8 +774,13 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
         wB_nx = __ldg(pB); wB_nx2 = __ldg(pB + 1); pB += 2;
         // prefetch the next pass's descriptors after this pass's loads are issued (a load
         // issued before the consumers of the previous prefetch would share its scoreboard)
+#if PHMM_DESC_SMEM
+        if (bA + 64 < nblk) cp_async16(dnA_s, A.blk + phys(bA + 64));
+        if (bB + 64 < nblk) cp_async16(dnB_s, A.blk + phys(bB + 64));
+#else
         if (bA + 64 < nblk) dnA = A.blk[phys(bA + 64)];
         if (bB + 64 < nblk) dnB = A.blk[phys(bB + 64)];
+#endif
         if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
           T a, bb, c;
           if constexpr (kG) gring_get3(ring_g, a, bb, c);
@@ -764,7 +807,8 @@ template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_sme
   const size_t b = (size_t)2 * WF_NCODE * WfT<T>::KC * 32 * 16 +
                    (size_t)((ring_global<kLong>() ? 0 : ring_len) + (PHMM_XCHG_SMEM ? 32 : 0)) *
                        ring_slot_bytes<T, kLong>() +
-                   32;  // the stream's segment table (wf_stream)
+                   32 +  // the stream's segment table (wf_stream)
+                   (PHMM_DESC_SMEM ? 32 * 32 : 0);  // per-lane next-pass descriptors
   return (b + 15) & ~(size_t)15;
 }
 template <typename T> cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm);
@@ -786,7 +830,8 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
   __syncwarp();
   const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
   const uint32_t xbuf_s = ring_s + (uint32_t)(ring_global<kLong>() ? 0 : A.ring_len) * ring_slot_bytes<T, kLong>();  // design A only
-  const uint32_t seg_s = (ptab_s + per_warp - 32u) & ~7u;  // 32 B at the end of the warp's area (16-B aligned size)
+  const uint32_t seg_s = (ptab_s + per_warp - 32u) & ~7u;   // the stream's segment table (last 32 B)
+  const uint32_t desc_s = seg_s - 32u * 32u * PHMM_DESC_SMEM;  // per-lane descriptor slots (before it)  // 32 B at the end of the warp's area (16-B aligned size)
   // global ring of this warp (long-row launch): persistent warps, one region each
   const uint64_t ring_g = ring_global<kLong>()
       ? (uint64_t)(A.gring + ((size_t)blockIdx.x * (blockDim.x >> 5) + wib) * (size_t)A.ring_len * ring_slot_bytes<T, kLong>())
@@ -803,7 +848,7 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
     int64_t s, e;
     wf_item(A, it, lane, bin, s, e);
     if (e <= s) continue;
-    pending = wf_stream<T, kLong>(A, ptab_s, ring_s, ring_g, xbuf_s, seg_s, lane, s, (int)(e - s), bin,
+    pending = wf_stream<T, kLong>(A, ptab_s, ring_s, ring_g, xbuf_s, seg_s, desc_s, lane, s, (int)(e - s), bin,
                                   it == A.launch_items[0]);
     __syncwarp();
   }
