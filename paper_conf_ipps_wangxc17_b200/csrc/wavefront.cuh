@@ -401,6 +401,29 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
 }
 
+#ifndef PHMM_RS_TARGET
+#define PHMM_RS_TARGET 112  // ring rescale: a ring row whose max is below 2^PHMM_RS_TRIG is scaled to ~2^PHMM_RS_TARGET
+#endif
+#ifndef PHMM_RS_TRIG
+#define PHMM_RS_TRIG 104
+#endif
+#ifndef PHMM_RS_CAP
+#define PHMM_RS_CAP 126  // saturation of the scaled ring row (a saturated pair goes to the FP64 rescue)
+#endif
+#ifndef PHMM_PF_L1
+#define PHMM_PF_L1 0  // L1 prefetch of the next group's tables + code words: 1 FP64 pass, 2 both
+#endif
+template <typename T>
+__device__ __forceinline__ void wf_prefetch_block(const WfArgs2<T>& A, const BlkDesc& d, int k, int gi,
+                                                  int copy_len) {
+  const char* t = reinterpret_cast<const char*>(A.tab + d.tab_blk);
+#pragma unroll
+  for (int o = 0; o < (int)sizeof(TBlock<T>); o += 128) asm volatile("prefetch.global.L1 [%0];" :: "l"(t + o));
+  asm volatile("prefetch.global.L1 [%0];" :: "l"(t + sizeof(TBlock<T>) - 1));
+  const uint32_t col0 = d.hap_off + (uint32_t)(k * (copy_len + 1));
+  asm volatile("prefetch.global.L1 [%0];" :: "l"(A.hcodes + (col0 - 1u - (uint32_t)gi)));
+}
+
 // Ring slots [0, ncols] *= 2^sh, saturating at 2^110; true if any value saturated (the
 // sampled max missed a peak: the pair then goes to the FP64 rescue). Not inlined: it runs
 // once per rescaled pass and must not perturb the register allocation of the hot loop.
@@ -447,7 +470,7 @@ __device__ __forceinline__ bool wf_ring_scale(uint64_t ring_a, int ncols, int la
   constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
   const int nw = (ncols + 1) * (int)(RS / sizeof(T));
   const T f = (T)__int_as_float((127 + sh) << 23);
-  const T cap = (T)__int_as_float((127 + 110) << 23);
+  const T cap = (T)__int_as_float((127 + PHMM_RS_CAP) << 23);
   bool sat = false;
   __syncwarp();
   for (int k = lane; k < nw; k += 32) {
@@ -464,7 +487,7 @@ __device__ __forceinline__ bool wf_ring_scale(uint64_t ring_a, int ncols, int la
 
 // The ring rescale decision of one pass, all lanes: if lane 0's block
 // continues the pair of the ring row (`cont` of lane 0) and the row's max has decayed below
-// 2^64 (but not below 2^-90), scale the row to 2^80 and add the power of 2 to the pair's
+// 2^104 (but not below 2^-90), scale the row to 2^112 and add the power of 2 to the pair's
 // exponent slot (lane 0; a saturated row marks the pair for the FP64 rescue). Not inlined,
 // so that it leaves the hot loop's register allocation alone.
 template <typename T, bool kPacked, bool kG = false>
@@ -473,8 +496,8 @@ __device__ __noinline__ void wf_ring_rescale(uint64_t ring_a, int ncols, int lan
   const float rm = (float)wf_ring_max<T, kPacked, kG>(ring_a, ncols, lane);
   if (!(rm > 0.f && rm <= 3.0e38f)) return;
   const int E = ilogbf(rm);
-  if (E < -90 || E >= 64) return;
-  const int sh = min(80 - E, 126);
+  if (E < -90 || E >= PHMM_RS_TRIG) return;
+  const int sh = min(PHMM_RS_TARGET - E, 126);
   const bool sat = wf_ring_scale<T, kPacked, kG>(ring_a, ncols, lane, sh);
   if (lane == 0 && exp_slot) *exp_slot += sat ? -(1 << 24) : sh;
 }
@@ -758,6 +781,17 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
         }
       }
       if (e == NGRP - 1) c31B = -1 - (G - 1);  // virtual lane 63
+#if !PHMM_DESC_SMEM
+      if constexpr (PHMM_PF_L1 == 2 || (PHMM_PF_L1 == 1 && sizeof(T) == 8)) {
+        // the next group's lanes pull their next blocks' tables and first code words into L1,
+        // one switch event (8 steps) before they switch
+        if (grp == e + 1 && q < npass) {
+          const int bA = q * 64 + 2 * lane;
+          if (bA < nblk) wf_prefetch_block<T>(A, dnA, (1 + giA) & 3, giA, copy_len);
+          if (bA + 1 < nblk) wf_prefetch_block<T>(A, dnB, (1 + giB) & 3, giB, copy_len);
+        }
+      }
+#endif
       if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
         const int bA = q * 64 + 2 * lane, bB = bA + 1;
         const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);

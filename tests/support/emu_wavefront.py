@@ -20,6 +20,7 @@ import numpy as np
 
 G, PADC, MINP = 8, 5, 72
 RESCALE_COLS = 768  # long rows: passes 64 steps longer, ring rescale on
+RS_TARGET, RS_TRIG, RS_CAP = 112, 104, 126  # ring rescale: below 2^RS_TRIG -> ~2^RS_TARGET, saturating at 2^RS_CAP
 
 
 def pass_len(ncols):
@@ -165,10 +166,10 @@ def run_stream(blocks, ncols, K, rescale=True):
     rescale = ncols >= RESCALE_COLS
 
     def ring_scale(sh):
-        # saturating at 2^110: a peak the sampled max missed sends the pair to the FP64 rescue
+        # saturating at 2^RS_CAP (a saturated pair goes to the FP64 rescue)
         x = ring[0:ncols + 1].astype(np.float64) * 2.0 ** sh
-        ring[0:ncols + 1] = np.minimum(x, 2.0 ** 110).astype(E)
-        return bool(np.any(x > 2.0 ** 110))
+        ring[0:ncols + 1] = np.minimum(x, 2.0 ** RS_CAP).astype(E)
+        return bool(np.any(x > 2.0 ** RS_CAP))
 
     for q in range(npass + 1):
         for e in range(8):
@@ -180,8 +181,8 @@ def run_stream(blocks, ncols, K, rescale=True):
                 rm = float(np.max(ring[0:ncols + 1])) if cont else 0.0  # the whole ring row
                 if cont and 0 < rm <= 3.0e38:
                     Ex = int(np.floor(np.log2(rm)))
-                    if -90 <= Ex < 64:
-                        sh = min(80 - Ex, 126)
+                    if -90 <= Ex < RS_TRIG:
+                        sh = min(RS_TARGET - Ex, 126)
                 if sh:
                     pr_ = blocks[b]["pair"]
                     sat = ring_scale(sh)
