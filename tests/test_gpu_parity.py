@@ -294,3 +294,21 @@ def test_c4_reduced_fp64(ctx64):
     b = synth.config_batch("C4", n_regions=1)
     got, _ = ctx64.compute_batch(b)
     _check(got, oracle.batch_log10(b), "fp64")
+
+
+def test_long_rows_flat_gap_chains_no_overflow(ctx32):
+    """The ring rescale's overflow bound (every cell after a rescale to 2^112
+    is <= 2 * ncols * the ring row's max) near its worst: gap continuation Q1 (mu = epsilon =
+    0.79: D chains that barely decay along a row; Q0 would make beta = 0 and P = 0) and the
+    largest gap-open probabilities R16 allows (Q4), on long reads of the C4 shape. Every pair
+    must come out finite and within the FP32 tolerance, whether the FP32 pass keeps it or the
+    FP64 rescue takes it."""
+    b = synth.config_batch("C4", n_regions=1).subset(range(24))
+    b.gcp_quals = np.ones_like(b.gcp_quals)
+    b.ins_quals = np.full_like(b.ins_quals, 4)
+    b.del_quals = np.full_like(b.del_quals, 4)
+    got, st = ctx32.compute_batch(b)
+    ref = oracle.batch_log10(b)
+    assert np.all(np.isfinite(got))
+    _check(got, ref, "fp32")
+    assert np.sum(st == 0) > 0  # some pairs stay in the FP32 pass (through the rescale)
