@@ -232,7 +232,7 @@ def main():
     import torch
     import torch.distributed as dist
 
-    from paper_conf_ipps_wangxc17_b200 import phmm, synth
+    from paper_conf_ipps_wangxc17_b200 import parallel, phmm, synth
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
@@ -246,11 +246,17 @@ def main():
 
     stream = torch.cuda.Stream(device=dev)
     ctx = phmm.PairHMM(device=local, precision="fp32", stream=stream.cuda_stream, timing=True)
+    # the result gather (parallel.py): every rank's slot is padded to the largest shard
+    n_slot = n_pairs
+    if ws > 1:
+        nn = torch.tensor([n_pairs], dtype=torch.int64, device=dev)
+        dist.all_reduce(nn, op=dist.ReduceOp.MAX)
+        n_slot = int(nn.item())
     with torch.cuda.stream(stream):
         db = phmm.DeviceBatch.from_host(batch, device=dev)
-        out = torch.empty(n_pairs, dtype=torch.float64, device=dev)
+        out_slot = torch.full((n_slot,), float("nan"), dtype=torch.float64, device=dev)
+        out = out_slot[:n_pairs]
         status = torch.empty(n_pairs, dtype=torch.uint8, device=dev)
-        gathered = torch.empty(n_pairs * ws, dtype=torch.float64, device=dev) if ws > 1 else None
         flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     torch.cuda.synchronize()
 
@@ -258,7 +264,7 @@ def main():
         ctx.compute_batch_dev(db, out=out, status=status)
         if ws > 1:
             with torch.cuda.stream(stream):
-                dist.all_gather_into_tensor(gathered, out)
+                parallel.gather_results(out_slot, ws)
 
     for _ in range(max(args.warmup, 0)):
         step()
@@ -336,8 +342,8 @@ def main():
             t0 = time.perf_counter()
             rc = ctx.compute_batch_raw(s, hout.data_ptr(), hst.data_ptr())
             if ws > 1:
-                hg = torch.from_numpy(hout.numpy()).to(dev, non_blocking=False)
-                dist.all_gather_into_tensor(gathered, hg)
+                out_slot[:n_pairs].copy_(torch.from_numpy(hout.numpy()).to(dev, non_blocking=False))
+                parallel.gather_results(out_slot, ws)
                 torch.cuda.synchronize()
             e_ms.append((time.perf_counter() - t0) * 1e3)
             assert rc == 0, rc
