@@ -125,7 +125,7 @@ __global__ void k_item_nblocks(const int32_t* __restrict__ item_read, int64_t n_
   const int64_t n = n_items_dev ? *n_items_dev : n_items;
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = item_read ? item_read[k] : k;
-    const int64_t m = roff[r + 1] - roff[r];
+    const int64_t m = r >= 0 ? roff[r + 1] - roff[r] : 0;  // r < 0: unused item
     item_nb[k] = m >= 1 ? nblocks_of<K>((int)(m > (1 << 20) ? 1 : m)) : 0;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) item_nb[n] = 0;
@@ -202,6 +202,32 @@ __global__ void k_rebase_chunk(const int64_t* __restrict__ roff, int64_t rlo, in
       pairs_c[2 * i] = pairs[2 * (p0 + i)] - (int32_t)rlo;
       pairs_c[2 * i + 1] = pairs[2 * (p0 + i) + 1] - (int32_t)hlo;
     }
+  }
+}
+
+// item list of the rescue pass, one table item per distinct read: the rescued pairs' read ids
+// were sorted (sorted_read, with their list positions sorted_pos); item j = the j-th distinct
+// read, items past the last distinct read are unused (item_read = -1, no blocks)
+__global__ void k_rescue_read_keys(const int32_t* __restrict__ pairs, const int32_t* __restrict__ list, int64_t n,
+                                   uint32_t* __restrict__ keys, int32_t* __restrict__ vals) {
+  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
+    keys[k] = (uint32_t)pairs[2 * (int64_t)list[k]];
+    vals[k] = (int32_t)k;
+  }
+}
+__global__ void k_rescue_head_flags(const uint32_t* __restrict__ sorted_read, int64_t n, int32_t* __restrict__ head) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    head[i] = (i == 0 || sorted_read[i] != sorted_read[i - 1]) ? 1 : 0;
+}
+// incl = inclusive scan of the head flags: sorted entry i belongs to item incl[i] - 1
+__global__ void k_rescue_items_dedup(const uint32_t* __restrict__ sorted_read, const int32_t* __restrict__ sorted_pos,
+                                     const int32_t* __restrict__ head, const int32_t* __restrict__ incl, int64_t n,
+                                     int32_t* __restrict__ item_read, int32_t* __restrict__ pair_item) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t item = incl[i] - 1;
+    pair_item[sorted_pos[i]] = item;
+    if (head[i]) item_read[item] = (int32_t)sorted_read[i];
+    if (i >= incl[n - 1]) item_read[i] = -1;  // unused items (past the distinct reads)
   }
 }
 

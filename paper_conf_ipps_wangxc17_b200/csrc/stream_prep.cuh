@@ -104,6 +104,7 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t it = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; it < n_items; it += nwarps) {
     const int64_t r = item_read ? item_read[it] : it;
+    if (r < 0) continue;  // unused item (rescue pass, past the distinct reads)
     const int64_t r0 = roff[r];
     const int m = (int)(roff[r + 1] - r0);
     if (m < 1) continue;

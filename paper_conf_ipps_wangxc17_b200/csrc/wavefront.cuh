@@ -410,6 +410,10 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
 #ifndef PHMM_RS_CAP
 #define PHMM_RS_CAP 126  // saturation of the scaled ring row (a saturated pair goes to the FP64 rescue)
 #endif
+#ifndef PHMM_RESCUE_DEDUP
+#define PHMM_RESCUE_DEDUP 1  // rescue pass: one FP64 table per distinct read, not per rescued pair
+#endif
+constexpr bool WF_RESCUE_DEDUP = PHMM_RESCUE_DEDUP;
 #ifndef PHMM_PF_L1
 #define PHMM_PF_L1 0  // L1 prefetch of the next group's tables + code words: 1 FP64 pass, 2 both
 #endif
