@@ -312,3 +312,34 @@ def test_long_rows_flat_gap_chains_no_overflow(ctx32):
     assert np.all(np.isfinite(got))
     _check(got, ref, "fp32")
     assert np.sum(st == 0) > 0  # some pairs stay in the FP32 pass (through the rescale)
+
+
+def test_rescue_tables_shared_by_read(ctx32):
+    """The FP64 rescue builds one table per distinct read of the rescued pairs (DESIGN.md
+    §4.6): 6 random reads against 10 random haplotypes each (every pair far below the FP32
+    range), the pairs shuffled so that a read's pairs are scattered through the rescue list,
+    plus a few in-range pairs in between. Rescued pairs must match the oracle at FP64
+    accuracy; the result must not depend on the pair order."""
+    b = synth.random_pairs_batch(31, 60, m_range=(120, 160), n_range=(180, 240), qual_range=(30, 40),
+                                 indel_qual_range=(40, 45), gcp_range=(10, 10), n_frac=0.0)
+    pairs = np.stack([np.repeat(np.arange(6), 10), np.arange(60)], axis=1).astype(np.int32)
+    good = np.stack([np.arange(6, 12), np.arange(6, 12)], axis=1).astype(np.int32)  # read i vs its own hap i
+    perm = np.random.default_rng(4).permutation(66)
+    b.pairs = np.ascontiguousarray(np.concatenate([pairs, good])[perm])
+    b.hap_offsets = b.hap_offsets.copy()
+    # haplotypes 6..11 become copies of reads 6..11 (in-range pairs)
+    reads = [b.read_bases[b.read_offsets[i]:b.read_offsets[i + 1]] for i in range(b.n_reads)]
+    haps = [b.hap_bases[b.hap_offsets[i]:b.hap_offsets[i + 1]] for i in range(b.n_haps)]
+    for i in range(6, 12):
+        haps[i] = reads[i].copy()
+    b.hap_bases = np.ascontiguousarray(np.concatenate(haps))
+    b.hap_offsets = np.concatenate([[0], np.cumsum([h.size for h in haps])]).astype(np.int64)
+    got, st = ctx32.compute_batch(b)
+    ref = oracle.batch_log10(b)
+    resc = st == 1
+    assert resc.sum() == 60 and np.all(st[~resc] == 0)
+    _check(got[resc], ref[resc], "fp64")
+    _check(got[~resc], ref[~resc], "fp32")
+    inv = np.argsort(perm)
+    got2, _ = ctx32.compute_batch(b.subset(inv))
+    assert np.array_equal(got2, got[inv])
