@@ -1,7 +1,7 @@
 // wavefront.cuh -- the PairHMM wavefront kernel for sm_100a (the hot loop), FP32 and FP64.
 //
 // PRODUCT PATH. Computes Eq. 6 of PAPER.md (L18@541) over "tall streams" of
-// K-row blocks (see phmm_common.cuh for the Z/R/S1/S2 pad-row layout that makes
+// K-row blocks (see phmm_common.cuh for the Z/R/S pad-row layout that makes
 // a pair's termination sum (L20@2262) fall out of the recurrence).
 //
 // The paper's PH2 kernel (L20@3509, Fig. 8) gives one warp one pair and lets each
@@ -20,7 +20,7 @@
 //  * no per-lane "is this column real" branch: columns outside a block read the PAD
 //    code (prior 0); by induction down the lanes an idle virtual lane then computes
 //    exactly the boundary column (M = I = 0, D = D(i,0)) before its block and freezes
-//    the S2 running sum after it.
+//    the S running sum after it.
 //  * virtual lanes switch blocks in groups of G = 8 (8 switch events per pass); a pass
 //    is P = max(ncols + G, 72) steps.
 //  * row above: half B of a lane takes its own half A one step later (no shuffle);
@@ -428,9 +428,8 @@ __device__ __forceinline__ void wf_prefetch_block(const WfArgs2<T>& A, const Blk
   asm volatile("prefetch.global.L1 [%0];" :: "l"(A.hcodes + (col0 - 1u - (uint32_t)gi)));
 }
 
-// Ring slots [0, ncols] *= 2^sh, saturating at 2^110; true if any value saturated (the
-// sampled max missed a peak: the pair then goes to the FP64 rescue). Not inlined: it runs
-// once per rescaled pass and must not perturb the register allocation of the hot loop.
+// Ring rescale helpers, used once per rescaled pass by the non-inlined
+// wf_ring_rescale, so they do not perturb the register allocation of the hot loop.
 // Max of the ring row (slots [0, ncols], every value incl. the FP32 slot padding, which is
 // 0 or a scaled copy of real values), reduced over the warp.
 template <typename T, bool kG>
@@ -467,6 +466,8 @@ __device__ __forceinline__ T wf_ring_max(uint64_t ring_a, int ncols, int lane) {
   return m;
 }
 
+// Ring slots [0, ncols] *= 2^sh, saturating at 2^PHMM_RS_CAP; true if any value saturated
+// (cannot happen with the exact row max; such a pair would go to the FP64 rescue).
 template <typename T, bool kPacked, bool kG = false>
 __device__ __forceinline__ bool wf_ring_scale(uint64_t ring_a, int ncols, int lane, int sh) {
   // the slots as a flat array of T (FP32: the 4th word of a 16-byte slot is padding and is

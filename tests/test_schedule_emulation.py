@@ -1,6 +1,6 @@
 """The FP32 kernel's schedule, modelled on the CPU (tests/support/emu_wavefront.py):
 64 virtual lanes, group switch events, PAD-code idle columns, the ring and the
-Z/R/S1/S2 pad rows. The model must reproduce the oracle within the FP32 tolerance for
+Z/R/S pad rows. The model must reproduce the oracle within the FP32 tolerance for
 both row counts the kernel can be built with, and be independent of pair order."""
 import os
 import sys
