@@ -49,6 +49,15 @@ WORKLOADS = {
     "C5": "C5-shaped shard: mixed 100-250 bp reads, N ~ U{m..2m}",
 }
 DEFAULT_REGIONS = {"C2": 8192, "C3": 4096, "C4": 256, "C5": 8192}
+# The paper's PairHMM numbers: other hardware and its HCC1954 dataset,
+# context only (vs_baseline stays null).
+PAPER_CONTEXT = {
+    "PH2_peak_gcups": 34.8, "PH2_avg_gcups": 6.0,
+    "hardware": "NVIDIA GTX Titan X (Maxwell), 6,611 GFLOP/s FP32",
+    "workload": "HCC1954 PairHMM batches of GATK 3.6 HaplotypeCaller (avg 189 pairs), incl. host<->device transfer",
+    "PH2_over_PH1": "2.1x on Quadro K1200 (kernel time)",
+    "source": "PAPER.md L24@2217, L24@2258, L26@1631",
+}
 
 
 def _ncu_traffic(workload):
@@ -406,7 +415,8 @@ def main():
                            "l2": "flushed between timed steps (256 MiB write, untimed)",
                            "parallelism": f"dp{ws} (independent pair shards, NCCL all-gather of results)"},
                 "gpu_launches": launches,
-                "roofline": roofline, "rescue": rescue, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks}
+                "roofline": roofline, "rescue": rescue, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "paper_context": PAPER_CONTEXT}
         print(json.dumps(line), flush=True)
     ctx.close()
     if ws > 1:
