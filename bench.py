@@ -39,6 +39,7 @@ sys.path.insert(0, ROOT)
 FP32_OPS_PER_CELL = 8
 FP32_LANES_PER_SM = 128
 FP64_LANES_PER_SM = 64
+DFMA_MEASURED_PER_SM = 57.13  # microbench/issue_rates.cu "dfma" (profiles/r01_microbench_issue_rates.jsonl)
 SM_MAX_MHZ_FALLBACK = 1965.0
 
 WORKLOADS = {
@@ -393,8 +394,13 @@ def main():
     r_gcups = resc_cells / (rms / 1e3) / 1e9 if rms > 0 else None
     rescue = {"pairs": int(np.sum(st_host >= 1)), "cells": resc_cells, "ms": rms, "achieved": r_gcups,
               "peak": peak64, "unit": "GCUPS", "frac": (r_gcups / peak64) if r_gcups else None,
-              "kernel": "k_wavefront<double> (+ its per-pair table build)",
-              "peak_basis": f"{nsm} SM x {FP64_LANES_PER_SM} FP64 lanes x {sm_max:.0f} MHz / {FP32_OPS_PER_CELL} ops per cell"}
+              "kernel": "k_wavefront<double> (+ its per-read table build)",
+              "peak_basis": f"{nsm} SM x {FP64_LANES_PER_SM} FP64 lanes x {sm_max:.0f} MHz / {FP32_OPS_PER_CELL} ops per cell",
+              # the DFMA rate the microbenchmark measured on this pool's B200 (57.1 lane-ops/clk/SM,
+              # profiles/r01_microbench_issue_rates.jsonl) instead of the nominal 64
+              "peak_measured_dfma": nsm * DFMA_MEASURED_PER_SM * sm_max * 1e6 / FP32_OPS_PER_CELL / 1e9,
+              "frac_measured_dfma": (r_gcups / (nsm * DFMA_MEASURED_PER_SM * sm_max * 1e6 / FP32_OPS_PER_CELL / 1e9))
+              if r_gcups else None}
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline and not args.profile_steps:
