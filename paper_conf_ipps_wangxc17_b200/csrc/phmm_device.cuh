@@ -249,16 +249,28 @@ __global__ void k_rescue_items(const int32_t* __restrict__ pairs, const int32_t*
 // self-scheduling). tail_div = 0: all items full-size. bin_nbig[b] = full-size items of bin b.
 __device__ __forceinline__ unsigned long long block_scan_1024(unsigned long long v, unsigned long long* sh,
                                                               unsigned long long* total) {
-  sh[threadIdx.x] = v;
-  __syncthreads();
-  for (int off = 1; off < 1024; off <<= 1) {
-    const unsigned long long a = (threadIdx.x >= off) ? sh[threadIdx.x - off] : 0ull;
-    __syncthreads();
-    sh[threadIdx.x] += a;
-    __syncthreads();
+  // warp inclusive scans by shuffle, then a scan of the 32 warp totals by warp 0
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  unsigned long long x = v;
+#pragma unroll
+  for (int off = 1; off < 32; off <<= 1) {
+    const unsigned long long y = __shfl_up_sync(0xffffffffu, x, off);
+    if (lane >= off) x += y;
   }
-  const unsigned long long incl = sh[threadIdx.x];
-  *total = sh[1023];
+  if (lane == 31) sh[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    unsigned long long t = sh[lane];
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const unsigned long long y = __shfl_up_sync(0xffffffffu, t, off);
+      if (lane >= off) t += y;
+    }
+    sh[32 + lane] = t;  // inclusive prefix of the warp totals
+  }
+  __syncthreads();
+  const unsigned long long incl = x + (w > 0 ? sh[32 + w - 1] : 0ull);
+  *total = sh[63];
   __syncthreads();
   return incl - v;  // exclusive
 }
