@@ -34,7 +34,7 @@ enum BufId {
   B_SW_REF, B_SW_ROFF, B_SW_ALT, B_SW_AOFF, B_SW_TASKS, B_SW_RES, B_SW_OPS,  // SW host-variant staging
   B_SW_BTSZ, B_SW_BTOFF, B_SW_OPCAP, B_SW_OPOFF, B_SW_BT, B_SW_KEYS, B_SW_VALS, B_SW_OPTMP, B_SW_NOPS,
   B_SW_NOPOFF,
-  B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_EXP32, B_GRING,
+  B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_EXP32,
   B_CH_ROFF, B_CH_HOFF, B_CH_PAIRS, B_CH_CNT,  // host-variant pipeline: one chunk's rebased offsets / pairs
   B_DEDUP,                                       // rescue pass: head flags + their scan (one table per read)
   B_COUNT
@@ -469,7 +469,6 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   A.lpt = WF_LPT;
   A.out = out;
   A.exp_out = exp_out;
-  A.gring = nullptr;
   CUDA_TRY(cudaMemsetAsync(scal->item_counter, 0, sizeof(scal->item_counter), s));
   if (timed) ev_record(c, EV_WF0);
   for (int i = 0; i < nl; ++i) {
@@ -479,11 +478,6 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     A.item_counter = &scal->item_counter[i];
     A.launch_items = launch_items + 2 * i;
     const size_t smem = (i == 1 ? wf_warp_smem<T, true>(L[i].ring_len) : wf_warp_smem<T>(L[i].ring_len)) * L[i].warps;
-    if (i == 1 && ring_global<true>()) {  // the long launch's rings: one per resident warp, zeroed
-      const size_t gb = (size_t)c->nsm * L[i].bps * L[i].warps * (size_t)L[i].ring_len * ring_slot_bytes<T, true>();
-      ST_TRY(ws(c, B_GRING, gb, &A.gring));
-      CUDA_TRY(cudaMemsetAsync(A.gring, 0, gb, s));
-    }
     CUDA_TRY(wf_launch<T>(i == 1, (unsigned)(c->nsm * L[i].bps), L[i].warps, smem, s, A));
     ++c->launches;
   }

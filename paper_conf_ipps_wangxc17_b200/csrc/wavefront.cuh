@@ -77,16 +77,6 @@ constexpr int WF_TAIL_SPLIT = PHMM_TAIL_SPLIT;  // short items are 1/WF_TAIL_SPL
 #define PHMM_LPT 1
 #endif
 constexpr int WF_LPT = PHMM_LPT;  // 1: longest-row bins first inside a launch
-#ifndef PHMM_DESC_SMEM
-#define PHMM_DESC_SMEM 0  // 1: next-pass block descriptors travel by cp.async into shared memory
-#endif
-#ifndef PHMM_CONCAT
-#define PHMM_CONCAT 0
-#endif
-// 1: streams append further work items of their bin (measured slower: the hot loop's register
-// allocation gets worse); 0 keeps only the stream's segment table in shared
-// memory, which frees registers across the hot loop
-constexpr bool WF_CONCAT = PHMM_CONCAT;
 constexpr int WF_TAIL_DIV = PHMM_TAIL_DIV;  // last 1/WF_TAIL_DIV of a launch's blocks in short work items (0: none)
 constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
 constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
@@ -205,7 +195,6 @@ struct WfArgs2 {
   T* out;
   int32_t* exp_out;  // FP32 pass: per output slot, the power of 2 the ring rescale applied
   int ring_len;  // slots, >= P + 4
-  unsigned char* gring;  // long-row launch: per-warp global rings (ring_len slots each), zeroed per launch
 };
 
 template <typename T>
@@ -270,31 +259,8 @@ __device__ __forceinline__ void ring_get3(uint32_t a, double& x, double& y, doub
 // ring slot: 16 / 32 bytes (one vector load); packed 24 bytes (three scalar loads) in the
 // FP64 long-row kernel, where the ring limits occupancy (C4 rescue: 3 -> 4 warps per SM;
 // packing the FP32 long-row ring measured slower)
-#ifndef PHMM_GRING
-#define PHMM_GRING 0  // 1: the long-row launch keeps its ring in global memory (L2), not shared memory (measured slower)
-#endif
 template <typename T, bool kLong = false> __host__ __device__ constexpr bool ring_packed() {
-  return kLong && sizeof(T) == 8 && !PHMM_GRING;
-}
-// the long-row launch's ring lives in global memory (L2-resident, 16 / 32-byte slots): its
-// shared memory is then the prior tables only and occupancy is register-bound
-template <bool kLong> __host__ __device__ constexpr bool ring_global() { return kLong && PHMM_GRING; }
-// global-ring accessors (ld.global.cg: the ring is written inside the kernel, L2 only)
-__device__ __forceinline__ void gring_get3(uint64_t a, float& x, float& y, float& z) {
-  float w;
-  asm volatile("ld.global.cg.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(x), "=f"(y), "=f"(z), "=f"(w) : "l"(a) : "memory");
-  (void)w;
-}
-__device__ __forceinline__ void gring_get3(uint64_t a, double& x, double& y, double& z) {
-  asm volatile("ld.global.cg.v2.f64 {%0, %1}, [%3];\n\tld.global.cg.f64 %2, [%3+16];"
-               : "=d"(x), "=d"(y), "=d"(z) : "l"(a) : "memory");
-}
-__device__ __forceinline__ void gring_put3(uint64_t a, float x, float y, float z) {
-  asm volatile("st.global.v4.f32 [%0], {%1, %2, %3, %4};" :: "l"(a), "f"(x), "f"(y), "f"(z), "f"(0.f) : "memory");
-}
-__device__ __forceinline__ void gring_put3(uint64_t a, double x, double y, double z) {
-  asm volatile("st.global.v2.f64 [%0], {%1, %2};\n\tst.global.f64 [%0+16], %3;"
-               :: "l"(a), "d"(x), "d"(y), "d"(z) : "memory");
+  return kLong && sizeof(T) == 8;
 }
 template <typename T, bool kLong = false> __host__ __device__ constexpr uint32_t ring_slot_bytes() {
   return ring_packed<T, kLong>() ? 3u * (uint32_t)sizeof(T) : (sizeof(T) == 4 ? 16u : 32u);
@@ -333,9 +299,6 @@ __device__ __forceinline__ void lds16(uint32_t a, float* v) {
 }
 __device__ __forceinline__ void lds16(uint32_t a, double* v) {
   asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v[0]), "=d"(v[1]) : "r"(a) : "memory");
-}
-__device__ __forceinline__ void cp_async16(uint32_t a, const void* g) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(a), "l"(g) : "memory");
 }
 __device__ __forceinline__ void sts16(uint32_t a, const uint4 v) {
   asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" :: "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
@@ -414,61 +377,38 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
 #define PHMM_RESCUE_DEDUP 1  // rescue pass: one FP64 table per distinct read, not per rescued pair
 #endif
 constexpr bool WF_RESCUE_DEDUP = PHMM_RESCUE_DEDUP;
-#ifndef PHMM_PF_L1
-#define PHMM_PF_L1 0  // L1 prefetch of the next group's tables + code words: 1 FP64 pass, 2 both
-#endif
-template <typename T>
-__device__ __forceinline__ void wf_prefetch_block(const WfArgs2<T>& A, const BlkDesc& d, int k, int gi,
-                                                  int copy_len) {
-  const char* t = reinterpret_cast<const char*>(A.tab + d.tab_blk);
-#pragma unroll
-  for (int o = 0; o < (int)sizeof(TBlock<T>); o += 128) asm volatile("prefetch.global.L1 [%0];" :: "l"(t + o));
-  asm volatile("prefetch.global.L1 [%0];" :: "l"(t + sizeof(TBlock<T>) - 1));
-  const uint32_t col0 = d.hap_off + (uint32_t)(k * (copy_len + 1));
-  asm volatile("prefetch.global.L1 [%0];" :: "l"(A.hcodes + (col0 - 1u - (uint32_t)gi)));
-}
-
 // Ring rescale helpers, used once per rescaled pass by the non-inlined
 // wf_ring_rescale, so they do not perturb the register allocation of the hot loop.
 // Max of the ring row (slots [0, ncols], every value incl. the FP32 slot padding, which is
 // 0 or a scaled copy of real values), reduced over the warp.
-template <typename T, bool kG>
+// (the ring addresses travel as 64-bit values: that is the code generation measured, §4.8)
+template <typename T>
 __device__ __forceinline__ T ring_ld1(uint64_t a) {
   T x;
-  if constexpr (kG) {
-    if constexpr (sizeof(T) == 4) asm volatile("ld.global.cg.f32 %0, [%1];" : "=f"(x) : "l"(a) : "memory");
-    else asm volatile("ld.global.cg.f64 %0, [%1];" : "=d"(x) : "l"(a) : "memory");
-  } else {
-    if constexpr (sizeof(T) == 4) asm volatile("ld.shared.f32 %0, [%1];" : "=f"(x) : "r"((uint32_t)a) : "memory");
-    else asm volatile("ld.shared.f64 %0, [%1];" : "=d"(x) : "r"((uint32_t)a) : "memory");
-  }
+  if constexpr (sizeof(T) == 4) asm volatile("ld.shared.f32 %0, [%1];" : "=f"(x) : "r"((uint32_t)a) : "memory");
+  else asm volatile("ld.shared.f64 %0, [%1];" : "=d"(x) : "r"((uint32_t)a) : "memory");
   return x;
 }
-template <typename T, bool kG>
+template <typename T>
 __device__ __forceinline__ void ring_st1(uint64_t a, T x) {
-  if constexpr (kG) {
-    if constexpr (sizeof(T) == 4) asm volatile("st.global.f32 [%0], %1;" :: "l"(a), "f"(x) : "memory");
-    else asm volatile("st.global.f64 [%0], %1;" :: "l"(a), "d"(x) : "memory");
-  } else {
-    if constexpr (sizeof(T) == 4) asm volatile("st.shared.f32 [%0], %1;" :: "r"((uint32_t)a), "f"(x) : "memory");
-    else asm volatile("st.shared.f64 [%0], %1;" :: "r"((uint32_t)a), "d"(x) : "memory");
-  }
+  if constexpr (sizeof(T) == 4) asm volatile("st.shared.f32 [%0], %1;" :: "r"((uint32_t)a), "f"(x) : "memory");
+  else asm volatile("st.shared.f64 [%0], %1;" :: "r"((uint32_t)a), "d"(x) : "memory");
 }
 
-template <typename T, bool kPacked, bool kG = false>
+template <typename T, bool kPacked>
 __device__ __forceinline__ T wf_ring_max(uint64_t ring_a, int ncols, int lane) {
   constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
   const int nw = (ncols + 1) * (int)(RS / sizeof(T));
   T m = 0;
   __syncwarp();
-  for (int k = lane; k < nw; k += 32) m = fmax(m, ring_ld1<T, kG>(ring_a + (uint64_t)(k * (int)sizeof(T))));
+  for (int k = lane; k < nw; k += 32) m = fmax(m, ring_ld1<T>(ring_a + (uint64_t)(k * (int)sizeof(T))));
   for (int o = 16; o > 0; o >>= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
   return m;
 }
 
 // Ring slots [0, ncols] *= 2^sh, saturating at 2^PHMM_RS_CAP; true if any value saturated
 // (cannot happen with the exact row max; such a pair would go to the FP64 rescue).
-template <typename T, bool kPacked, bool kG = false>
+template <typename T, bool kPacked>
 __device__ __forceinline__ bool wf_ring_scale(uint64_t ring_a, int ncols, int lane, int sh) {
   // the slots as a flat array of T (FP32: the 4th word of a 16-byte slot is padding and is
   // scaled too): consecutive lanes on consecutive words, no bank conflicts
@@ -480,11 +420,11 @@ __device__ __forceinline__ bool wf_ring_scale(uint64_t ring_a, int ncols, int la
   __syncwarp();
   for (int k = lane; k < nw; k += 32) {
     const uint64_t a = ring_a + (uint64_t)(k * (int)sizeof(T));
-    T x = ring_ld1<T, kG>(a);
+    T x = ring_ld1<T>(a);
     x *= f;
     sat |= x > cap;
     x = fmin(x, cap);
-    ring_st1<T, kG>(a, x);
+    ring_st1<T>(a, x);
   }
   __syncwarp();
   return __any_sync(0xffffffffu, sat);
@@ -495,15 +435,15 @@ __device__ __forceinline__ bool wf_ring_scale(uint64_t ring_a, int ncols, int la
 // 2^104 (but not below 2^-90), scale the row to 2^112 and add the power of 2 to the pair's
 // exponent slot (lane 0; a saturated row marks the pair for the FP64 rescue). Not inlined,
 // so that it leaves the hot loop's register allocation alone.
-template <typename T, bool kPacked, bool kG = false>
+template <typename T, bool kPacked>
 __device__ __noinline__ void wf_ring_rescale(uint64_t ring_a, int ncols, int lane, bool cont, int32_t* exp_slot) {
   if (!__shfl_sync(0xffffffffu, (int)cont, 0)) return;
-  const float rm = (float)wf_ring_max<T, kPacked, kG>(ring_a, ncols, lane);
+  const float rm = (float)wf_ring_max<T, kPacked>(ring_a, ncols, lane);
   if (!(rm > 0.f && rm <= 3.0e38f)) return;
   const int E = ilogbf(rm);
   if (E < -90 || E >= PHMM_RS_TRIG) return;
   const int sh = min(PHMM_RS_TARGET - E, 126);
-  const bool sat = wf_ring_scale<T, kPacked, kG>(ring_a, ncols, lane, sh);
+  const bool sat = wf_ring_scale<T, kPacked>(ring_a, ncols, lane, sh);
   if (lane == 0 && exp_slot) *exp_slot += sat ? -(1 << 24) : sh;
 }
 
@@ -557,18 +497,17 @@ __device__ __forceinline__ unsigned long long wf_claim(const WfArgs2<T>& A, int 
   return __shfl_sync(0xffffffffu, it, 0);
 }
 
-// One warp streams through blocks [s, s+nblk) of one bin (ncols columns each), and -- with
-// WF_CONCAT, off by default -- through the blocks of the further work items it claims while the stream
-// nears its end, as long as they are in the same bin and hold >= 64 blocks: the stream is the
-// concatenation of their block ranges (logical block b -> physical block through the last two
-// segments), so no pass is left partly idle between items and there is one drain per stream,
-// not one per item (a pair always starts on Z rows, so the junction needs no care). Returns an
-// item claimed but not taken (another bin or < 64 blocks; >= launch end: none left), or ~0.
+// One warp streams through blocks [s, s+nblk) of one bin (ncols columns each). The stream's
+// block range lives in a per-warp shared-memory segment table (read at switch events only),
+// which keeps it out of the registers of the hot loop (212 instead of 218
+// registers). The table has room for a second segment: appending the next work item of the
+// same bin to a stream (one drain per stream instead of per item) was measured slower and
+// removed. Returns the next work item to run (~0: claim a new one).
 // kLong: the launch of the long-row bins (the only one with the ring rescale compiled in).
 template <typename T, bool kLong>
 __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s,
-                                                        uint64_t ring_g, uint32_t xbuf_s, uint32_t seg_s,
-                                                        uint32_t desc_s, int lane,
+                                                        uint32_t xbuf_s, uint32_t seg_s,
+                                                        int lane,
                                                         int64_t s, int nblk, int bin, bool trace = false) {
   const int ncols = bin * A.bucket;
   // segments of the concatenated stream, kept in shared memory (warp-uniform, read at switch
@@ -578,13 +517,11 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
   __syncwarp();
   if (lane == 0) { seg[0] = s; seg[1] = s; seg[2] = 0; seg[3] = 0; }
   __syncwarp();
-  unsigned long long pending = ~0ull;
-  bool more = WF_CONCAT;  // may still claim items to append
+  const unsigned long long pending = ~0ull;
   auto phys = [&](int b) -> int64_t {
     const int64_t cL = seg[2];
     return b >= cL ? seg[0] + (b - cL) : seg[1] + (b - seg[3]);
   };
-  constexpr bool kG = ring_global<kLong>();  // ring in global memory (ring_g) instead of shared (ring_s)
   using V = typename WfT<T>::V;
   constexpr int K = WfT<T>::K;
   constexpr int PER = 16 / sizeof(T);
@@ -618,57 +555,11 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
   int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
   int c31B = -(1 << 20);  // (uniform) column of virtual lane 63 (lane 31, half B)
   T rvM = 0, rvI = 0, rvD = 0;  // lane 31: ring slot for virtual lane 0's next column
-  // global ring: lane 31 loads each slot 4 steps before its use (step r of a group loads the
-  // slot of step r of the next group into rq*[r])
-  T rqM[4] = {0, 0, 0, 0}, rqI[4] = {0, 0, 0, 0}, rqD[4] = {0, 0, 0, 0};
-#if PHMM_DESC_SMEM
-  // descriptors of the lane's next blocks, copied one pass ahead by cp.async into a per-lane
-  // shared-memory slot (no registers held across the hot loop)
-  const uint32_t dnA_s = desc_s + 32u * lane, dnB_s = dnA_s + 16u;
-  {
-    const uint4 none = make_uint4(0u, 0u, 0xffffffffu, 1u);  // tab 0, hap 0, out -1, n 1, flags 0
-    __syncwarp();
-    sts16(dnA_s, none);
-    sts16(dnB_s, none);
-    if (2 * lane < nblk) cp_async16(dnA_s, A.blk + s + 2 * lane);
-    if (2 * lane + 1 < nblk) cp_async16(dnB_s, A.blk + s + 2 * lane + 1);
-  }
-  auto ld_desc = [](uint32_t a) {
-    asm volatile("cp.async.wait_all;" ::: "memory");
-    uint4 v;
-    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a)
-                 : "memory");
-    BlkDesc d;
-    d.tab_blk = v.x; d.hap_off = v.y; d.out_idx = (int32_t)v.z; d.n = (uint16_t)(v.w & 0xffffu);
-    d.flags = (uint16_t)(v.w >> 16);
-    return d;
-  };
-#else
   BlkDesc dnA, dnB;  // descriptors of the lane's next blocks (loaded one pass ahead)
   dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.n = 1; dnA.flags = 0;
   dnB = dnA;
   if (2 * lane < nblk) dnA = A.blk[s + 2 * lane];
   if (2 * lane + 1 < nblk) dnB = A.blk[s + 2 * lane + 1];
-#endif
-  // append the next work item when the stream would end within this pass or the next (its
-  // blocks then fill the passes whose descriptors are prefetched from here on)
-  auto try_append = [&](int q) {
-    while (more && (q + 2) * 64 >= nblk) {
-      const unsigned long long it = wf_claim(A, lane);
-      if (it >= A.launch_items[1]) { pending = it; more = false; break; }
-      int b2;
-      int64_t s2, e2;
-      wf_item(A, it, lane, b2, s2, e2);
-      if (e2 <= s2) continue;  // empty after pair alignment
-      if (b2 != bin || e2 - s2 < 64) { pending = it; more = false; break; }
-      __syncwarp();
-      if (lane == 0) { seg[1] = seg[0]; seg[3] = seg[2]; seg[0] = s2; seg[2] = nblk; }
-      __syncwarp();
-      nblk += (int)(e2 - s2);
-      npass = (nblk + 63) >> 6;
-      break;
-    }
-  };
 #ifdef PHMM_DBG_TRACE
   int tstep = 0;
 #endif
@@ -685,9 +576,7 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
   constexpr bool rescale = kLong && PHMM_RING_RESCALE && sizeof(T) == 4;  // long-row launch: ncols >= WF_RESCALE_COLS
 
   auto step = [&](const int r) {
-    if constexpr (!kG) {
-      if (is31) rget<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
-    }
+    if (is31) rget<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
     // code byte r (= code*WF_CB) placed in byte 1 -> the code's rows in the table
     // code stride of this pass's table relative to the code byte's (powers of 2)
     constexpr int kKC = WfT<T>::KC;
@@ -708,19 +597,11 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
     const T m3a = lo(L.M[LR]), i3a = lo(L.I[LR]), d3a = lo(L.D[LR]);
     const T m3b = hi(L.M[LR]), i3b = hi(L.I[LR]), d3b = hi(L.D[LR]);
     // half B of lane-1 -> half A of lane; lane 31 sends the ring slot instead (virtual 63 -> 0)
-    const T sM = is31 ? (kG ? rqM[r] : rvM) : m3b;
-    const T sI = is31 ? (kG ? rqI[r] : rvI) : i3b;
-    const T sD = is31 ? (kG ? rqD[r] : rvD) : d3b;
-    if constexpr (kG) {
-      // lane 31 loads the slot of c0 four steps later into the registers it just sent; across
-      // a pass end (slots up to P + 4) the loads are stale and replaced by the reload at the
-      // next pass start
-      if (is31) gring_get3(ring_g + (uint64_t)(RS * (uint32_t)(c0 + 6)), rqM[r], rqI[r], rqD[r]);
-    }
-    if (is31 && (unsigned)(c31B + 1) <= (unsigned)ncols) {  // -1 <= c31B < ncols
-      if constexpr (kG) gring_put3(ring_g + RS * (uint64_t)(c31B + 1), m3b, i3b, d3b);
-      else rput<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c31B + 1), m3b, i3b, d3b);
-    }
+    const T sM = is31 ? rvM : m3b;
+    const T sI = is31 ? rvI : i3b;
+    const T sD = is31 ? rvD : d3b;
+    if (is31 && (unsigned)(c31B + 1) <= (unsigned)ncols)  // -1 <= c31B < ncols
+      rput<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c31B + 1), m3b, i3b, d3b);
     dgM = upM; dgI = upI; dgD = upD;
     // next step: half A's row above = lane-1's half B; half B's row above = this lane's half A
 #if PHMM_XCHG_SMEM
@@ -762,7 +643,6 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
   };
 
   for (int q = 0; q <= npass; ++q) {
-    if (q < npass) try_append(q);
 #pragma unroll 1
     for (int e = 0; e < NGRP; ++e) {
       if (e == 0) {
@@ -770,41 +650,16 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
         if constexpr (rescale) {
           // lane 0's block of this pass continues the pair of virtual lane 63's last block?
           // (rows shorter than WF_RESCALE_COLS have no complete ring row at the pass start)
-#if PHMM_DESC_SMEM
-          const BlkDesc dnA = ld_desc(dnA_s);
-#endif
           const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && ncols >= WF_RESCALE_COLS;
-          wf_ring_rescale<T, ring_packed<T, kLong>(), kG>(kG ? ring_g : (uint64_t)ring_s, ncols, lane, cont,
-                                                          A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
-        }
-        if constexpr (kG) {  // lane 31: (re)load the first 4 slots of the pass (after any rescale)
-          __syncwarp();
-          if (is31) {
-#pragma unroll
-            for (int r = 0; r < 4; ++r) gring_get3(ring_g + RS * (uint64_t)(r + 1), rqM[r], rqI[r], rqD[r]);
-          }
+          wf_ring_rescale<T, ring_packed<T, kLong>()>((uint64_t)ring_s, ncols, lane, cont,
+                                                      A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
         }
       }
       if (e == NGRP - 1) c31B = -1 - (G - 1);  // virtual lane 63
-#if !PHMM_DESC_SMEM
-      if constexpr (PHMM_PF_L1 == 2 || (PHMM_PF_L1 == 1 && sizeof(T) == 8)) {
-        // the next group's lanes pull their next blocks' tables and first code words into L1,
-        // one switch event (8 steps) before they switch
-        if (grp == e + 1 && q < npass) {
-          const int bA = q * 64 + 2 * lane;
-          if (bA < nblk) wf_prefetch_block<T>(A, dnA, (1 + giA) & 3, giA, copy_len);
-          if (bA + 1 < nblk) wf_prefetch_block<T>(A, dnB, (1 + giB) & 3, giB, copy_len);
-        }
-      }
-#endif
       if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
         const int bA = q * 64 + 2 * lane, bB = bA + 1;
         const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
-#if PHMM_DESC_SMEM
-        const BlkDesc dA = ld_desc(dnA_s), dB = ld_desc(dnB_s);  // copied one pass ago (pass 0: before the loop)
-#else
         const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
-#endif
         if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S row: the last-row M+I sum (L20@2262)
         if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
         pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
@@ -813,17 +668,11 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
         wB_nx = __ldg(pB); wB_nx2 = __ldg(pB + 1); pB += 2;
         // prefetch the next pass's descriptors after this pass's loads are issued (a load
         // issued before the consumers of the previous prefetch would share its scoreboard)
-#if PHMM_DESC_SMEM
-        if (bA + 64 < nblk) cp_async16(dnA_s, A.blk + phys(bA + 64));
-        if (bB + 64 < nblk) cp_async16(dnB_s, A.blk + phys(bB + 64));
-#else
         if (bA + 64 < nblk) dnA = A.blk[phys(bA + 64)];
         if (bB + 64 < nblk) dnB = A.blk[phys(bB + 64)];
-#endif
         if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
           T a, bb, c;
-          if constexpr (kG) gring_get3(ring_g, a, bb, c);
-          else rget<ring_packed<T, kLong>()>(ring_s, a, bb, c);
+          rget<ring_packed<T, kLong>()>(ring_s, a, bb, c);
           upM = set_half<0>(upM, a); upI = set_half<0>(upI, bb); upD = set_half<0>(upD, c);
         }
       }
@@ -844,10 +693,9 @@ template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_sme
   // prior tables, ring, and (design-A ablation only) the exchange line buffer; a multiple of
   // 16 bytes so that every warp's tables stay 16-byte aligned
   const size_t b = (size_t)2 * WF_NCODE * WfT<T>::KC * 32 * 16 +
-                   (size_t)((ring_global<kLong>() ? 0 : ring_len) + (PHMM_XCHG_SMEM ? 32 : 0)) *
+                   (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) *
                        ring_slot_bytes<T, kLong>() +
-                   32 +  // the stream's segment table (wf_stream)
-                   (PHMM_DESC_SMEM ? 32 * 32 : 0);  // per-lane next-pass descriptors
+                   32;  // the stream's segment table (wf_stream)
   return (b + 15) & ~(size_t)15;
 }
 template <typename T> cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm);
@@ -868,13 +716,8 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
   for (uint32_t i = 4 * lane; i < per_warp; i += 128) *reinterpret_cast<uint32_t*>(base + i) = 0u;
   __syncwarp();
   const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
-  const uint32_t xbuf_s = ring_s + (uint32_t)(ring_global<kLong>() ? 0 : A.ring_len) * ring_slot_bytes<T, kLong>();  // design A only
+  const uint32_t xbuf_s = ring_s + (uint32_t)A.ring_len * ring_slot_bytes<T, kLong>();  // design A only
   const uint32_t seg_s = (ptab_s + per_warp - 32u) & ~7u;   // the stream's segment table (last 32 B)
-  const uint32_t desc_s = seg_s - 32u * 32u * PHMM_DESC_SMEM;  // per-lane descriptor slots (before it)  // 32 B at the end of the warp's area (16-B aligned size)
-  // global ring of this warp (long-row launch): persistent warps, one region each
-  const uint64_t ring_g = ring_global<kLong>()
-      ? (uint64_t)(A.gring + ((size_t)blockIdx.x * (blockDim.x >> 5) + wib) * (size_t)A.ring_len * ring_slot_bytes<T, kLong>())
-      : 0ull;
   // work items of the launch, claimed from an atomic counter; a stream may append further
   // items of its bin (wf_stream) and hands back the one it claimed but could not take
   const unsigned long long it1 = A.launch_items[1];
@@ -887,7 +730,7 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
     int64_t s, e;
     wf_item(A, it, lane, bin, s, e);
     if (e <= s) continue;
-    pending = wf_stream<T, kLong>(A, ptab_s, ring_s, ring_g, xbuf_s, seg_s, desc_s, lane, s, (int)(e - s), bin,
+    pending = wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, seg_s, lane, s, (int)(e - s), bin,
                                   it == A.launch_items[0]);
     __syncwarp();
   }
