@@ -1,0 +1,33 @@
+"""bench.py on the GPU keeps the driver's JSON contract (one line; value, roofline, e2e,
+clocks, gpu_launches, cpu_baseline) on a reduced C2 shard."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_bench_json_line():
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--regions", "512", "--steps", "3",
+                        "--warmup", "3", "--cpu-seconds", "1"], capture_output=True, text=True, timeout=900,
+                       cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.strip()]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "gpu_launches", "roofline", "cpu_baseline", "e2e", "clocks"):
+        assert k in d, k
+    assert d["n_gpus"] == 1 and d["steps"] == 3 and d["warmup"] == 3 and d["value"] > 0
+    assert d["gpu_launches"] > 0 and d["scaling"] == "weak" and d["vs_baseline"] is None
+    rf = d["roofline"]
+    assert rf["bound"] == "alu" and 0 < rf["frac"] < 1 and rf["achieved"] > d["value"]
+    e = d["e2e"]
+    assert 0 < e["value"] <= d["value"] * 1.05 and e["h2d_bytes_per_step"] > 0 and e["d2h_bytes_per_step"] > 0
+    c = d["cpu_baseline"]
+    assert c["kind"] == "oracle" and c["cores"] >= 1 and c["parity_max_abs_log10"] <= 1e-3
+    assert d["clocks"]["samples"] >= 1

@@ -343,3 +343,17 @@ def test_rescue_tables_shared_by_read(ctx32):
     inv = np.argsort(perm)
     got2, _ = ctx32.compute_batch(b.subset(inv))
     assert np.array_equal(got2, got[inv])
+
+
+def test_full_c2_fp64_mode_sampled(ctx64):
+    """The FP64 path (PHMM_PREC_FP64) on the whole of BASELINE configs[1] (2^20 pairs):
+    a seeded sample against the oracle at the north star's 1e-9 relative tolerance."""
+    import torch
+
+    b = synth.config_batch("C2")
+    db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+    out, st = ctx64.compute_batch_dev(db)
+    torch.cuda.synchronize()
+    out = out.cpu().numpy()
+    sample = np.random.default_rng(321).choice(b.n_pairs, 2000, replace=False)
+    _check(out[sample], oracle.batch_log10(b, pair_idx=sample), "fp64")
