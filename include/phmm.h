@@ -118,6 +118,11 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg);
  * and, if non-NULL, out_status (n_pairs bytes) are written.
  * out_log10[p] = log10 P(read | hap) of pair p; -inf when P underflows even
  * the FP64 rescue or is exactly 0 (Q0 inputs).
+ * With the environment variable PHMM_CHUNKS=n (2..4) set when the context is
+ * created, batches of >= 2^17 pairs are copied and computed in n chunks whose
+ * copies overlap the previous chunk's FP32 pass (same results bit for bit;
+ * measured slower on B200, so off by default). Inputs are
+ * validated chunk by chunk; an error still leaves the outputs untouched.
  */
 phmm_status phmm_compute_batch(phmm_ctx* ctx, const phmm_batch* b, double* out_log10,
                                uint8_t* out_status);

@@ -4,7 +4,8 @@ cat > /tmp/san_case.py <<'PY'
 import sys; sys.path.insert(0, '.')
 import numpy as np
 from paper_conf_ipps_wangxc17_b200 import phmm, synth
-b = synth.concat_batches([synth.config_batch("C2", n_regions=4), synth.random_pairs_batch(3, 100, m_range=(1, 60), n_range=(1, 80))])
+b = synth.concat_batches([synth.config_batch("C2", n_regions=4), synth.random_pairs_batch(3, 100, m_range=(1, 60), n_range=(1, 80)),
+                          synth.config_batch("C3", n_regions=1), synth.config_batch("C4", n_regions=1).subset(range(6))])
 for prec in ("fp32", "fp64"):
     with phmm.PairHMM(precision=prec) as h:
         out, st = h.compute_batch(b)
