@@ -350,10 +350,11 @@ def main(out_path: str = os.path.join(ROOT, "profiles", "r01_shuffle_study.json"
         b = _bench_kernel(lib)
         r = b["roofline"]
         ptx = os.path.join(_PKG, "ptxas_info.txt") if tag.startswith("B") else lib + ".ptxas.txt"
-        regs = _ptxas_regs(ptx, "_ZN4phmm11k_wavefrontIfEEvNS_7WfArgs2IT_EE") or 0
-        mangled = "_ZN4phmm11k_wavefrontIfEEvNS_7WfArgs2IT_EE"
+        mangled = "_ZN4phmm11k_wavefrontIfLb0EEEvNS_7WfArgs2IT_EE"  # k_wavefront<float, false>
+        regs = _ptxas_regs(ptx, mangled) or 0
         ncols = 304  # C2: N = 300 -> ncols 304, P = 312, ring 316 slots of 16 B
-        smem_block = 4 * (2 * 6 * 2 * 32 * 16 + (316 + (32 if tag.startswith("A") else 0)) * 16)
+        # wf_warp_smem<float>: prior tables + ring (+ design A's line buffer) + segment table
+        smem_block = 4 * ((2 * 6 * 2 * 32 * 16 + (316 + (32 if tag.startswith("A") else 0)) * 16 + 32 + 15) & ~15)
         designs[tag] = {"lib": os.path.relpath(lib, ROOT), "kernel_gcups": r["achieved"], "frac": r["frac"],
                         "wavefront_ms": r["wavefront_ms"], "step_gcups": b["value"], "regs_per_thread": regs,
                         "smem_per_block": smem_block, "ncols": ncols,
