@@ -223,6 +223,10 @@ def latency_table(results: Sequence[MicroResult]) -> Dict[str, float]:
     return derive_latencies(slopes)
 
 
+# the short-row FP32 wavefront kernel, k_wavefront<float, false> (csrc/wavefront.cuh)
+WF32_SYMBOL = "_ZN4phmm11k_wavefrontIfLb0EEEvNS_7WfArgs2IT_EE"
+
+
 def hot_loop_mix(so_path: str, mangled: str) -> Dict[str, int]:
     """Opcode counts of the innermost loop with the most packed FP32 instructions of a
     kernel (cuobjdump -sass), i.e. one group of 4 steps of the wavefront kernel."""
@@ -350,7 +354,7 @@ def main(out_path: str = os.path.join(ROOT, "profiles", "r01_shuffle_study.json"
         b = _bench_kernel(lib)
         r = b["roofline"]
         ptx = os.path.join(_PKG, "ptxas_info.txt") if tag.startswith("B") else lib + ".ptxas.txt"
-        mangled = "_ZN4phmm11k_wavefrontIfLb0EEEvNS_7WfArgs2IT_EE"  # k_wavefront<float, false>
+        mangled = WF32_SYMBOL
         regs = _ptxas_regs(ptx, mangled) or 0
         ncols = 304  # C2: N = 300 -> ncols 304, P = 312, ring 316 slots of 16 B
         # wf_warp_smem<float>: prior tables + ring (+ design A's line buffer) + segment table

@@ -129,3 +129,22 @@ print("ok", d)
         outs.append(np.load(fn))
         os.unlink(fn)
     assert np.array_equal(outs[0], outs[1])
+
+
+@pytest.mark.parametrize("lib", ["libphmm.so", "libphmm_xsmem.so"])
+def test_hot_loop_mix_finds_the_wavefront_kernel(lib):
+    """The study's SASS / ptxas lookups name the kernel that the libraries actually contain
+    (a stale symbol would silently drop the design comparison's instruction mix)."""
+    so = os.path.join(ROOT, "paper_conf_ipps_wangxc17_b200", lib)
+    if not os.path.exists(so):
+        pytest.skip("library not built")
+    mix = ss.hot_loop_mix(so, ss.WF32_SYMBOL)
+    # one group of 4 steps x 16 cells per lane: the 5-op rescaled cell is 320 FP32 lane-ops
+    fp_ops = 2 * (mix.get("FFMA2", 0) + mix.get("FMUL2", 0) + mix.get("FADD2", 0)) + \
+        mix.get("FFMA", 0) + mix.get("FMUL", 0) + mix.get("FADD", 0)
+    assert fp_ops == 320, mix
+    assert mix.get("SHFL", 0) > 0 if lib == "libphmm.so" else mix.get("STS", 0) > mix.get("SHFL", 0)
+    ptx = os.path.join(ROOT, "paper_conf_ipps_wangxc17_b200",
+                       "ptxas_info.txt" if lib == "libphmm.so" else lib + ".ptxas.txt")
+    if os.path.exists(ptx):
+        assert 0 < ss._ptxas_regs(ptx, ss.WF32_SYMBOL) <= 255
