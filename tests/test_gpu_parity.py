@@ -357,3 +357,16 @@ def test_full_c2_fp64_mode_sampled(ctx64):
     out = out.cpu().numpy()
     sample = np.random.default_rng(321).choice(b.n_pairs, 2000, replace=False)
     _check(out[sample], oracle.batch_log10(b, pair_idx=sample), "fp64")
+
+
+@pytest.mark.parametrize("seed", [41, 42])
+def test_fully_ragged_one_batch(ctx32, ctx64, seed):
+    """One batch that spans every launch kind at once: random m in 1..400 and N in 1..2000
+    (many length bins, multi-block reads, long-row launches with ring carry) with random
+    Q0..60 base qualities (part of the pairs fall below the FP32 range and are rescued)."""
+    b = synth.random_pairs_batch(seed, 160, m_range=(1, 400), n_range=(1, 2000))
+    ref = oracle.batch_log10(b)
+    got32, st = ctx32.compute_batch(b)
+    _check(got32, ref, "fp32")
+    assert set(np.unique(st)) <= {0, 1, 2}
+    _check(ctx64.compute_batch(b)[0], ref, "fp64")
