@@ -32,11 +32,35 @@
  *
  * Errors: every call validates its arguments and inputs before any output is
  * written; on error it returns a negative status and leaves the outputs
- * untouched. Input-content errors (bad base, quality > 127, empty sequence,
- * pair index out of range) are detected on the device in the same pass that
- * reads the data; the call then returns the error without writing outputs.
- * CUDA failures return PHMM_E_CUDA. A context is bound to one device, is not
+ * untouched (both variants compute into context scratch and copy the results
+ * to the caller's buffers only after the whole path, FP64 rescue included,
+ * succeeded). Input-content errors (bad base, bad quality, empty sequence,
+ * pair index out of range, length caps) are detected on the device in the
+ * same pass that reads the data; the call then returns the error without
+ * writing outputs. CUDA failures return PHMM_E_CUDA (the context stays usable
+ * after a recoverable one). A context is bound to one device, is not
  * thread-safe, and holds no global state: use one context per host thread.
+ *
+ * Input limits (each violation -> the status named, outputs untouched):
+ *   - bases: 'A','C','G','T','N' only (uppercase)          -> PHMM_E_INVALID_BASE
+ *   - every quality <= 127                                  -> PHMM_E_INVALID_QUAL
+ *   - every read base with e(qi) + e(qd) <= 1, i.e. no base
+ *     with qi or qd <= 3 whose two gap-open probabilities
+ *     sum above 1 (reading R16: the transitions
+ *     out of M must be a distribution; checked on EVERY
+ *     read of the batch, used by a pair or not)            -> PHMM_E_INVALID_QUAL
+ *   - a read or haplotype used by a pair has length >= 1   -> PHMM_E_EMPTY_SEQ
+ *   - pair indices inside [0, n_reads) x [0, n_haps)       -> PHMM_E_INDEX
+ *   - a haplotype used by a pair has N <= 4094 bases and a
+ *     read used by a pair has m <= 2^20 bases (unused
+ *     sequences may be longer)                             -> PHMM_E_INVALID_ARG
+ *   - n_pairs, n_reads, n_haps <= 2^31 - 1                 -> PHMM_E_INVALID_ARG
+ *
+ * Synchronisation: every compute call returns only when its results are in
+ * the caller's buffers (the path reads device-computed sizes back to the host
+ * a few times per call, so it cannot be captured in a CUDA graph). Work is
+ * issued on the context's stream: the cuda_stream of phmm_config, or the one
+ * set by phmm_set_stream, or (NULL) a stream the context owns.
  */
 #ifndef PHMM_H_
 #define PHMM_H_
@@ -47,15 +71,15 @@
 extern "C" {
 #endif
 
-#define PHMM_ABI_VERSION 2
+#define PHMM_ABI_VERSION 3
 
 typedef struct phmm_ctx phmm_ctx; /* opaque */
 
 typedef enum {
   PHMM_OK = 0,
-  PHMM_E_INVALID_ARG = -1,  /* NULL pointer, negative count, bad offsets, bad config */
+  PHMM_E_INVALID_ARG = -1,  /* NULL pointer, negative count, bad offsets, bad config, length caps */
   PHMM_E_INVALID_BASE = -2, /* a base outside 'A','C','G','T','N' (uppercase only) */
-  PHMM_E_INVALID_QUAL = -3, /* a quality > 127 */
+  PHMM_E_INVALID_QUAL = -3, /* a quality > 127, or e(qi) + e(qd) > 1 (reading R16) */
   PHMM_E_EMPTY_SEQ = -4,    /* a read or haplotype of length 0 used by a pair */
   PHMM_E_INDEX = -5,        /* a pair's read or haplotype index out of range */
   PHMM_E_CUDA = -6,         /* a CUDA runtime error */
@@ -129,13 +153,24 @@ phmm_status phmm_compute_batch(phmm_ctx* ctx, const phmm_batch* b, double* out_l
 
 /*
  * Device-buffer variant (for torch tensors): every array in *b, dev_out_log10
- * and dev_out_status (optional) are device pointers on the context's device.
- * Work is enqueued on the context stream; the call synchronises that stream
- * once at the end to report input-content errors, so outputs are final when
- * it returns PHMM_OK.
+ * (n_pairs doubles) and dev_out_status (optional, n_pairs bytes) are device
+ * pointers on the context's device. Work is enqueued on the context stream,
+ * which must be ordered after whatever produced the inputs (the Python binding
+ * sets it to torch's current stream with phmm_set_stream before each call);
+ * the call synchronises that stream before returning, so outputs are final
+ * when it returns PHMM_OK.
  */
 phmm_status phmm_compute_batch_dev(phmm_ctx* ctx, const phmm_batch* b, double* dev_out_log10,
                                    uint8_t* dev_out_status);
+
+/*
+ * Make later calls on ctx enqueue their work on `cuda_stream` (a cudaStream_t of
+ * the context's device; NULL = the context's own stream, created on demand).
+ * The caller keeps ownership of the stream and must keep it alive while the
+ * context uses it. Returns PHMM_E_INVALID_ARG for a NULL ctx, PHMM_E_CUDA if a
+ * stream cannot be created.
+ */
+phmm_status phmm_set_stream(phmm_ctx* ctx, void* cuda_stream);
 
 /* Release the context and its device workspace. NULL-safe, idempotent per pointer. */
 void phmm_destroy(phmm_ctx* ctx);

@@ -71,8 +71,27 @@ def build_xsmem(force: bool = False) -> str:
     return build(out=XSMEM_LIB, defines=["PHMM_XCHG_SMEM=1"])
 
 
+SYNTH_LIB = os.path.join(PKG, "libsynth.so")
+SYNTH_SRC = os.path.join(CSRC, "synth_gen.c")
+
+
+def build_synth(force: bool = False) -> str:
+    """libsynth.so: the native synthetic batch generator (plain C, OpenMP; not the method)."""
+    if not force and os.path.exists(SYNTH_LIB) and os.path.getmtime(SYNTH_LIB) >= os.path.getmtime(SYNTH_SRC):
+        return SYNTH_LIB
+    tmp = SYNTH_LIB + f".tmp{os.getpid()}"
+    res = subprocess.run(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-std=c11", "-o", tmp, SYNTH_SRC, "-lm"],
+                         capture_output=True, text=True)
+    if res.returncode != 0:
+        sys.stderr.write(res.stdout + res.stderr)
+        raise RuntimeError("gcc failed building libsynth.so")
+    os.replace(tmp, SYNTH_LIB)
+    return SYNTH_LIB
+
+
 def build_all(force: bool = False, verbose: bool = False) -> None:
     build(force=force, verbose=verbose)
+    build_synth(force=force)
     build_xsmem(force=force)
     build_latency(force=force)
 

@@ -75,7 +75,7 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
         const int64_t m = roff[r + 1] - roff[r], nh = hoff[h + 1] - hoff[h];
         if (m < 1 || nh < 1) {
           e |= ERR_EMPTY;
-        } else if (nh > kMaxHapLen || m > (1 << 20)) {
+        } else if (nh > kMaxHapLen || m > kMaxReadLen) {
           e |= ERR_ARG;
         } else {
           const int nc = ncols_of((int)nh, bucket);
@@ -126,7 +126,7 @@ __global__ void k_item_nblocks(const int32_t* __restrict__ item_read, int64_t n_
   for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = item_read ? item_read[k] : k;
     const int64_t m = r >= 0 ? roff[r + 1] - roff[r] : 0;  // r < 0: unused item
-    item_nb[k] = m >= 1 ? nblocks_of<K>((int)(m > (1 << 20) ? 1 : m)) : 0;
+    item_nb[k] = m >= 1 ? nblocks_of<K>((int)(m > kMaxReadLen ? 1 : m)) : 0;
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) item_nb[n] = 0;
 }

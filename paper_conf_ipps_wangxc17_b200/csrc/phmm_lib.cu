@@ -68,8 +68,8 @@ constexpr int64_t kChunkMinPairs = 65536;
 
 struct phmm_ctx {
   int device = 0;
-  cudaStream_t stream = nullptr;
-  bool own_stream = false;
+  cudaStream_t stream = nullptr;        // the stream calls enqueue on (phmm_set_stream)
+  cudaStream_t owned_stream = nullptr;  // the context's own stream, if it made one
   phmm_precision prec = PHMM_PREC_FP32_RESCUE;
   uint32_t flags = 0;
   int bucket = 4;
@@ -933,8 +933,11 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
   if (cfg->cuda_stream) {
     c->stream = reinterpret_cast<cudaStream_t>(cfg->cuda_stream);
   } else {
-    if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) return fail(PHMM_E_CUDA);
-    c->own_stream = true;
+    if (cudaStreamCreateWithFlags(&c->owned_stream, cudaStreamNonBlocking) != cudaSuccess) {
+      c->owned_stream = nullptr;
+      return fail(PHMM_E_CUDA);
+    }
+    c->stream = c->owned_stream;
   }
   if (cudaMallocHost(&c->host_scal, sizeof(Scalars)) != cudaSuccess) {
     c->host_scal = nullptr;
@@ -971,7 +974,10 @@ void phmm_destroy(phmm_ctx* c) {
   if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
   if (c->host_scal) cudaFreeHost(c->host_scal);
   if (c->host_sizes) cudaFreeHost(c->host_sizes);
-  if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+  if (c->owned_stream) {
+    cudaStreamSynchronize(c->owned_stream);
+    cudaStreamDestroy(c->owned_stream);
+  }
   cudaGetLastError();
   delete c;
 }
@@ -979,6 +985,25 @@ void phmm_destroy(phmm_ctx* c) {
 phmm_status phmm_get_stats(const phmm_ctx* c, phmm_stats* out) {
   if (!c || !out) return PHMM_E_INVALID_ARG;
   *out = c->st;
+  return PHMM_OK;
+}
+
+phmm_status phmm_set_stream(phmm_ctx* c, void* stream) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  if (cudaSetDevice(c->device) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  cudaStream_t s = stream ? reinterpret_cast<cudaStream_t>(stream) : c->owned_stream;
+  if (!s) {  // created on a caller's stream: make a private one for the NULL case
+    if (cudaStreamCreateWithFlags(&c->owned_stream, cudaStreamNonBlocking) != cudaSuccess) {
+      cudaGetLastError();
+      c->owned_stream = nullptr;
+      return PHMM_E_CUDA;
+    }
+    s = c->owned_stream;
+  }
+  c->stream = s;
   return PHMM_OK;
 }
 
@@ -994,13 +1019,27 @@ phmm_status phmm_compute_batch_dev(phmm_ctx* c, const phmm_batch* b, double* dev
   DevBatch d{b->read_bases, b->base_quals, b->ins_quals, b->del_quals, b->gcp_quals, b->hap_bases,
              b->read_offsets, b->hap_offsets, b->pairs, b->n_reads, b->n_haps, b->n_pairs,
              b->total_read_bases, b->total_hap_bases};
+  // results go to context scratch first and reach the caller's buffers only after the
+  // whole path (FP32 pass and FP64 rescue) succeeded: outputs stay untouched on error
+  double* out = nullptr;
+  uint8_t* status = nullptr;
+  if (b->n_pairs > 0) {
+    ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
+    if (dev_status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
+  }
   ev_record(c, EV_START);
   ev_record(c, EV_H2D);
-  phmm_status st = compute_dev(c, d, dev_out, dev_status);
+  phmm_status st = compute_dev(c, d, out, status);
   if (st != PHMM_OK) {
     cudaStreamSynchronize(c->stream);
     cudaGetLastError();
     return st;
+  }
+  if (b->n_pairs > 0) {
+    CUDA_TRY(cudaMemcpyAsync(dev_out, out, sizeof(double) * (size_t)b->n_pairs, cudaMemcpyDeviceToDevice,
+                             c->stream));
+    if (dev_status)
+      CUDA_TRY(cudaMemcpyAsync(dev_status, status, (size_t)b->n_pairs, cudaMemcpyDeviceToDevice, c->stream));
   }
   ev_record(c, EV_END);
   if (cudaStreamSynchronize(c->stream) != cudaSuccess) {

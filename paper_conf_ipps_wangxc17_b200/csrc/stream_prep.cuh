@@ -106,8 +106,11 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
     const int64_t r = item_read ? item_read[it] : it;
     if (r < 0) continue;  // unused item (rescue pass, past the distinct reads)
     const int64_t r0 = roff[r];
-    const int m = (int)(roff[r + 1] - r0);
-    if (m < 1) continue;
+    const int64_t m64 = roff[r + 1] - r0;
+    // reads longer than kMaxReadLen bases have a 1-block reservation (k_item_nblocks) and no table:
+    // a pair that uses one is rejected by k_pair_bins, an unused one must not be written
+    if (m64 < 1 || m64 > kMaxReadLen) continue;
+    const int m = (int)m64;
     const int nb = nblocks_of<K>(m);
     const int f = nb * K - (m + 2);  // >= 1 Z rows
     TBlock<T>* __restrict__ Tb = tab + item_tab_off[it];

@@ -84,8 +84,8 @@ SW_OPS = "MID"
 
 # every symbol include/phmm.h declares (checked by tests/test_abi.py)
 EXPORTED_SYMBOLS = ("phmm_create", "phmm_compute_batch", "phmm_compute_batch_dev", "phmm_destroy",
-                    "phmm_status_string", "phmm_get_stats", "phmm_abi_version", "phmm_sw_align_batch",
-                    "phmm_sw_align_batch_dev")
+                    "phmm_status_string", "phmm_get_stats", "phmm_abi_version", "phmm_set_stream",
+                    "phmm_sw_align_batch", "phmm_sw_align_batch_dev")
 
 _lib = None
 
@@ -113,6 +113,8 @@ def load_library(path: str = LIB_PATH):
     L.phmm_get_stats.restype = ctypes.c_int
     L.phmm_abi_version.argtypes = []
     L.phmm_abi_version.restype = ctypes.c_int
+    L.phmm_set_stream.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
+    L.phmm_set_stream.restype = ctypes.c_int
     for f in (L.phmm_sw_align_batch, L.phmm_sw_align_batch_dev):
         f.argtypes = [ctypes.c_void_p, ctypes.POINTER(_SwBatch), ctypes.POINTER(_SwParams), ctypes.c_void_p,
                       ctypes.c_void_p]
@@ -193,6 +195,27 @@ class DeviceBatch:
                            pairs=t(np.asarray(b.pairs, dtype=np.int32).reshape(-1, 2), np.int32),
                            total_read_bases=int(b.read_offsets[-1]), total_hap_bases=int(b.hap_offsets[-1]))
 
+    _DTYPES = dict(read_bases="uint8", base_quals="uint8", ins_quals="uint8", del_quals="uint8",
+                   gcp_quals="uint8", read_offsets="int64", hap_bases="uint8", hap_offsets="int64", pairs="int32")
+
+    def check(self) -> None:
+        """Every tensor contiguous, of its ABI dtype and on the pairs' device; sizes
+        consistent (the library validates the contents)."""
+        dev = self.pairs.device
+        for k, dt in self._DTYPES.items():
+            x = getattr(self, k)
+            if str(x.dtype) != "torch." + dt or not x.is_contiguous() or x.device != dev:
+                raise ValueError(f"DeviceBatch.{k}: need a contiguous {dt} tensor on {dev}, got "
+                                 f"{x.dtype} on {x.device} (contiguous={x.is_contiguous()})")
+        if self.pairs.dim() != 2 or self.pairs.shape[1] != 2:
+            raise ValueError("DeviceBatch.pairs must be (n_pairs, 2)")
+        nr = int(self.read_bases.numel())
+        for k in ("base_quals", "ins_quals", "del_quals", "gcp_quals"):
+            if int(getattr(self, k).numel()) != nr:
+                raise ValueError(f"DeviceBatch.{k} must have as many bytes as read_bases")
+        if nr != int(self.total_read_bases) or int(self.hap_bases.numel()) != int(self.total_hap_bases):
+            raise ValueError("DeviceBatch.total_read_bases / total_hap_bases disagree with the tensors")
+
     def struct(self) -> _Batch:
         s = _Batch()
         for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets",
@@ -205,6 +228,12 @@ class DeviceBatch:
         s.total_read_bases = int(self.total_read_bases)
         s.total_hap_bases = int(self.total_hap_bases)
         return s
+
+
+def _check_out(t, dtype, n: int, dev, name: str) -> None:
+    if t.dtype != dtype or not t.is_contiguous() or t.device != dev or t.numel() < n:
+        raise ValueError(f"{name}: need a contiguous {dtype} tensor of >= {n} elements on {dev}, got "
+                         f"{t.dtype}, {t.numel()} elements on {t.device} (contiguous={t.is_contiguous()})")
 
 
 class PairHMM:
@@ -227,6 +256,10 @@ class PairHMM:
         self._L = L
         self.device = int(device)
         self.precision = precision
+        # without an explicit stream the device variant follows torch's current stream
+        # (set before every call), so it is ordered after the ops that produced its inputs
+        self._follow_torch = stream is None
+        self._cur_stream = None
 
     # ------------------------------------------------------------ host API
     def compute_batch(self, batch, out: Optional[np.ndarray] = None, status: Optional[np.ndarray] = None,
@@ -252,16 +285,37 @@ class PairHMM:
                                               ctypes.cast(status_ptr, _u8p) if status_ptr else None))
 
     # ------------------------------------------------------------ device API
+    def set_stream(self, stream) -> None:
+        """``phmm_set_stream``: enqueue later calls on ``stream`` (an int cudaStream_t,
+        a torch.cuda.Stream, or None for the context's own stream)."""
+        handle = getattr(stream, "cuda_stream", stream)
+        rc = self._L.phmm_set_stream(self._h, int(handle) if handle else None)
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_set_stream")
+        self._cur_stream = handle
+
     def compute_batch_dev(self, db: DeviceBatch, out=None, status=None, want_status: bool = True):
-        """``phmm_compute_batch_dev``: torch CUDA tensors in and out."""
+        """``phmm_compute_batch_dev``: torch CUDA tensors in and out. Unless the context was
+        created on an explicit stream, the call runs on torch's current stream of the
+        batch's device."""
         import torch
 
         n = db.n_pairs
         dev = db.pairs.device
+        if dev.type != "cuda" or dev.index != self.device:
+            raise ValueError(f"batch on {dev}, context on cuda:{self.device}")
+        db.check()
         if out is None:
             out = torch.empty(n, dtype=torch.float64, device=dev)
         if status is None and want_status:
             status = torch.empty(n, dtype=torch.uint8, device=dev)
+        _check_out(out, torch.float64, n, dev, "out")
+        if status is not None:
+            _check_out(status, torch.uint8, n, dev, "status")
+        if self._follow_torch:
+            cur = torch.cuda.current_stream(dev).cuda_stream
+            if cur != self._cur_stream:
+                self.set_stream(cur)
         s = db.struct()
         rc = self._L.phmm_compute_batch_dev(self._h, ctypes.byref(s), out.data_ptr() if n else None,
                                             status.data_ptr() if (status is not None and n) else None)
@@ -312,6 +366,10 @@ class PairHMM:
         dev = T["tasks"].device
         if res is None:
             res = torch.empty((n, 6), dtype=torch.int32, device=dev)
+        if self._follow_torch:
+            cur = torch.cuda.current_stream(dev).cuda_stream
+            if cur != self._cur_stream:
+                self.set_stream(cur)
         p = _SwParams(*params)
         rc = self._L.phmm_sw_align_batch_dev(self._h, ctypes.byref(s), ctypes.byref(p), res.data_ptr(),
                                              ops.data_ptr())

@@ -94,3 +94,24 @@ def test_sw_entry_points_reject_null_without_gpu(lib):
     """The Smith-Waterman calls validate their arguments before touching the device."""
     assert lib.phmm_sw_align_batch(None, None, None, None, None) == -1
     assert lib.phmm_sw_align_batch_dev(None, None, None, None, None) == -1
+
+
+def test_device_batch_checks_dtypes_and_sizes_on_cpu_tensors():
+    """DeviceBatch.check (the binding's marshalling guard) on CPU tensors: wrong dtype,
+    non-contiguous or mismatched sizes raise ValueError before any library call."""
+    import torch
+
+    b = synth.random_pairs_batch(1, 5)
+    db = phmm.DeviceBatch.from_host(b, device="cpu")
+    db.check()
+    bad = phmm.DeviceBatch(**{**db.__dict__, "pairs": db.pairs.to(torch.int64)})
+    with pytest.raises(ValueError):
+        bad.check()
+    bad = phmm.DeviceBatch(**{**db.__dict__, "ins_quals": db.ins_quals[:-1]})
+    with pytest.raises(ValueError):
+        bad.check()
+    bad = phmm.DeviceBatch(**{**db.__dict__, "read_offsets": db.read_offsets.repeat(2)[::2]})
+    with pytest.raises(ValueError):
+        bad.check()
+    with pytest.raises(ValueError):
+        phmm._check_out(torch.empty(3, dtype=torch.float32), torch.float64, 3, torch.device("cpu"), "out")

@@ -370,3 +370,110 @@ def test_fully_ragged_one_batch(ctx32, ctx64, seed):
     _check(got32, ref, "fp32")
     assert set(np.unique(st)) <= {0, 1, 2}
     _check(ctx64.compute_batch(b)[0], ref, "fp64")
+
+
+@pytest.mark.parametrize("seed,iq", [(51, (60, 127)), (52, (60, 127)), (53, (4, 127))])
+def test_high_indel_and_gcp_qualities_near_rescue_threshold(ctx32, ctx64, seed, iq):
+    """Indel and gap-continuation qualities drawn per base from Q60-127 (or Q4-127): the
+    rescaled 5-op form stores M^ = a_i M with a_i = k_i zeta_i down to 10^-12.7, so these
+    push the FP32 pass's values toward the subnormal range. Reads with 8-22 substitutions
+    against their own haplotype put log10 P on both sides of the rescue threshold (-64.1);
+    the pairs the FP32 pass keeps must be within 1e-3 like every other pair, and the FP64
+    mode within 1e-9 relative."""
+    b = synth.near_threshold_batch(seed, 400, indel_qual_range=iq, gcp_range=iq)
+    ref = oracle.batch_log10(b)
+    near = (ref > -64.1236) & (ref < -58.0)
+    assert near.sum() >= 20 and (ref < -64.2).sum() >= 50
+    got, st = ctx32.compute_batch(b)
+    _check(got, ref, "fp32")
+    # the near-threshold pairs are the FP32 pass's own results (scaled sum >= 1e-28)
+    assert np.all(st[near & (ref > -63.5)] == 0)
+    _check(ctx64.compute_batch(b)[0], ref, "fp64")
+
+
+@pytest.mark.parametrize("qi,qd", [(3, 3), (0, 10), (2, 3), (10, 0)])
+def test_r16_non_distribution_transitions_rejected(ctx32, ctx64, qi, qd):
+    """DESIGN.md reading R16: e(qi) + e(qd) > 1 (only possible with qi or qd <= 3) makes the
+    transitions out of M exceed 1; the call returns PHMM_E_INVALID_QUAL and leaves the
+    outputs untouched, in both precisions."""
+    b = synth.random_pairs_batch(3, 10, indel_qual_range=(20, 40))
+    b.ins_quals = b.ins_quals.copy()
+    b.del_quals = b.del_quals.copy()
+    k = int(b.read_offsets[4]) + 1 if b.read_offsets[5] - b.read_offsets[4] > 1 else int(b.read_offsets[4])
+    b.ins_quals[k] = qi
+    b.del_quals[k] = qd
+    for ctx in (ctx32, ctx64):
+        out, st = _sentinel(b.n_pairs)
+        with pytest.raises(phmm.PhmmError) as ei:
+            ctx.compute_batch(b, out=out, status=st)
+        assert ei.value.code == -3
+        assert np.all(out == 12345.0) and np.all(st == 77)
+    # qi = qd = 4: e(4) + e(4) = 0.796 <= 1 is accepted
+    b.ins_quals[k] = 4
+    b.del_quals[k] = 4
+    _check(ctx32.compute_batch(b)[0], oracle.batch_log10(b), "fp32")
+
+
+def test_unused_read_longer_than_cap_is_harmless(ctx32, ctx64):
+    """A read of 2^20 + 1 bases that no pair uses (reads longer than 2^20 are only an error
+    when a pair uses them, include/phmm.h): the per-read table pass must not write past its
+    1-block reservation into other reads' tables. Every other pair must match
+    the oracle; a pair that does use the long read returns PHMM_E_INVALID_ARG."""
+    small = synth.random_pairs_batch(61, 40, m_range=(1, 120), n_range=(1, 200))
+    L = (1 << 20) + 1
+    rng = np.random.default_rng(5)
+    longb = synth.Batch(read_bases=np.frombuffer(b"ACGT", np.uint8)[rng.integers(0, 4, L)].copy(),
+                        base_quals=np.full(L, 30, np.uint8), ins_quals=np.full(L, 45, np.uint8),
+                        del_quals=np.full(L, 45, np.uint8), gcp_quals=np.full(L, 10, np.uint8),
+                        read_offsets=np.array([0, L], np.int64),
+                        hap_bases=np.frombuffer(b"ACGT" * 10, np.uint8).copy(),
+                        hap_offsets=np.array([0, 40], np.int64), pairs=np.array([[0, 0]], np.int32))
+    # the long read sits in the middle of the read array: its table slot precedes others
+    b = synth.concat_batches([synth.random_pairs_batch(62, 20, m_range=(1, 120)), longb, small])
+    used = np.ones(b.n_pairs, bool)
+    used[20] = False  # the long read's own pair
+    ok = b.subset(np.nonzero(used)[0])
+    ref = oracle.batch_log10(ok)
+    _check(ctx32.compute_batch(ok)[0], ref, "fp32")
+    _check(ctx64.compute_batch(ok)[0], ref, "fp64")
+    out, st = _sentinel(b.n_pairs)
+    with pytest.raises(phmm.PhmmError) as ei:
+        ctx32.compute_batch(b, out=out, status=st)
+    assert ei.value.code == -1
+    assert np.all(out == 12345.0)
+
+
+def test_dev_variant_follows_torch_stream_and_leaves_outputs_on_error(ctx32):
+    """compute_batch_dev on a context without an explicit stream runs on torch's current
+    stream (phmm_set_stream): inputs produced by a still-running op on that stream are seen
+    complete. On an input error the device outputs keep their contents (results reach them
+    only after the whole path succeeded)."""
+    import torch
+
+    b = synth.config_batch("C2", n_regions=4)
+    ref, _ = ctx32.compute_batch(b)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+        # delay the stream, then overwrite the pairs with the real ones: a library call that
+        # did not wait for this stream would read the zeros
+        real = db.pairs.clone()
+        db.pairs.zero_()
+        torch.cuda._sleep(200_000_000)
+        db.pairs.copy_(real)
+        out, st = ctx32.compute_batch_dev(db)
+        got = out.cpu().numpy()
+    assert np.array_equal(got, ref)
+    with torch.cuda.stream(s):
+        bad = phmm.DeviceBatch.from_host(b, device="cuda:0")
+        bad.read_bases[7] = ord("x")
+        o = torch.full((b.n_pairs,), 12345.0, dtype=torch.float64, device="cuda:0")
+        t = torch.full((b.n_pairs,), 77, dtype=torch.uint8, device="cuda:0")
+        with pytest.raises(phmm.PhmmError) as ei:
+            ctx32.compute_batch_dev(bad, out=o, status=t)
+        assert ei.value.code == -2
+        assert bool(torch.all(o == 12345.0)) and bool(torch.all(t == 77))
+        with pytest.raises(ValueError):
+            ctx32.compute_batch_dev(db, out=torch.empty(b.n_pairs, dtype=torch.float32, device="cuda:0"))
+        with pytest.raises(ValueError):
+            ctx32.compute_batch_dev(db, out=torch.empty(b.n_pairs - 1, dtype=torch.float64, device="cuda:0"))

@@ -155,6 +155,70 @@ def test_p4_hand_values(read, hap, expected):
     assert abs(lp - expected) < 1e-13 * max(1.0, abs(expected))
 
 
+GOLDEN_ROWS = os.path.join(os.path.dirname(__file__), "golden", "hand_values_rows.tsv")
+
+
+def _golden_rows():
+    rows = []
+    with open(GOLDEN_ROWS) as f:
+        for line in f:
+            if line.startswith("#") or line.startswith("read\t") or not line.strip():
+                continue
+            read, hap, q, qi, qd, qg, val, _ = line.rstrip("\n").split("\t")
+            ints = lambda s: [int(x) for x in s.split(",")]
+            rows.append((read, hap, ints(q), ints(qi), ints(qd), ints(qg), float(val)))
+    return rows
+
+
+@pytest.mark.parametrize("read,hap,q,qi,qd,qg,expected", _golden_rows())
+def test_p4_hand_values_per_row_qualities(read, hap, q, qi, qd, qg, expected):
+    """qi != qd and per-row qualities: pins which quality feeds M->I and M->D (R2) and
+    that a transition uses its destination row's qualities (R3)."""
+    lp = core.phred_log10(read, q, qi, qd, qg, hap)
+    assert abs(lp - expected) < 1e-13 * max(1.0, abs(expected)), (lp, expected)
+    # the same inputs with qi and qd swapped must NOT give the hand value (the pin is not
+    # symmetric in the two gap-open qualities)
+    swapped = core.phred_log10(read, q, qd, qi, qg, hap)
+    assert abs(swapped - expected) > 0.1, (swapped, expected)
+
+
+@pytest.mark.parametrize("seed", range(20))
+def test_insertion_quality_governs_extra_read_base(seed):
+    """A 2-base read against a 1-base haplotype can only be explained by an insertion
+    after the first base (column 0 of row 2 is 0): P = e(qi_2) * (1 - e(qg_1)) * pm_1,
+    exactly, for ANY deletion qualities (R2: delta = e(qi) is the M->I transition, R3:
+    the destination row's qi)."""
+    rng = random.Random(seed)
+    q = [rng.randint(6, 60) for _ in range(2)]
+    qi = [rng.randint(4, 60) for _ in range(2)]
+    qg = [rng.randint(4, 60) for _ in range(2)]
+    e = lambda x: 10.0 ** (-x / 10.0)
+    want = math.log10(e(qi[1]) * (1.0 - e(qg[0])) * (1.0 - e(q[0])))
+    vals = set()
+    for _ in range(4):
+        qd = [rng.randint(4, 127) for _ in range(2)]
+        lp = core.phred_log10("AA", q, qi, qd, qg, "A")
+        assert abs(lp - want) < 1e-13 * abs(want), (lp, want)
+        vals.add(lp)
+    assert len(vals) == 1  # bitwise independent of qd
+
+
+@pytest.mark.parametrize("qd1", [15, 20, 25, 30])
+def test_deletion_quality_governs_missing_hap_base(qd1):
+    """Read "AC" against haplotype "AGC" at Q80 base qualities and a tiny insertion rate:
+    every path but the deletion of the haplotype's G (M(1,1) -> D(1,2) -> M(2,3)) carries a
+    mismatch (px = 3.3e-9) or an insertion (1e-9), so P is proportional to zeta_1 = e(qd_1),
+    the deletion quality of the row the deletion happens in (R2, R3): P(qd1) / P(qd1 + 10)
+    = 10 to 1e-3."""
+    q, qi, qg = [80, 80], [90, 90], [10, 10]
+    a = core.phred_log10("AC", q, qi, [qd1, 40], qg, "AGC")
+    b = core.phred_log10("AC", q, qi, [qd1 + 10, 40], qg, "AGC")
+    assert abs((a - b) - 1.0) < 1e-3, a - b
+    # the row-2 deletion quality barely matters (a D move in row 2 ends in D, not counted)
+    c = core.phred_log10("AC", q, qi, [qd1, 10], qg, "AGC")
+    assert abs(c - a) < 1e-4
+
+
 def test_p4_q0_zero_probability():
     """Q0 base quality gives pm = 1 - 10^0 = 0: a 1-base read that matches a
     1-base haplotype has P = 0 exactly (log10 = -inf), SURVEY §8c P7."""
