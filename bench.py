@@ -8,11 +8,15 @@ Contract (see the task statement / DESIGN.md §7):
 A "step" is one pass of the whole hot path (validate, per-read tables,
 length binning, FP32 wavefront, finalize, FP64 rescue) over one batch of
 synthetic input: ``phmm_compute_batch_dev`` on
-device-resident inputs for ``value``; ``phmm_compute_batch`` from pinned host
-buffers (H2D + compute + D2H of every result) for ``e2e``. For N > 1 each rank
-processes its own shard of regions (weak scaling, regions addressed by
-(seed, region id)) and the step ends with the NCCL all-gather of the results
-(the path's one exchange step).
+device-resident inputs for ``value``; ``phmm_compute_batch`` from pinned and
+from pageable host buffers (H2D + compute + D2H of every result) for ``e2e``.
+Each rank generates its own regions from (seed, region id) -- no input moves --
+and for N > 1 the step ends with one NCCL all-gather of the results plus their
+global pair ids (the path's one exchange step; parallel.py):
+  * C5 (default --scaling strong): the fixed 2^26-pair job is split into
+    whole-region ranges balanced by cells; ``result_sha256`` (the job's results
+    in global pair order) is the same for every GPU count;
+  * C2..C4 (default --scaling weak): every rank runs the config's region count.
 
 metric = GCUPS = sum over pairs of m*N / seconds / 1e9 (PAPER.md L22@1416:
 the three M/I/D updates of one cell count as one cell update).
@@ -21,6 +25,7 @@ from __future__ import annotations
 
 import argparse
 import glob
+import hashlib
 import json
 import os
 import statistics
@@ -47,9 +52,10 @@ WORKLOADS = {
           "2% decoy reads, FP32 + FP64 underflow rescue",
     "C3": "C3: HaplotypeCaller-shaped regions, 250 bp reads x 4-8 haplotypes of 250-500 bp",
     "C4": "C4: long-read stress, 1000 bp reads x 1500 bp haplotypes",
-    "C5": "C5-shaped shard: mixed 100-250 bp reads, N ~ U{m..2m}",
+    "C5": "C5: 64M pairs (262144 regions x 32 reads x 8 haplotypes), mixed 100-250 bp reads, N ~ U{m..2m}",
 }
-DEFAULT_REGIONS = {"C2": 8192, "C3": 4096, "C4": 256, "C5": 8192}
+# regions per rank (weak split) or of the whole job (strong split: C5, the full 2^26 pairs)
+DEFAULT_REGIONS = {"C2": 8192, "C3": 4096, "C4": 256, "C5": 262144}
 # The paper's PairHMM numbers: other hardware and its HCC1954 dataset,
 # context only (vs_baseline stays null).
 PAPER_CONTEXT = {
@@ -220,18 +226,124 @@ def cpu_baseline(args, batch):
             "sample_1core": f"first {n1} pairs of that sample ({c1} cells, {dt1:.1f} s, 1 thread)"}, sample, ref
 
 
+def _e2e_leg(args, ctx, batch, ws, flush, stream, gloo, n_slot, pair_start, pinned: bool):
+    """Same metric through the host-buffer C-ABI call: H2D of the step's inputs, the whole
+    path, D2H of the results, every step (wall clock around the synchronous call, max over
+    ranks). pinned: inputs and outputs in page-locked host memory; otherwise plain numpy
+    (pageable) arrays, which the library stages through its own pinned buffers. N > 1: the
+    host results of every rank are gathered (gloo, no re-upload to the GPU)."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_wangxc17_b200 import phmm
+
+    keys = ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets", "hap_bases",
+            "hap_offsets", "pairs")
+    host = {}
+    for k in keys:
+        a = np.ascontiguousarray(getattr(batch, k))
+        host[k] = torch.from_numpy(a).pin_memory() if pinned else torch.from_numpy(a.copy())
+    s = phmm._Batch()
+    for k, t in host.items():
+        setattr(s, k, t.data_ptr())
+    s.n_reads, s.n_haps, s.n_pairs = batch.n_reads, batch.n_haps, batch.n_pairs
+    s.total_read_bases = int(batch.read_offsets[-1])
+    s.total_hap_bases = int(batch.hap_offsets[-1])
+    n = batch.n_pairs
+    hslot = torch.full((n_slot + 2,), float("nan"), dtype=torch.float64)
+    if pinned:
+        hslot = hslot.pin_memory()
+    hslot[0], hslot[1] = float(pair_start), float(n)
+    hout = hslot[2:2 + n]
+    hst = torch.empty(n, dtype=torch.uint8)
+    if pinned:
+        hst = hst.pin_memory()
+    hg = torch.empty(ws * (n_slot + 2), dtype=torch.float64) if ws > 1 else None
+    h2d = int(sum(t.numel() * t.element_size() for t in host.values()))
+    d2h = n * (8 + 1)
+
+    def one():
+        rc = ctx.compute_batch_raw(s, hout.data_ptr(), hst.data_ptr())
+        assert rc == 0, rc
+        if ws > 1:
+            dist.all_gather_into_tensor(hg, hslot, group=gloo)
+
+    for _ in range(max(1, args.warmup)):
+        one()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e_ms = []
+    for i in range(args.steps):
+        with torch.cuda.stream(stream):
+            flush.fill_(i & 0xff)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        one()
+        e_ms.append((time.perf_counter() - t0) * 1e3)
+    t_e = sum(e_ms) / 1e3
+    if ws > 1:
+        tt = torch.tensor([t_e], dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX, group=gloo)
+        t_e = float(tt.item())
+    return {"unit": "GCUPS", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+            "ms_per_step": 1e3 * t_e / args.steps, "seconds": t_e,
+            "host_buffers": "pinned (page-locked)" if pinned else "pageable numpy (library-staged)"}
+
+
+def run_extra(ctx, workload, n_regions, args, stream, flush):
+    """A secondary workload on the same context (the HaplotypeCaller-shaped C3 beside C2):
+    device-resident GCUPS, wavefront and rescue time."""
+    import torch
+
+    from paper_conf_ipps_wangxc17_b200 import phmm, synth
+
+    b = synth.config_batch(workload, n_regions=n_regions)
+    with torch.cuda.stream(stream):
+        db = phmm.DeviceBatch.from_host(b, device=torch.cuda.current_device())
+        out = torch.empty(b.n_pairs, dtype=torch.float64, device=db.pairs.device)
+        st = torch.empty(b.n_pairs, dtype=torch.uint8, device=db.pairs.device)
+    for _ in range(2):
+        ctx.compute_batch_dev(db, out=out, status=st)
+    torch.cuda.synchronize()
+    ms, wf, rs = [], [], []
+    for i in range(max(3, args.steps // 2)):
+        with torch.cuda.stream(stream):
+            flush.fill_(i & 0xff)
+        a, z = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        ctx.compute_batch_dev(db, out=out, status=st)
+        z.record(stream)
+        z.synchronize()
+        ms.append(a.elapsed_time(z))
+        x = ctx.stats()
+        wf.append(x["ms_wavefront"])
+        rs.append(x["ms_rescue"])
+    cells = b.cells()
+    st_h = st.cpu().numpy()
+    return {"workload": WORKLOADS[workload], "regions": n_regions, "pairs": b.n_pairs, "cells": cells,
+            "value": cells / (np.mean(ms) / 1e3) / 1e9, "unit": "GCUPS", "ms_per_step": float(np.mean(ms)),
+            "wavefront_ms": float(np.mean(wf)), "kernel_gcups": cells / (np.mean(wf) / 1e3) / 1e9,
+            "rescue_ms": float(np.mean(rs)), "rescued_pairs": int(np.sum(st_h >= 1))}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--workload", default="C2", choices=sorted(WORKLOADS))
-    ap.add_argument("--regions", type=int, default=None, help="regions per rank (default: the config's)")
+    ap.add_argument("--regions", type=int, default=None,
+                    help="strong: the job's regions; weak: regions per rank (default: the config's)")
+    ap.add_argument("--scaling", default=None, choices=["weak", "strong"],
+                    help="N > 1 split (default: strong for C5 -- the fixed 2^26-pair job split by cells "
+                         "(SURVEY §8e) -- weak, a fixed shard per rank, otherwise)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-regions", type=int, default=16, help="regions per step for --impl reference")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-extra", action="store_true", help="skip the secondary C3 object")
     ap.add_argument("--profile-steps", action="store_true", help="short run for ncu (no clocks/cpu)")
     args = ap.parse_args()
 
@@ -246,35 +358,42 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    gloo = None
     if ws > 1:
         dist.init_process_group("nccl", device_id=dev)
+        gloo = dist.new_group(backend="gloo")  # host-side reductions / the e2e legs' host gather
 
+    scaling = args.scaling or ("strong" if args.workload == "C5" else "weak")
     n_regions = args.regions or DEFAULT_REGIONS[args.workload]
-    batch = synth.config_batch(args.workload, n_regions=n_regions, region_start=rank * n_regions)
-    cells = batch.cells()
+    r0, r1, pair_start, total_pairs, total_cells, cells = parallel.shard(args.workload, rank, ws, scaling,
+                                                                         n_regions)
+    batch = synth.config_batch(args.workload, n_regions=r1 - r0, region_start=r0)
+    assert batch.cells() == cells
     n_pairs = batch.n_pairs
 
     stream = torch.cuda.Stream(device=dev)
     ctx = phmm.PairHMM(device=local, precision="fp32", stream=stream.cuda_stream, timing=True)
-    # the result gather (parallel.py): every rank's slot is padded to the largest shard
+    # the result gather (parallel.py): every rank's slot = [pair_start, count, results, pad]
     n_slot = n_pairs
     if ws > 1:
-        nn = torch.tensor([n_pairs], dtype=torch.int64, device=dev)
-        dist.all_reduce(nn, op=dist.ReduceOp.MAX)
+        nn = torch.tensor([n_pairs], dtype=torch.int64)
+        dist.all_reduce(nn, op=dist.ReduceOp.MAX, group=gloo)
         n_slot = int(nn.item())
     with torch.cuda.stream(stream):
         db = phmm.DeviceBatch.from_host(batch, device=dev)
-        out_slot = torch.full((n_slot,), float("nan"), dtype=torch.float64, device=dev)
-        out = out_slot[:n_pairs]
+        slot = parallel.pack_slot(torch.empty(0, dtype=torch.float64, device=dev), pair_start, n_slot)
+        slot[1] = float(n_pairs)
+        out = slot[2:2 + n_pairs]  # the library writes its results straight into the slot
         status = torch.empty(n_pairs, dtype=torch.uint8, device=dev)
         flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     torch.cuda.synchronize()
+    gathered = [None]
 
     def step():
         ctx.compute_batch_dev(db, out=out, status=status)
         if ws > 1:
             with torch.cuda.stream(stream):
-                parallel.gather_results(out_slot, ws)
+                gathered[0] = parallel.gather_slots(slot, ws)
 
     for _ in range(max(args.warmup, 0)):
         step()
@@ -307,64 +426,35 @@ def main():
     clocks = clk.stop() if not args.profile_steps else {}
     t_rank = sum(step_ms) / 1e3
     if ws > 1:
-        tt = torch.tensor([t_rank], dtype=torch.float64, device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        tt = torch.tensor([t_rank], dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX, group=gloo)
         t_max = float(tt.item())
-        cc = torch.tensor([float(cells)], dtype=torch.float64, device=dev)
-        dist.all_reduce(cc, op=dist.ReduceOp.SUM)
-        cells_all = float(cc.item())
     else:
-        t_max, cells_all = t_rank, float(cells)
-    value = cells_all * args.steps / t_max / 1e9
+        t_max = t_rank
+    # the whole job's cells (strong: the fixed region set; weak: every rank's shard)
+    job_cells = total_cells
+    value = job_cells * args.steps / t_max / 1e9
 
-    # ---- e2e: host API from pinned host buffers (H2D + compute + D2H each step)
+    # the job's results in global pair order (rank 0), and their hash: identical for every GPU
+    # count under the strong split (every pair's arithmetic is independent of its shard)
+    result_hash = None
+    if rank == 0:
+        g = gathered[0].cpu().numpy() if ws > 1 else slot.view(1, -1).cpu().numpy()
+        glob = parallel.unpack_global(g, total_pairs)
+        result_hash = hashlib.sha256(glob.tobytes()).hexdigest()
+
+    # ---- e2e: host API (H2D + compute + D2H each step), pinned and pageable host buffers
     e2e = None
     if not args.no_e2e and not args.profile_steps:
-        pinned = {}
-        for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets", "hap_bases",
-                  "hap_offsets", "pairs"):
-            a = np.ascontiguousarray(getattr(batch, k))
-            t = torch.from_numpy(a).pin_memory()
-            pinned[k] = t
-        s = phmm._Batch()
-        for k, t in pinned.items():
-            setattr(s, k, t.data_ptr())
-        s.n_reads = batch.n_reads
-        s.n_haps = batch.n_haps
-        s.n_pairs = n_pairs
-        s.total_read_bases = int(batch.read_offsets[-1])
-        s.total_hap_bases = int(batch.hap_offsets[-1])
-        hout = torch.empty(n_pairs, dtype=torch.float64).pin_memory()
-        hst = torch.empty(n_pairs, dtype=torch.uint8).pin_memory()
-        h2d = int(sum(t.numel() * t.element_size() for t in pinned.values()))
-        d2h = n_pairs * (8 + 1)
-        for _ in range(max(1, args.warmup)):
-            rc = ctx.compute_batch_raw(s, hout.data_ptr(), hst.data_ptr())
-            assert rc == 0, rc
-        if ws > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-        e_ms = []
-        for i in range(args.steps):
-            with torch.cuda.stream(stream):
-                flush.fill_(i & 0xff)
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            rc = ctx.compute_batch_raw(s, hout.data_ptr(), hst.data_ptr())
-            if ws > 1:
-                out_slot[:n_pairs].copy_(torch.from_numpy(hout.numpy()).to(dev, non_blocking=False))
-                parallel.gather_results(out_slot, ws)
-                torch.cuda.synchronize()
-            e_ms.append((time.perf_counter() - t0) * 1e3)
-            assert rc == 0, rc
-        t_e = sum(e_ms) / 1e3
-        if ws > 1:
-            tt = torch.tensor([t_e], dtype=torch.float64, device=dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            t_e = float(tt.item())
-        e2e = {"value": cells_all * args.steps / t_e / 1e9, "unit": "GCUPS", "h2d_bytes_per_step": h2d,
-               "d2h_bytes_per_step": d2h, "ms_per_step": 1e3 * t_e / args.steps,
-               "timing": "host wall clock around phmm_compute_batch (synchronous C-ABI call)"}
+        e_pin = _e2e_leg(args, ctx, batch, ws, flush, stream, gloo, n_slot, pair_start, pinned=True)
+        e_pag = _e2e_leg(args, ctx, batch, ws, flush, stream, gloo, n_slot, pair_start, pinned=False)
+        e2e = {"value": job_cells * args.steps / e_pin["seconds"] / 1e9, "unit": "GCUPS",
+               "h2d_bytes_per_step": e_pin["h2d_bytes_per_step"], "d2h_bytes_per_step": e_pin["d2h_bytes_per_step"],
+               "ms_per_step": e_pin["ms_per_step"], "host_buffers": e_pin["host_buffers"],
+               "timing": "host wall clock around phmm_compute_batch (synchronous C-ABI call), max over ranks",
+               "pageable": {"value": job_cells * args.steps / e_pag["seconds"] / 1e9, "unit": "GCUPS",
+                            "ms_per_step": e_pag["ms_per_step"], "host_buffers": e_pag["host_buffers"]}}
+        e2e["pageable_over_pinned"] = e2e["pageable"]["value"] / e2e["value"]
 
     # ---- roofline of the dominant kernel (the FP32 wavefront), live CUDA events
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
@@ -409,20 +499,28 @@ def main():
         fin = np.isfinite(ref)
         cpu["parity_max_abs_log10"] = float(np.max(np.abs(got[fin] - ref[fin]))) if fin.any() else 0.0
 
+    extra = None
+    if ws == 1 and not args.no_extra and not args.profile_steps and args.workload == "C2" and args.regions is None:
+        extra = {"C3": run_extra(ctx, "C3", DEFAULT_REGIONS["C3"], args, stream, flush)}
+
     if rank == 0:
+        split = (f"strong: the fixed {n_regions}-region job split over {ws} rank(s) by cells (whole regions)"
+                 if scaling == "strong" else f"weak: {n_regions} regions per rank")
         line = {"metric": "PairHMM GCUPS", "value": value, "unit": "GCUPS", "n_gpus": ws, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": 1e3 * t_max / args.steps,
                 "ms_per_step_median": float(np.median(step_ms)), "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-                "config": {"workload": WORKLOADS[args.workload], "regions_per_rank": n_regions,
-                           "pairs_per_rank": n_pairs, "cells_per_rank": cells,
-                           "padded_cells_per_rank": ctx.stats()["padded_cells"],
-                           "rescued_pairs_per_rank": rescued,
+                "scaling": scaling, "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": WORKLOADS[args.workload], "split": split,
+                           "regions_rank0": r1 - r0, "pairs_rank0": n_pairs, "cells_rank0": cells,
+                           "job_pairs": total_pairs, "job_cells": total_cells,
+                           "padded_cells_rank0": ctx.stats()["padded_cells"],
+                           "rescued_pairs_rank0": rescued, "chunks_rank0": ctx.stats()["n_chunks"],
                            "l2": "flushed between timed steps (256 MiB write, untimed)",
-                           "parallelism": f"dp{ws} (independent pair shards, NCCL all-gather of results)"},
+                           "parallelism": f"dp{ws} (independent region shards, one NCCL all-gather of results)"},
+                "result_sha256": result_hash,
                 "gpu_launches": launches,
                 "roofline": roofline, "rescue": rescue, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
-                "paper_context": PAPER_CONTEXT}
+                "extra": extra, "paper_context": PAPER_CONTEXT}
         print(json.dumps(line), flush=True)
     ctx.close()
     if ws > 1:

@@ -136,17 +136,18 @@ typedef struct {
 phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg);
 
 /*
- * Host-buffer variant. Copies the batch to the device (pinned staging,
- * async H2D on the context stream), runs the whole path, copies the results
- * back and returns when out_log10 (n_pairs doubles, caller-owned host memory)
- * and, if non-NULL, out_status (n_pairs bytes) are written.
+ * Host-buffer variant. Copies the batch to the device on the context stream,
+ * runs the whole path, copies the results back and returns when out_log10
+ * (n_pairs doubles, caller-owned host memory) and, if non-NULL, out_status
+ * (n_pairs bytes) are written.
  * out_log10[p] = log10 P(read | hap) of pair p; -inf when P underflows even
  * the FP64 rescue or is exactly 0 (Q0 inputs).
- * With the environment variable PHMM_CHUNKS=n (2..4) set when the context is
- * created, batches of >= 2^17 pairs are copied and computed in n chunks whose
- * copies overlap the previous chunk's FP32 pass (same results bit for bit;
- * measured slower on B200, so off by default). Inputs are
- * validated chunk by chunk; an error still leaves the outputs untouched.
+ * Copies: a buffer that is page-locked (cudaMallocHost / cudaHostRegister) is
+ * copied by one cudaMemcpyAsync; a pageable buffer goes through the context's
+ * pinned staging ring (4 x 8 MiB, filled by a pool of host threads while the
+ * previous piece is in flight; phmm_stats.staged_bytes counts these bytes). The
+ * number of host threads is min(8, cores / 2), or PHMM_STAGE_THREADS when the
+ * context is created.
  */
 phmm_status phmm_compute_batch(phmm_ctx* ctx, const phmm_batch* b, double* out_log10,
                                uint8_t* out_status);
@@ -189,7 +190,7 @@ typedef struct {
   int64_t padded_cells;     /* cells the wavefront kernels actually computed (pad rows/cols) */
   int64_t n_rescued;        /* pairs re-run in FP64 */
   int64_t n_fp64_underflow; /* pairs whose FP64 sum was 0 or subnormal */
-  int32_t n_bins;           /* haplotype-length bins of the FP32 pass */
+  int32_t n_chunks;         /* pair chunks the call ran as (batches > 2^23 pairs run in chunks) */
   int32_t kernel_launches;  /* kernels launched by the call */
   float ms_total;           /* whole call on the stream (device side) */
   float ms_h2d;             /* host->device copies (host variant only) */
@@ -198,6 +199,7 @@ typedef struct {
   float ms_rescue;          /* FP64 rescue pass (prep + wavefront) */
   float ms_finalize;        /* log10 + scatter */
   float ms_d2h;             /* device->host copy (host variant only) */
+  int64_t staged_bytes;     /* host variant: bytes copied through the pinned staging buffers */
 } phmm_stats;
 
 phmm_status phmm_get_stats(const phmm_ctx* ctx, phmm_stats* out);

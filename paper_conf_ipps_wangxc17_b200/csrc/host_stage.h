@@ -1,0 +1,209 @@
+// host_stage.h -- host <-> device copies of the host-buffer call (phmm_compute_batch) through
+// context-owned pinned staging buffers ("stage into pinned memory, then
+// H2D"; the paper's end-to-end times include these transfers, PAPER.md L24@1130, §V-B).
+//
+// A caller's buffer that is already page-locked (cudaMallocHost / cudaHostRegister) is copied
+// by one cudaMemcpyAsync. A pageable buffer is cut into pieces of kStagePiece bytes that cycle
+// through a ring of kStageSlots pinned slots: host threads memcpy piece k into its slot while
+// the DMA engine moves piece k-1 to the device (one cudaMemcpyAsync per piece, an event per
+// slot tells when the slot may be refilled). Results travel back the same way in reverse.
+// Host part of libphmm only (no kernels).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <condition_variable>
+#include <cstdint>
+#include <cstring>
+#include <functional>
+#include <mutex>
+#include <thread>
+#include <vector>
+
+namespace phmm {
+
+// A fixed pool of host threads for parallel memcpy (one job at a time, split evenly).
+class CopyPool {
+ public:
+  explicit CopyPool(int n) {
+    for (int i = 0; i < n; ++i) th_.emplace_back([this, i] { run(i); });
+  }
+  ~CopyPool() {
+    {
+      std::lock_guard<std::mutex> g(m_);
+      stop_ = true;
+    }
+    cv_.notify_all();
+    for (auto& t : th_) t.join();
+  }
+  int size() const { return (int)th_.size() + 1; }
+  // dst[0..n) = src[0..n), split over the pool's threads and the caller's
+  void memcpy_par(void* dst, const void* src, size_t n) {
+    const int parts = size();
+    if (n < (size_t)1 << 20 || parts == 1) {
+      std::memcpy(dst, src, n);
+      return;
+    }
+    {
+      std::lock_guard<std::mutex> g(m_);
+      dst_ = static_cast<char*>(dst);
+      src_ = static_cast<const char*>(src);
+      n_ = n;
+      pending_ = (int)th_.size();
+      ++gen_;
+    }
+    cv_.notify_all();
+    part(0, parts);
+    std::unique_lock<std::mutex> lk(m_);
+    done_cv_.wait(lk, [this] { return pending_ == 0; });
+  }
+
+ private:
+  void part(int k, int parts) {
+    const size_t per = ((n_ + parts - 1) / parts + 63) & ~(size_t)63;
+    const size_t a = std::min(n_, per * (size_t)k), z = std::min(n_, a + per);
+    if (z > a) std::memcpy(dst_ + a, src_ + a, z - a);
+  }
+  void run(int i) {
+    uint64_t seen = 0;
+    while (true) {
+      {
+        std::unique_lock<std::mutex> lk(m_);
+        cv_.wait(lk, [&] { return stop_ || gen_ != seen; });
+        if (stop_) return;
+        seen = gen_;
+      }
+      part(i + 1, size());
+      {
+        std::lock_guard<std::mutex> g(m_);
+        if (--pending_ == 0) done_cv_.notify_one();
+      }
+    }
+  }
+  std::vector<std::thread> th_;
+  std::mutex m_;
+  std::condition_variable cv_, done_cv_;
+  bool stop_ = false;
+  uint64_t gen_ = 0;
+  int pending_ = 0;
+  char* dst_ = nullptr;
+  const char* src_ = nullptr;
+  size_t n_ = 0;
+};
+
+constexpr int kStageSlots = 4;
+constexpr size_t kStagePiece = (size_t)8 << 20;
+
+struct Stager {
+  void* slot[kStageSlots] = {};
+  cudaEvent_t ev[kStageSlots] = {};
+  bool used[kStageSlots] = {};
+  int next = 0;
+  CopyPool* pool = nullptr;
+  int64_t staged_bytes = 0;  // bytes of the last call that went through the slots
+
+  cudaError_t init(int threads) {
+    for (int i = 0; i < kStageSlots; ++i) {
+      cudaError_t e = cudaMallocHost(&slot[i], kStagePiece);
+      if (e != cudaSuccess) {
+        slot[i] = nullptr;
+        return e;
+      }
+      e = cudaEventCreateWithFlags(&ev[i], cudaEventDisableTiming);
+      if (e != cudaSuccess) {
+        ev[i] = nullptr;
+        return e;
+      }
+    }
+    pool = new CopyPool(std::max(0, threads - 1));
+    return cudaSuccess;
+  }
+  void release() {
+    for (int i = 0; i < kStageSlots; ++i) {
+      if (ev[i]) cudaEventSynchronize(ev[i]);
+      if (slot[i]) cudaFreeHost(slot[i]);
+      if (ev[i]) cudaEventDestroy(ev[i]);
+      slot[i] = nullptr;
+      ev[i] = nullptr;
+    }
+    delete pool;
+    pool = nullptr;
+  }
+
+  static bool is_pinned(const void* p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    return a.type == cudaMemoryTypeHost;
+  }
+
+  // the next free slot (waits for its previous DMA)
+  cudaError_t take(int* k) {
+    *k = next;
+    next = (next + 1) % kStageSlots;
+    if (used[*k]) {
+      cudaError_t e = cudaEventSynchronize(ev[*k]);
+      if (e != cudaSuccess) return e;
+    }
+    used[*k] = true;
+    return cudaSuccess;
+  }
+
+  // host -> device on stream s
+  cudaError_t h2d(void* dst, const void* src, size_t n, cudaStream_t s) {
+    if (n == 0) return cudaSuccess;
+    if (is_pinned(src)) return cudaMemcpyAsync(dst, src, n, cudaMemcpyHostToDevice, s);
+    for (size_t off = 0; off < n; off += kStagePiece) {
+      const size_t b = std::min(kStagePiece, n - off);
+      int k;
+      cudaError_t e = take(&k);
+      if (e != cudaSuccess) return e;
+      pool->memcpy_par(slot[k], static_cast<const char*>(src) + off, b);
+      e = cudaMemcpyAsync(static_cast<char*>(dst) + off, slot[k], b, cudaMemcpyHostToDevice, s);
+      if (e != cudaSuccess) return e;
+      e = cudaEventRecord(ev[k], s);
+      if (e != cudaSuccess) return e;
+      staged_bytes += (int64_t)b;
+    }
+    return cudaSuccess;
+  }
+
+  // device -> host on stream s; returns when dst holds the data
+  cudaError_t d2h(void* dst, const void* src, size_t n, cudaStream_t s) {
+    if (n == 0) return cudaSuccess;
+    if (is_pinned(dst)) {
+      cudaError_t e = cudaMemcpyAsync(dst, src, n, cudaMemcpyDeviceToHost, s);
+      return e != cudaSuccess ? e : cudaStreamSynchronize(s);
+    }
+    // keep up to kStageSlots pieces in flight; copy each out as soon as it arrived
+    const size_t npieces = (n + kStagePiece - 1) / kStagePiece;
+    int slot_of[kStageSlots];
+    size_t issued = 0, drained = 0;
+    while (drained < npieces) {
+      while (issued < npieces && issued - drained < (size_t)kStageSlots) {
+        const size_t off = issued * kStagePiece, b = std::min(kStagePiece, n - off);
+        int k;
+        cudaError_t e = take(&k);
+        if (e != cudaSuccess) return e;
+        e = cudaMemcpyAsync(slot[k], static_cast<const char*>(src) + off, b, cudaMemcpyDeviceToHost, s);
+        if (e != cudaSuccess) return e;
+        e = cudaEventRecord(ev[k], s);
+        if (e != cudaSuccess) return e;
+        slot_of[issued % kStageSlots] = k;
+        ++issued;
+      }
+      const int k = slot_of[drained % kStageSlots];
+      cudaError_t e = cudaEventSynchronize(ev[k]);
+      if (e != cudaSuccess) return e;
+      const size_t off = drained * kStagePiece, b = std::min(kStagePiece, n - off);
+      pool->memcpy_par(static_cast<char*>(dst) + off, slot[k], b);
+      staged_bytes += (int64_t)b;
+      ++drained;
+    }
+    return cudaSuccess;
+  }
+};
+
+}  // namespace phmm

@@ -187,14 +187,17 @@ __global__ void k_finalize_fp64(const double* __restrict__ s64, const int32_t* _
   }
 }
 
-// One chunk of a host batch (phmm_compute_batch's copy/compute pipeline): the chunk's
-// offsets relative to its first read / haplotype and its pairs relative to both, so that the
-// chunk is an ordinary batch over [rlo, rlo + nr) reads and [hlo, hlo + nh) haplotypes.
+// One chunk of a batch: its pairs relative to its first read / haplotype (rlo, hlo), and the
+// offsets of its reads [rlo, rlo + nr) / haplotypes [hlo, hlo + nh). relative = 1 (the host
+// variant's copy/compute pipeline, whose chunk arrays start at the chunk's first byte): the
+// offsets relative to that byte; relative = 0 (a chunked device call, which addresses the
+// batch's base arrays): the offsets keep their values.
 __global__ void k_rebase_chunk(const int64_t* __restrict__ roff, int64_t rlo, int64_t nr, int64_t* __restrict__ roff_c,
                                const int64_t* __restrict__ hoff, int64_t hlo, int64_t nh, int64_t* __restrict__ hoff_c,
-                               const int32_t* __restrict__ pairs, int64_t p0, int64_t np, int32_t* __restrict__ pairs_c) {
+                               const int32_t* __restrict__ pairs, int64_t p0, int64_t np, int32_t* __restrict__ pairs_c,
+                               int relative) {
   const int64_t n = (nr + 1 > nh + 1 ? nr + 1 : nh + 1) > np ? (nr + 1 > nh + 1 ? nr + 1 : nh + 1) : np;
-  const int64_t r0 = roff[rlo], h0 = hoff[hlo];
+  const int64_t r0 = relative ? roff[rlo] : 0, h0 = relative ? hoff[hlo] : 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     if (i <= nr) roff_c[i] = roff[rlo + i] - r0;
     if (i <= nh) hoff_c[i] = hoff[hlo + i] - h0;
@@ -202,6 +205,36 @@ __global__ void k_rebase_chunk(const int64_t* __restrict__ roff, int64_t rlo, in
       pairs_c[2 * i] = pairs[2 * (p0 + i)] - (int32_t)rlo;
       pairs_c[2 * i + 1] = pairs[2 * (p0 + i) + 1] - (int32_t)hlo;
     }
+  }
+}
+
+// Index ranges of the chunks of a chunked device call: chunk blockIdx.y = pairs
+// [y * chunk_pairs, ...); rng[4y .. 4y+3] = min / max read index, min / max haplotype index
+// (minima preset to UINT_MAX, maxima to 0). Out-of-range indices raise ERR_INDEX.
+__global__ void k_chunk_ranges(const int32_t* __restrict__ pairs, int64_t n_pairs, int64_t chunk_pairs,
+                               int64_t n_reads, int64_t n_haps, uint32_t* __restrict__ rng, uint32_t* err) {
+  const int64_t p0 = (int64_t)blockIdx.y * chunk_pairs;
+  const int64_t p1 = min(n_pairs, p0 + chunk_pairs);
+  uint32_t rmin = 0xffffffffu, rmax = 0, hmin = 0xffffffffu, hmax = 0, e = 0;
+  for (int64_t p = p0 + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < p1; p += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
+    if (r < 0 || r >= n_reads || h < 0 || h >= n_haps) {
+      e |= ERR_INDEX;
+      continue;
+    }
+    rmin = min(rmin, (uint32_t)r); rmax = max(rmax, (uint32_t)r);
+    hmin = min(hmin, (uint32_t)h); hmax = max(hmax, (uint32_t)h);
+  }
+  rmin = __reduce_min_sync(0xffffffffu, rmin); rmax = __reduce_max_sync(0xffffffffu, rmax);
+  hmin = __reduce_min_sync(0xffffffffu, hmin); hmax = __reduce_max_sync(0xffffffffu, hmax);
+  e = __reduce_or_sync(0xffffffffu, e);
+  if ((threadIdx.x & 31) == 0) {
+    uint32_t* g = rng + 4 * blockIdx.y;
+    if (rmin != 0xffffffffu) {
+      atomicMin(g, rmin); atomicMax(g + 1, rmax);
+      atomicMin(g + 2, hmin); atomicMax(g + 3, hmax);
+    }
+    if (e) atomicOr(err, e);
   }
 }
 

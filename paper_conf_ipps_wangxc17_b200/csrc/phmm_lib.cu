@@ -18,6 +18,7 @@
 
 #include "../../include/phmm.h"
 #include "phmm_device.cuh"
+#include "host_stage.h"
 #include "stream_prep.cuh"
 #include "sw.cuh"
 
@@ -35,8 +36,9 @@ enum BufId {
   B_SW_BTSZ, B_SW_BTOFF, B_SW_OPCAP, B_SW_OPOFF, B_SW_BT, B_SW_KEYS, B_SW_VALS, B_SW_OPTMP, B_SW_NOPS,
   B_SW_NOPOFF,
   B_SKEYS, B_SVALS, B_NBS, B_BLKOFF, B_SORT_TMP, B_EXP32,
-  B_CH_ROFF, B_CH_HOFF, B_CH_PAIRS, B_CH_CNT,  // host-variant pipeline: one chunk's rebased offsets / pairs
+  B_CH_ROFF, B_CH_HOFF, B_CH_PAIRS,            // chunked device call: one chunk's offsets / rebased pairs
   B_DEDUP,                                       // rescue pass: head flags + their scan (one table per read)
+  B_CH_RANGES,                                   // chunked device call: read / haplotype index range per chunk
   B_COUNT
 };
 
@@ -57,12 +59,14 @@ struct Scalars {
   unsigned int item_counter[2];  // work-item counters of the (at most 2) wavefront launches
 };
 
-constexpr int kEvents = 10;
+constexpr int kEvents = 11;
 constexpr int kThreads = 256;
-// host variant (phmm_compute_batch): the pairs are cut into up to kMaxChunks chunks of at least
-// kChunkMinPairs; chunk k+1's inputs are copied on a second stream while chunk k computes
-constexpr int kMaxChunks = 4;
-constexpr int64_t kChunkMinPairs = 65536;
+// device path: batches of more pairs than this run as consecutive chunks (compute_dev)
+constexpr int64_t kDevChunkPairs = 1ll << 23;
+
+struct PhaseMs {
+  float prep, wf, fin, resc;
+};
 
 }  // namespace
 
@@ -80,11 +84,13 @@ struct phmm_ctx {
   int64_t* host_sizes = nullptr;  // pinned, 2 values
   int64_t sw_ops_cap = 0;         // last SW call: sum over tasks of M + N
   cudaEvent_t ev[kEvents] = {};
-  cudaStream_t copy_stream = nullptr;     // host variant: H2D of the next chunk
-  cudaEvent_t cev[kMaxChunks + 1] = {};   // chunk k's inputs on the device / the call's start
-  int max_chunks = 1;                     // PHMM_CHUNKS=n (<= kMaxChunks) turns the pipeline on (measured slower)
+  Stager stage;                           // host variant: pinned staging of pageable buffers
   phmm_stats st{};
+  PhaseMs acc{};                          // per-phase times summed over a call's chunks
   int launches = 0;
+  int64_t chunk_pairs = kDevChunkPairs;   // PHMM_CHUNK_PAIRS=n overrides (tests)
+  uint32_t* host_ranges = nullptr;        // pinned: per-chunk index ranges of a chunked call
+  int64_t host_ranges_n = 0;
 };
 
 namespace {
@@ -162,7 +168,7 @@ phmm_status map_err(uint32_t e) {
   return PHMM_E_INVALID_ARG;
 }
 
-enum { EV_START, EV_H2D, EV_PREP, EV_WF0, EV_WF1, EV_RESC0, EV_RESC1, EV_FIN, EV_D2H, EV_END };
+enum { EV_START, EV_H2D, EV_PREP, EV_WF0, EV_WF1, EV_RESC0, EV_RESC1, EV_FIN, EV_D2H, EV_END, EV_CH0 };
 
 void ev_record(phmm_ctx* c, int i) {
   if (c->flags & PHMM_FLAG_TIMING) cudaEventRecord(c->ev[i], c->stream);
@@ -538,22 +544,41 @@ phmm_status rescue_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   if (timed) ev_record(c, EV_RESC1);
   CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaStreamSynchronize(s));
-  c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
+  c->st.n_fp64_underflow += (int64_t)c->host_scal->n_underflow;
   return PHMM_OK;
 }
 
-// The whole path on device-resident inputs. Writes dev_out (+ dev_status).
-phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status) {
+// Per-phase times of one compute_one (PHMM_FLAG_TIMING), added to the call's totals once its
+// last event completed.
+void acc_phases(phmm_ctx* c) {
+  if (!(c->flags & PHMM_FLAG_TIMING)) return;
+  const bool fp64 = c->prec == PHMM_PREC_FP64;
+  cudaEventSynchronize(c->ev[fp64 ? EV_FIN : EV_RESC1]);
+  auto add = [&](float& acc, int a, int b) {
+    const float ms = ev_ms(c, a, b);
+    if (ms >= 0.f) acc += ms;
+  };
+  add(c->acc.prep, EV_CH0, EV_PREP);
+  add(c->acc.wf, EV_WF0, EV_WF1);
+  if (fp64) {
+    add(c->acc.fin, EV_WF1, EV_FIN);
+  } else {
+    add(c->acc.fin, EV_WF1, EV_RESC0);
+    add(c->acc.resc, EV_RESC0, EV_RESC1);
+  }
+}
+
+// The whole path on one (validated) batch or chunk: the FP32 pass and the FP64 rescue of its
+// underflowing pairs (or the FP64 pass), results into out / status (context scratch).
+// Accumulates the call's statistics; ends synchronised.
+phmm_status compute_one(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status) {
   cudaStream_t s = c->stream;
-  c->st = phmm_stats{};
-  c->st.n_pairs = d.n_pairs;
-  if (d.n_pairs == 0) return PHMM_OK;
-  ST_TRY(run_validate(c, d));
   PassInfo pi;
   int64_t total_tab = 0, total_hc = 0;
   uint8_t* hc = nullptr;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
+  ev_record(c, EV_CH0);
   if (c->prec == PHMM_PREC_FP64) {
     ST_TRY((pass_prepare<double>(c, d, nullptr, d.n_pairs, &pi, &total_tab, &total_hc)));
     ST_TRY(build_hap_codes(c, d, total_hc, pi.max_ncols, &hc));
@@ -570,8 +595,8 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     ev_record(c, EV_FIN);
     CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
-    c->st.n_fp64_underflow = (int64_t)c->host_scal->n_underflow;
-    c->st.cells = (int64_t)pi.cells;
+    c->st.n_fp64_underflow += (int64_t)c->host_scal->n_underflow;
+    c->st.cells += (int64_t)pi.cells;
     c->st.padded_cells += (int64_t)pi.padded_cells;
   } else {
     int32_t* rlist;
@@ -582,9 +607,79 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     const int64_t nr = c->host_scal->n_rescue;
-    c->st.n_rescued = nr;
+    c->st.n_rescued += nr;
     if (nr > 0) ST_TRY(rescue_pass(c, d, dev_out, dev_status, rlist, nr, hc, total_hc, true));
     else ev_record(c, EV_RESC1);
+  }
+  acc_phases(c);
+  ++c->st.n_chunks;
+  return PHMM_OK;
+}
+
+// The whole path on device-resident inputs. Writes dev_out (+ dev_status), which are context
+// scratch (the callers copy them to the caller's buffers after success).
+// Batches of more than kDevChunkPairs pairs run as consecutive chunks of pairs, each an
+// ordinary batch over the reads and haplotypes its pairs use (same results bit for bit:
+// a pair's arithmetic does not depend on its batch, R14), so the per-read tables and block
+// descriptors stay a few GB whatever the batch size (the 2^26-pair C5 at N = 1).
+phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status) {
+  cudaStream_t s = c->stream;
+  c->st = phmm_stats{};
+  c->acc = PhaseMs{};
+  c->st.n_pairs = d.n_pairs;
+  if (d.n_pairs == 0) return PHMM_OK;
+  ST_TRY(run_validate(c, d));
+  const int64_t cp = c->chunk_pairs;
+  if (d.n_pairs <= cp) return compute_one(c, d, dev_out, dev_status);
+  // chunk k = pairs [k*cp, min((k+1)*cp, n)); its read / haplotype index ranges in one pass
+  const int64_t nch = (d.n_pairs + cp - 1) / cp;
+  Scalars* scal;
+  uint32_t* rng;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  ST_TRY(ws(c, B_CH_RANGES, (size_t)4 * nch, &rng));
+  CUDA_TRY(cudaMemsetAsync(rng, 0, sizeof(uint32_t) * 4 * nch, s));
+  for (int64_t k = 0; k < nch; ++k) {  // minima start at UINT_MAX
+    CUDA_TRY(cudaMemsetAsync(rng + 4 * k, 0xff, sizeof(uint32_t), s));
+    CUDA_TRY(cudaMemsetAsync(rng + 4 * k + 2, 0xff, sizeof(uint32_t), s));
+  }
+  {
+    const int bpc = (int)std::max<int64_t>(1, std::min<int64_t>((cp + kThreads - 1) / kThreads, 4 * c->nsm));
+    k_chunk_ranges<<<dim3((unsigned)bpc, (unsigned)nch), kThreads, 0, s>>>(d.pairs, d.n_pairs, cp, d.n_reads,
+                                                                              d.n_haps, rng, &scal->err);
+    LAUNCHED(c);
+  }
+  uint32_t* hr = c->host_ranges;
+  if (c->host_ranges_n < nch) {
+    if (hr) cudaFreeHost(hr);
+    c->host_ranges = nullptr;
+    c->host_ranges_n = 0;
+    if (cudaMallocHost(&hr, sizeof(uint32_t) * 4 * nch) != cudaSuccess) {
+      cudaGetLastError();
+      return PHMM_E_OOM;
+    }
+    c->host_ranges = hr;
+    c->host_ranges_n = nch;
+  }
+  CUDA_TRY(cudaMemcpyAsync(hr, rng, sizeof(uint32_t) * 4 * nch, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  if (c->host_scal->err) return map_err(c->host_scal->err);
+  int64_t *roff_c, *hoff_c;
+  int32_t* pairs_c;
+  for (int64_t k = 0; k < nch; ++k) {
+    const int64_t p0 = k * cp, np = std::min(cp, d.n_pairs - p0);
+    const int64_t rlo = hr[4 * k], nr = (int64_t)hr[4 * k + 1] + 1 - rlo;
+    const int64_t hlo = hr[4 * k + 2], nh = (int64_t)hr[4 * k + 3] + 1 - hlo;
+    ST_TRY(ws(c, B_CH_ROFF, (size_t)nr + 1, &roff_c));
+    ST_TRY(ws(c, B_CH_HOFF, (size_t)nh + 1, &hoff_c));
+    ST_TRY(ws(c, B_CH_PAIRS, (size_t)2 * np, &pairs_c));
+    // the chunk's offsets keep their absolute values (the chunk addresses the batch's base
+    // arrays); its pair indices become relative to rlo / hlo
+    k_rebase_chunk<<<grid_for(c, std::max(std::max(nr, nh) + 1, np)), kThreads, 0, s>>>(
+        d.roff, rlo, nr, roff_c, d.hoff, hlo, nh, hoff_c, d.pairs, p0, np, pairs_c, 0);
+    LAUNCHED(c);
+    DevBatch dk{d.rb, d.q, d.qi, d.qd, d.qg, d.hap, roff_c, hoff_c, pairs_c, nr, nh, np, d.n_rb, d.n_hb};
+    ST_TRY(compute_one(c, dk, dev_out + p0, dev_status ? dev_status + p0 : nullptr));
   }
   return PHMM_OK;
 }
@@ -729,147 +824,14 @@ void finish_stats(phmm_ctx* c) {
   if (c->flags & PHMM_FLAG_TIMING) {
     cudaEventSynchronize(c->ev[EV_END]);
     c->st.ms_total = ev_ms(c, EV_START, EV_END);
-    c->st.ms_wavefront = ev_ms(c, EV_WF0, EV_WF1);
-    if (c->prec == PHMM_PREC_FP64) {
-      c->st.ms_prep = ev_ms(c, EV_H2D, EV_PREP);
-      c->st.ms_finalize = ev_ms(c, EV_WF1, EV_FIN);
-      c->st.ms_rescue = 0.f;
-    } else {
-      c->st.ms_prep = ev_ms(c, EV_H2D, EV_PREP);
-      c->st.ms_finalize = ev_ms(c, EV_WF1, EV_RESC0);
-      c->st.ms_rescue = ev_ms(c, EV_RESC0, EV_RESC1);
-    }
+    c->st.ms_prep = c->acc.prep;
+    c->st.ms_wavefront = c->acc.wf;
+    c->st.ms_finalize = c->acc.fin;
+    c->st.ms_rescue = c->prec == PHMM_PREC_FP64 ? 0.f : c->acc.resc;
   } else {
     c->st.ms_total = c->st.ms_h2d = c->st.ms_prep = c->st.ms_wavefront = -1.f;
     c->st.ms_rescue = c->st.ms_finalize = c->st.ms_d2h = -1.f;
   }
-}
-
-// ------------------------------------------------------------ host variant: copy/compute pipeline
-// phmm_compute_batch cuts the pairs into chunks; while chunk k computes on the context stream,
-// chunk k+1's inputs travel on the copy stream. Every read / haplotype is copied once: chunk k
-// copies the reads [rc0, rc1) not copied before (rc1 = one past the largest read index seen so
-// far, the last chunk takes the rest), and computes as an ordinary batch over the reads
-// [rlo, rhi) (rlo <= its smallest read index, and <= rc0 so that the chunks' read ranges
-// together cover -- and validate -- every read); same for haplotypes. The FP64 rescue runs once,
-// over the whole batch, after the last chunk; results travel back once, at the end, so an input
-// error found in a later chunk still leaves the caller's outputs untouched.
-struct ChunkPlan {
-  int64_t p0, p1, rlo, rhi, rc0, rc1, hlo, hhi, hc0, hc1;
-};
-
-phmm_status plan_chunk(const phmm_batch* b, int64_t p0, int64_t p1, int64_t rdone, int64_t hdone, bool last,
-                       ChunkPlan* cp) {
-  int64_t rmin = INT64_MAX, rmax = -1, hmin = INT64_MAX, hmax = -1;
-  const int32_t* pr = b->pairs;
-  for (int64_t p = p0; p < p1; ++p) {
-    const int64_t r = pr[2 * p], h = pr[2 * p + 1];
-    rmin = r < rmin ? r : rmin;
-    rmax = r > rmax ? r : rmax;
-    hmin = h < hmin ? h : hmin;
-    hmax = h > hmax ? h : hmax;
-  }
-  if (rmin < 0 || rmax >= b->n_reads || hmin < 0 || hmax >= b->n_haps) return PHMM_E_INDEX;
-  cp->p0 = p0;
-  cp->p1 = p1;
-  cp->rc0 = rdone;
-  cp->rc1 = last ? b->n_reads : std::max(rdone, rmax + 1);
-  cp->rlo = std::min(rmin, rdone);
-  cp->rhi = cp->rc1;
-  cp->hc0 = hdone;
-  cp->hc1 = last ? b->n_haps : std::max(hdone, hmax + 1);
-  cp->hlo = std::min(hmin, hdone);
-  cp->hhi = cp->hc1;
-  // the host offsets at the chunk's boundaries address the device copies: they must be ordered
-  // and in range (the device validates every offset inside the chunk's range)
-  auto ok = [](const int64_t* off, int64_t a, int64_t z, int64_t total) {
-    return off[a] >= 0 && off[a] <= off[z] && off[z] <= total;
-  };
-  if (!ok(b->read_offsets, cp->rlo, cp->rhi, b->total_read_bases) ||
-      !ok(b->read_offsets, cp->rc0, cp->rc1, b->total_read_bases) ||
-      !ok(b->hap_offsets, cp->hlo, cp->hhi, b->total_hap_bases) ||
-      !ok(b->hap_offsets, cp->hc0, cp->hc1, b->total_hap_bases))
-    return PHMM_E_INVALID_ARG;
-  return PHMM_OK;
-}
-
-phmm_status compute_host_chunked(phmm_ctx* c, const phmm_batch* b, int nchunks, uint8_t* rb, uint8_t* q, uint8_t* qi,
-                                 uint8_t* qd, uint8_t* qg, uint8_t* hap, int64_t* roff, int64_t* hoff, int32_t* pairs,
-                                 double* out, uint8_t* status) {
-  cudaStream_t s = c->stream, cs = c->copy_stream;
-  c->st = phmm_stats{};
-  c->st.n_pairs = b->n_pairs;
-  const int64_t np_max = (b->n_pairs + nchunks - 1) / nchunks;
-  int64_t *roff_c, *hoff_c, *cnt;
-  int32_t *pairs_c, *rlist;
-  ST_TRY(ws(c, B_CH_ROFF, (size_t)b->n_reads + 1, &roff_c));
-  ST_TRY(ws(c, B_CH_HOFF, (size_t)b->n_haps + 1, &hoff_c));
-  ST_TRY(ws(c, B_CH_PAIRS, (size_t)2 * np_max, &pairs_c));
-  ST_TRY(ws(c, B_CH_CNT, 2, &cnt));
-  ST_TRY(ws(c, B_RLIST, (size_t)b->n_pairs, &rlist));
-  const int64_t* ro = b->read_offsets;
-  const int64_t* ho = b->hap_offsets;
-  auto copy_chunk = [&](const ChunkPlan& P, int k) -> phmm_status {
-    if (k == 0) {  // all offsets with the first chunk (the rebase and the rescue read them)
-      CUDA_TRY(cudaMemcpyAsync(roff, ro, sizeof(int64_t) * (b->n_reads + 1), cudaMemcpyHostToDevice, cs));
-      CUDA_TRY(cudaMemcpyAsync(hoff, ho, sizeof(int64_t) * (b->n_haps + 1), cudaMemcpyHostToDevice, cs));
-    }
-    const int64_t a0 = ro[P.rc0], a1 = ro[P.rc1];
-    if (a1 > a0) {
-      const uint8_t* src[5] = {b->read_bases, b->base_quals, b->ins_quals, b->del_quals, b->gcp_quals};
-      uint8_t* dst[5] = {rb, q, qi, qd, qg};
-      for (int i = 0; i < 5; ++i)
-        CUDA_TRY(cudaMemcpyAsync(dst[i] + a0, src[i] + a0, (size_t)(a1 - a0), cudaMemcpyHostToDevice, cs));
-    }
-    const int64_t h0 = ho[P.hc0], h1 = ho[P.hc1];
-    if (h1 > h0) CUDA_TRY(cudaMemcpyAsync(hap + h0, b->hap_bases + h0, (size_t)(h1 - h0), cudaMemcpyHostToDevice, cs));
-    CUDA_TRY(cudaMemcpyAsync(pairs + 2 * P.p0, b->pairs + 2 * P.p0, sizeof(int32_t) * 2 * (P.p1 - P.p0),
-                             cudaMemcpyHostToDevice, cs));
-    CUDA_TRY(cudaEventRecord(c->cev[k], cs));
-    return PHMM_OK;
-  };
-  ChunkPlan plan[kMaxChunks];
-  auto bound = [&](int k) { return b->n_pairs * k / nchunks; };
-  ST_TRY(plan_chunk(b, bound(0), bound(1), 0, 0, nchunks == 1, &plan[0]));
-  // the copies start after whatever the caller queued on the context stream
-  CUDA_TRY(cudaEventRecord(c->cev[kMaxChunks], s));
-  CUDA_TRY(cudaStreamWaitEvent(cs, c->cev[kMaxChunks], 0));
-  ev_record(c, EV_START);
-  ST_TRY(copy_chunk(plan[0], 0));
-  CUDA_TRY(cudaMemsetAsync(cnt, 0, 2 * sizeof(int64_t), s));
-  for (int k = 0; k < nchunks; ++k) {
-    if (k + 1 < nchunks) {
-      ST_TRY(plan_chunk(b, bound(k + 1), bound(k + 2), plan[k].rc1, plan[k].hc1, k + 2 == nchunks, &plan[k + 1]));
-      ST_TRY(copy_chunk(plan[k + 1], k + 1));
-    }
-    const ChunkPlan& P = plan[k];
-    CUDA_TRY(cudaStreamWaitEvent(s, c->cev[k], 0));
-    const int64_t nr = P.rhi - P.rlo, nh = P.hhi - P.hlo, np = P.p1 - P.p0;
-    k_rebase_chunk<<<grid_for(c, std::max(std::max(nr, nh) + 1, np)), kThreads, 0, s>>>(
-        roff, P.rlo, nr, roff_c, hoff, P.hlo, nh, hoff_c, pairs, P.p0, np, pairs_c);
-    LAUNCHED(c);
-    const int64_t a0 = ro[P.rlo], h0 = ho[P.hlo];
-    DevBatch dk{rb + a0, q + a0, qi + a0, qd + a0, qg + a0, hap + h0, roff_c, hoff_c, pairs_c,
-                nr, nh, np, ro[P.rhi] - a0, ho[P.hhi] - h0};
-    ST_TRY(run_validate(c, dk));
-    PassInfo pi;
-    uint8_t* hc = nullptr;
-    int64_t total_hc = 0;
-    ST_TRY(fp32_pass(c, dk, out + P.p0, status ? status + P.p0 : nullptr, rlist, P.p0, cnt, &pi, &hc, &total_hc,
-                     false));
-  }
-  int64_t* hcnt = c->host_sizes;
-  CUDA_TRY(cudaMemcpyAsync(hcnt, cnt, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-  CUDA_TRY(cudaStreamSynchronize(s));
-  const int64_t nres = hcnt[0];
-  c->st.n_rescued = nres;
-  if (nres > 0) {  // the FP64 rescue over the whole batch (its own haplotype code regions)
-    DevBatch dg{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs,
-                b->total_read_bases, b->total_hap_bases};
-    ST_TRY(rescue_pass(c, dg, out, status, rlist, nres, nullptr, 0, false));
-  }
-  ev_record(c, EV_D2H);
-  return PHMM_OK;
 }
 
 }  // namespace
@@ -949,13 +911,15 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
   }
   for (int i = 0; i < kEvents; ++i)
     if (cudaEventCreate(&c->ev[i]) != cudaSuccess) return fail(PHMM_E_CUDA);
-  if (cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking) != cudaSuccess) {
-    c->copy_stream = nullptr;
-    return fail(PHMM_E_CUDA);
+  {
+    int threads = (int)std::min(8u, std::max(1u, std::thread::hardware_concurrency() / 2));
+    if (const char* e = std::getenv("PHMM_STAGE_THREADS")) threads = std::max(1, std::min(64, std::atoi(e)));
+    if (c->stage.init(threads) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(PHMM_E_OOM);
+    }
   }
-  for (int i = 0; i <= kMaxChunks; ++i)
-    if (cudaEventCreateWithFlags(&c->cev[i], cudaEventDisableTiming) != cudaSuccess) return fail(PHMM_E_CUDA);
-  if (const char* e = std::getenv("PHMM_CHUNKS")) c->max_chunks = std::max(1, std::min(kMaxChunks, std::atoi(e)));
+  if (const char* e = std::getenv("PHMM_CHUNK_PAIRS")) c->chunk_pairs = std::max<int64_t>(64, std::atoll(e));
   *out = c;
   return PHMM_OK;
 }
@@ -968,12 +932,10 @@ void phmm_destroy(phmm_ctx* c) {
     if (c->buf[i].p) cudaFree(c->buf[i].p);
   for (int i = 0; i < kEvents; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
-  if (c->copy_stream) cudaStreamSynchronize(c->copy_stream);
-  for (int i = 0; i <= kMaxChunks; ++i)
-    if (c->cev[i]) cudaEventDestroy(c->cev[i]);
-  if (c->copy_stream) cudaStreamDestroy(c->copy_stream);
+  c->stage.release();
   if (c->host_scal) cudaFreeHost(c->host_scal);
   if (c->host_sizes) cudaFreeHost(c->host_sizes);
+  if (c->host_ranges) cudaFreeHost(c->host_ranges);
   if (c->owned_stream) {
     cudaStreamSynchronize(c->owned_stream);
     cudaStreamDestroy(c->owned_stream);
@@ -1086,38 +1048,20 @@ phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log
   ST_TRY(ws(c, B_PAIRS, (size_t)b->n_pairs * 2, &pairs));
   ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
   if (out_status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
-  int nchunks = (int)std::min<int64_t>(c->max_chunks, b->n_pairs / kChunkMinPairs);
-  if (c->prec != PHMM_PREC_FP32_RESCUE) nchunks = 1;
-  if (nchunks > 1) {
-    phmm_status st = compute_host_chunked(c, b, nchunks, rb, q, qi, qd, qg, hap, roff, hoff, pairs, out, status);
-    if (st != PHMM_OK) {
-      cudaStreamSynchronize(c->copy_stream);
-      cudaStreamSynchronize(s);
-      cudaGetLastError();
-      return st;
-    }
-    CUDA_TRY(cudaMemcpyAsync(out_log10, out, sizeof(double) * b->n_pairs, cudaMemcpyDeviceToHost, s));
-    if (out_status) CUDA_TRY(cudaMemcpyAsync(out_status, status, b->n_pairs, cudaMemcpyDeviceToHost, s));
-    ev_record(c, EV_END);
-    CUDA_TRY(cudaStreamSynchronize(s));
-    c->st.kernel_launches = c->launches;
-    c->st.ms_total = ev_ms(c, EV_START, EV_END);
-    c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
-    c->st.ms_h2d = c->st.ms_prep = c->st.ms_wavefront = c->st.ms_rescue = c->st.ms_finalize = -1.f;  // overlapped
-    return PHMM_OK;
-  }
+  // H2D: page-locked caller buffers directly, pageable ones through the context's pinned
+  // staging ring (host_stage.h); the small arrays first
+  Stager& S = c->stage;
+  S.staged_bytes = 0;
   ev_record(c, EV_START);
-  if (nr) {
-    CUDA_TRY(cudaMemcpyAsync(rb, b->read_bases, nr, cudaMemcpyHostToDevice, s));
-    CUDA_TRY(cudaMemcpyAsync(q, b->base_quals, nr, cudaMemcpyHostToDevice, s));
-    CUDA_TRY(cudaMemcpyAsync(qi, b->ins_quals, nr, cudaMemcpyHostToDevice, s));
-    CUDA_TRY(cudaMemcpyAsync(qd, b->del_quals, nr, cudaMemcpyHostToDevice, s));
-    CUDA_TRY(cudaMemcpyAsync(qg, b->gcp_quals, nr, cudaMemcpyHostToDevice, s));
-  }
-  if (nh) CUDA_TRY(cudaMemcpyAsync(hap, b->hap_bases, nh, cudaMemcpyHostToDevice, s));
-  CUDA_TRY(cudaMemcpyAsync(roff, b->read_offsets, sizeof(int64_t) * (b->n_reads + 1), cudaMemcpyHostToDevice, s));
-  CUDA_TRY(cudaMemcpyAsync(hoff, b->hap_offsets, sizeof(int64_t) * (b->n_haps + 1), cudaMemcpyHostToDevice, s));
-  CUDA_TRY(cudaMemcpyAsync(pairs, b->pairs, sizeof(int32_t) * 2 * b->n_pairs, cudaMemcpyHostToDevice, s));
+  CUDA_TRY(S.h2d(roff, b->read_offsets, sizeof(int64_t) * (b->n_reads + 1), s));
+  CUDA_TRY(S.h2d(hoff, b->hap_offsets, sizeof(int64_t) * (b->n_haps + 1), s));
+  CUDA_TRY(S.h2d(pairs, b->pairs, sizeof(int32_t) * 2 * b->n_pairs, s));
+  CUDA_TRY(S.h2d(hap, b->hap_bases, nh, s));
+  CUDA_TRY(S.h2d(rb, b->read_bases, nr, s));
+  CUDA_TRY(S.h2d(q, b->base_quals, nr, s));
+  CUDA_TRY(S.h2d(qi, b->ins_quals, nr, s));
+  CUDA_TRY(S.h2d(qd, b->del_quals, nr, s));
+  CUDA_TRY(S.h2d(qg, b->gcp_quals, nr, s));
   ev_record(c, EV_H2D);
   DevBatch d{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs, (int64_t)nr, (int64_t)nh};
   phmm_status st = compute_dev(c, d, out, status);
@@ -1127,13 +1071,14 @@ phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log
     return st;
   }
   ev_record(c, EV_D2H);
-  CUDA_TRY(cudaMemcpyAsync(out_log10, out, sizeof(double) * b->n_pairs, cudaMemcpyDeviceToHost, s));
-  if (out_status) CUDA_TRY(cudaMemcpyAsync(out_status, status, b->n_pairs, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s));
+  if (out_status) CUDA_TRY(S.d2h(out_status, status, b->n_pairs, s));
   ev_record(c, EV_END);
   CUDA_TRY(cudaStreamSynchronize(s));
   finish_stats(c);
   c->st.ms_h2d = ev_ms(c, EV_START, EV_H2D);
   c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
+  c->st.staged_bytes = S.staged_bytes;
   return PHMM_OK;
 }
 
@@ -1204,12 +1149,14 @@ phmm_status phmm_sw_align_batch(phmm_ctx* c, const phmm_sw_batch* b, const phmm_
   ST_TRY(ws(c, B_SW_TASKS, (size_t)b->n_tasks * 2, &tasks));
   ST_TRY(ws(c, B_SW_RES, (size_t)b->n_tasks * 6, &res));
   ST_TRY(ws(c, B_SW_OPS, (size_t)std::max<int64_t>(ops_total, 1), &ops));
+  Stager& S = c->stage;
+  S.staged_bytes = 0;
   ev_record(c, EV_START);
-  if (nr) CUDA_TRY(cudaMemcpyAsync(ref, b->ref_bases, nr, cudaMemcpyHostToDevice, s));
-  if (na) CUDA_TRY(cudaMemcpyAsync(alt, b->alt_bases, na, cudaMemcpyHostToDevice, s));
-  CUDA_TRY(cudaMemcpyAsync(roff, b->ref_offsets, sizeof(int64_t) * (b->n_refs + 1), cudaMemcpyHostToDevice, s));
-  CUDA_TRY(cudaMemcpyAsync(aoff, b->alt_offsets, sizeof(int64_t) * (b->n_alts + 1), cudaMemcpyHostToDevice, s));
-  CUDA_TRY(cudaMemcpyAsync(tasks, b->tasks, sizeof(int32_t) * 2 * b->n_tasks, cudaMemcpyHostToDevice, s));
+  CUDA_TRY(S.h2d(ref, b->ref_bases, nr, s));
+  CUDA_TRY(S.h2d(alt, b->alt_bases, na, s));
+  CUDA_TRY(S.h2d(roff, b->ref_offsets, sizeof(int64_t) * (b->n_refs + 1), s));
+  CUDA_TRY(S.h2d(aoff, b->alt_offsets, sizeof(int64_t) * (b->n_alts + 1), s));
+  CUDA_TRY(S.h2d(tasks, b->tasks, sizeof(int32_t) * 2 * b->n_tasks, s));
   ev_record(c, EV_H2D);
   SwDev d{ref, alt, roff, aoff, tasks, b->n_refs, b->n_alts, b->n_tasks, (int64_t)nr, (int64_t)na};
   phmm_status st = sw_compute_dev(c, d, p, res, ops);
@@ -1219,11 +1166,10 @@ phmm_status phmm_sw_align_batch(phmm_ctx* c, const phmm_sw_batch* b, const phmm_
     return st;
   }
   ev_record(c, EV_D2H);
-  CUDA_TRY(cudaMemcpyAsync(out_res, res, sizeof(int32_t) * 6 * b->n_tasks, cudaMemcpyDeviceToHost, s));
-  CUDA_TRY(cudaStreamSynchronize(s));
+  CUDA_TRY(S.d2h(out_res, res, sizeof(int32_t) * 6 * b->n_tasks, s));
   int64_t used = 0;  // packed runs: only these travel back
   for (int64_t t = 0; t < b->n_tasks; ++t) used += out_res[6 * t + 5];
-  if (used > 0) CUDA_TRY(cudaMemcpyAsync(out_ops, ops, sizeof(uint32_t) * used, cudaMemcpyDeviceToHost, s));
+  if (used > 0) CUDA_TRY(S.d2h(out_ops, ops, sizeof(uint32_t) * used, s));
   ev_record(c, EV_END);
   CUDA_TRY(cudaStreamSynchronize(s));
   c->st.kernel_launches = c->launches;

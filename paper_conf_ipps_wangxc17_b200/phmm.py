@@ -60,10 +60,10 @@ class _Batch(ctypes.Structure):
 class _Stats(ctypes.Structure):
     _fields_ = [("n_pairs", ctypes.c_int64), ("cells", ctypes.c_int64), ("padded_cells", ctypes.c_int64),
                 ("n_rescued", ctypes.c_int64), ("n_fp64_underflow", ctypes.c_int64),
-                ("n_bins", ctypes.c_int32), ("kernel_launches", ctypes.c_int32),
+                ("n_chunks", ctypes.c_int32), ("kernel_launches", ctypes.c_int32),
                 ("ms_total", ctypes.c_float), ("ms_h2d", ctypes.c_float), ("ms_prep", ctypes.c_float),
                 ("ms_wavefront", ctypes.c_float), ("ms_rescue", ctypes.c_float),
-                ("ms_finalize", ctypes.c_float), ("ms_d2h", ctypes.c_float)]
+                ("ms_finalize", ctypes.c_float), ("ms_d2h", ctypes.c_float), ("staged_bytes", ctypes.c_int64)]
 
 
 class _SwBatch(ctypes.Structure):

@@ -28,6 +28,23 @@ def test_bench_json_line():
     assert rf["bound"] == "alu" and 0 < rf["frac"] < 1 and rf["achieved"] > d["value"]
     e = d["e2e"]
     assert 0 < e["value"] <= d["value"] * 1.05 and e["h2d_bytes_per_step"] > 0 and e["d2h_bytes_per_step"] > 0
+    assert 0 < e["pageable"]["value"] <= d["value"] * 1.05
+    assert len(d["result_sha256"]) == 64
     c = d["cpu_baseline"]
     assert c["kind"] == "oracle" and c["cores"] >= 1 and c["parity_max_abs_log10"] <= 1e-3
     assert d["clocks"]["samples"] >= 1
+
+
+def test_bench_c5_strong_split_line():
+    """--workload C5 (strong split of a fixed region set; here 64 regions = 16,384 pairs at
+    N = 1): the job's pairs and cells, and the result hash of the job in global pair order."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--workload", "C5", "--regions", "64",
+                        "--steps", "3", "--warmup", "3", "--no-e2e", "--no-cpu-baseline"], capture_output=True,
+                       text=True, timeout=900, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    d = json.loads([l for l in r.stdout.splitlines() if l.strip()][-1])
+    assert d["scaling"] == "strong" and d["config"]["job_pairs"] == 64 * 32 * 8
+    assert d["config"]["job_cells"] == d["config"]["cells_rank0"]
+    from paper_conf_ipps_wangxc17_b200 import synth
+    assert d["config"]["job_cells"] == synth.config_batch("C5", n_regions=64).cells()
+    assert len(d["result_sha256"]) == 64

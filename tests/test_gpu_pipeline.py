@@ -1,8 +1,11 @@
-"""The host-buffer call's optional copy/compute pipeline (phmm_compute_batch with
-PHMM_CHUNKS=n; off by default, measured slower): large batches are cut into chunks whose H2D overlaps the previous chunk's FP32 pass, with one
-FP64 rescue over the whole batch at the end. Results must be bitwise those of the
-device-buffer call (one pass over the whole batch) and of the unchunked host call, for any
-pair order, and an input error in a late chunk must still leave the outputs untouched."""
+"""The host-buffer call's copies and the device call's chunking.
+
+* phmm_compute_batch stages pageable host buffers through the context's pinned ring
+  (host_stage.h) and copies page-locked ones directly: results bitwise equal to the device
+  call for either kind of buffer, staged_bytes counting the staged input + output bytes.
+* phmm_compute_batch_dev runs batches of more than kDevChunkPairs pairs as consecutive
+  chunks (the full 2^26-pair C5 on one GPU): bitwise equal to the one-pass call.
+"""
 import os
 
 import numpy as np
@@ -16,89 +19,85 @@ pytestmark = pytest.mark.gpu
 
 @pytest.fixture(scope="module")
 def batch():
-    b = synth.config_batch("C2", n_regions=2048)  # 2^18 pairs: 4 chunks
+    b = synth.config_batch("C2", n_regions=2048)  # 2^18 pairs, 26 MB per read array: several 8 MiB pieces
     assert b.n_pairs == 1 << 18
     return b
 
 
 @pytest.fixture(scope="module")
 def ctx():
-    os.environ["PHMM_CHUNKS"] = "4"
-    try:
-        h = phmm.PairHMM(precision="fp32")
-    finally:
-        del os.environ["PHMM_CHUNKS"]
+    h = phmm.PairHMM(precision="fp32")
     yield h
     h.close()
 
 
-@pytest.fixture(scope="module")
-def ctx_one_shot():
-    os.environ["PHMM_CHUNKS"] = "1"
-    try:
-        h = phmm.PairHMM(precision="fp32")
-    finally:
-        del os.environ["PHMM_CHUNKS"]
-    yield h
-    h.close()
-
-
-@pytest.fixture(scope="module")
-def reference(batch, ctx):
+def test_pageable_and_pinned_host_buffers_are_bitwise_the_device_call(ctx, batch):
     import torch
 
     db = phmm.DeviceBatch.from_host(batch, device="cuda:0")
-    out, st = ctx.compute_batch_dev(db)
+    dev, dst = ctx.compute_batch_dev(db)
     torch.cuda.synchronize()
-    return out.cpu().numpy(), st.cpu().numpy(), ctx.stats()["n_rescued"]
-
-
-def test_chunked_host_call_is_bitwise_the_device_call(batch, ctx, ctx_one_shot, reference):
-    ref, ref_st, n_resc = reference
+    dev, dst = dev.cpu().numpy(), dst.cpu().numpy()
+    # pageable numpy arrays, pageable outputs
     got, st = ctx.compute_batch(batch)
-    assert ctx.stats()["n_rescued"] == n_resc > 0
-    assert np.array_equal(got, ref) and np.array_equal(st, ref_st)
-    one, st1 = ctx_one_shot.compute_batch(batch)
-    assert np.array_equal(one, ref) and np.array_equal(st1, ref_st)
-    # and against the oracle on a sample (plus rescued pairs)
-    rng = np.random.default_rng(5)
-    sample = np.unique(np.concatenate([rng.choice(batch.n_pairs, 500, replace=False), np.nonzero(st)[0][:500]]))
-    d = np.abs(got[sample] - oracle.batch_log10(batch, pair_idx=sample))
-    assert d.max() <= 1e-3
+    assert np.array_equal(got, dev) and np.array_equal(st, dst)
+    n = batch.n_pairs
+    staged = ctx.stats()["staged_bytes"]
+    assert staged == batch.nbytes_inputs() + 9 * n, (staged, batch.nbytes_inputs() + 9 * n)
+    # page-locked inputs and outputs: no staging
+    pin = {k: torch.from_numpy(np.ascontiguousarray(getattr(batch, k))).pin_memory().numpy()
+           for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets",
+                     "hap_bases", "hap_offsets", "pairs")}
+    pb = synth.Batch(**pin)
+    out = torch.empty(n, dtype=torch.float64).pin_memory().numpy()
+    sto = torch.empty(n, dtype=torch.uint8).pin_memory().numpy()
+    got2, st2 = ctx.compute_batch(pb, out=out, status=sto)
+    assert np.array_equal(got2, dev) and np.array_equal(st2, dst)
+    assert ctx.stats()["staged_bytes"] == 0
+    # a small batch (below one piece) and an odd-sized one agree with the oracle
+    small = synth.random_pairs_batch(3, 77)
+    g3, _ = ctx.compute_batch(small)
+    ref = oracle.batch_log10(small)
+    fin = np.isfinite(ref)
+    assert np.max(np.abs(g3[fin] - ref[fin])) <= 1e-3
 
 
-def test_chunked_any_pair_order(batch, ctx, reference):
-    """Shuffled pairs: every chunk references reads all over the batch (wide chunk ranges)."""
-    ref, ref_st, _ = reference
-    perm = np.random.default_rng(9).permutation(batch.n_pairs)
-    got, st = ctx.compute_batch(batch.subset(perm))
-    assert np.array_equal(got, ref[perm]) and np.array_equal(st, ref_st[perm])
-    # reversed order: the reads of the first chunk are the last ones copied
-    rev = np.arange(batch.n_pairs)[::-1].copy()
-    got, _ = ctx.compute_batch(batch.subset(rev))
-    assert np.array_equal(got, ref[rev])
+@pytest.mark.parametrize("prec", ["fp32", "fp64"])
+def test_device_call_chunking_is_bitwise(prec):
+    """compute_dev runs batches of more than kDevChunkPairs pairs (2^23; PHMM_CHUNK_PAIRS
+    lowers it here) as consecutive chunks of pairs over the reads / haplotypes each chunk uses
+    (so the full 2^26-pair C5 fits one GPU): results, statuses and the statistics' cell count
+    must equal the one-pass call bit for bit, also when a chunk's pairs use reads scattered
+    over the whole batch (shuffled pair order) and for a ragged last chunk."""
+    import torch
 
-
-@pytest.mark.parametrize("kind,code", [("base", -2), ("qual", -3), ("index", -5)])
-def test_error_in_last_chunk_leaves_outputs_untouched(batch, ctx, kind, code):
-    b = batch.subset(np.arange(batch.n_pairs))
-    b.read_bases = b.read_bases.copy()
-    b.ins_quals = b.ins_quals.copy()
-    b.pairs = b.pairs.copy()
-    last_read = int(b.pairs[-1, 0])
-    x = int(b.read_offsets[last_read]) + 1
-    if kind == "base":
-        b.read_bases[x] = ord("x")
-    elif kind == "qual":
-        b.ins_quals[x] = 200
-    else:
-        b.pairs[-1, 1] = b.n_haps
-    out = np.full(b.n_pairs, 12345.0)
-    st = np.full(b.n_pairs, 77, np.uint8)
-    with pytest.raises(phmm.PhmmError) as ei:
-        ctx.compute_batch(b, out=out, status=st)
-    assert ei.value.code == code
-    assert np.all(out == 12345.0) and np.all(st == 77)
-    small = synth.random_pairs_batch(3, 8)
-    got, _ = ctx.compute_batch(small)
-    assert np.max(np.abs(got - oracle.batch_log10(small))) <= 1e-3
+    b = synth.concat_batches([synth.config_batch("C3", n_regions=4), synth.random_pairs_batch(8, 300)])
+    b = b.subset(np.random.default_rng(1).permutation(b.n_pairs))
+    whole = phmm.PairHMM(precision=prec)
+    os.environ["PHMM_CHUNK_PAIRS"] = "1000"
+    try:
+        chunked = phmm.PairHMM(precision=prec, timing=True)
+    finally:
+        del os.environ["PHMM_CHUNK_PAIRS"]
+    try:
+        db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+        o1, s1 = whole.compute_batch_dev(db)
+        o2, s2 = chunked.compute_batch_dev(db)
+        torch.cuda.synchronize()
+        assert np.array_equal(o1.cpu().numpy(), o2.cpu().numpy())
+        assert np.array_equal(s1.cpu().numpy(), s2.cpu().numpy())
+        st = chunked.stats()
+        assert st["n_chunks"] == (b.n_pairs + 999) // 1000 and st["cells"] == b.cells()
+        assert st["ms_wavefront"] > 0
+        h, _ = chunked.compute_batch(b)  # the host variant chunks the same way
+        assert np.array_equal(h, o1.cpu().numpy())
+        # an index error in the last chunk: no output written
+        bad = b.subset(np.arange(b.n_pairs))
+        bad.pairs[-1, 0] = b.n_reads
+        out = np.full(b.n_pairs, 5.0)
+        with pytest.raises(phmm.PhmmError) as ei:
+            chunked.compute_batch(bad, out=out)
+        assert ei.value.code == -5 and np.all(out == 5.0)
+    finally:
+        whole.close()
+        chunked.close()
