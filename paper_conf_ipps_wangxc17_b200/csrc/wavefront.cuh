@@ -55,6 +55,9 @@ __device__ int g_trace_steps;
 #ifndef PHMM_F64_MINB
 #define PHMM_F64_MINB 2
 #endif
+#ifndef PHMM_CW_PREFETCH
+#define PHMM_CW_PREFETCH 0  // 1: code words of a lane's next block prefetched one pass ahead
+#endif
 #ifndef PHMM_XCHG_SMEM
 #define PHMM_XCHG_SMEM 0  // 1: design-A ablation build (row exchange through shared memory)
 #endif
@@ -321,37 +324,61 @@ __host__ __device__ inline int wf_hc_copy_len(int ncols) {
   return ((int)WF_HC_FRONT + wf_pass_len(ncols) + 24 + 3) & ~3;  // + prefetch distance
 }
 
+// Value u of coefficient field f of a TBlock<T> held as 16-byte words w[f * KC + chunk]
+// (FP32: 4 floats per word, FP64: 2 doubles per word).
+template <typename T>
+__device__ __forceinline__ T coef_of(const uint4* w, int f, int u);
+template <>
+__device__ __forceinline__ float coef_of<float>(const uint4* w, int f, int u) {
+  const uint4 x = w[f * WF_KC32 + u / 4];
+  const uint32_t b = (u & 3) == 0 ? x.x : (u & 3) == 1 ? x.y : (u & 3) == 2 ? x.z : x.w;
+  return __uint_as_float(b);
+}
+template <>
+__device__ __forceinline__ double coef_of<double>(const uint4* w, int f, int u) {
+  const uint4 x = w[f * WF_KC64 + u / 2];
+  return (u & 1) == 0 ? __hiloint2double((int)x.y, (int)x.x) : __hiloint2double((int)x.w, (int)x.z);
+}
+
+// The 32-bit-aligned code pointer of a block for a lane whose first step is column -1 - gi
+// (the all-PAD region when there is no block): copy k = (1 + gi) mod 4 of the haplotype's
+// code region has column 0 at hap_off + k*(copy_len + 1), so the byte of column (-1 - gi)
+// is 4-aligned.
+template <typename T>
+__device__ __forceinline__ const uint32_t* wf_code_ptr(const WfArgs2<T>& A, bool have, const BlkDesc& d, int gi,
+                                                       int copy_len) {
+  if (!have) return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
+  const int k = (1 + gi) & 3;
+  const uint32_t col0 = d.hap_off + (uint32_t)(k * (copy_len + 1));
+  return reinterpret_cast<const uint32_t*>(A.hcodes + (col0 - 1u - (uint32_t)gi));
+}
+
 // Load a block (or nothing) into half H of a lane. Returns the 32-bit-aligned code
 // pointer for the lane's first step (column -1 - gi).
 template <int H, typename T>
 __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>& L, uint32_t tab_s, bool have,
                                                    const BlkDesc& d, T d0, int& out_idx, int gi, int copy_len) {
   constexpr int K = WfT<T>::K;
-  constexpr int PER = 16 / sizeof(T);  // values per 16-byte chunk
   if (have) {
     const uint4* __restrict__ s4 = reinterpret_cast<const uint4*>(A.tab + d.tab_blk);
     constexpr int KC = WfT<T>::KC;
-    union { uint4 u[WF_NCOEF * KC]; T v[WF_NCOEF][K]; } cw;
+    // the 4 coefficient fields as 16-byte words, unpacked value by value (no type punning)
+    uint4 cw[WF_NCOEF * KC];
 #pragma unroll
-    for (int k = 0; k < WF_NCOEF * KC; ++k) cw.u[k] = __ldg(s4 + k);
+    for (int k = 0; k < WF_NCOEF * KC; ++k) cw[k] = __ldg(s4 + k);
 #pragma unroll
     for (int k = 0; k < 5 * KC; ++k)  // prior[code][chunk]
       sts16(tab_s + 512u * k, __ldg(s4 + WF_NCOEF * KC + k));
     const int rrow = (d.flags >> WF_RROW_SHIFT) & 15;
 #pragma unroll
     for (int u = 0; u < K; ++u) {
-      L.uu[u] = set_half<H>(L.uu[u], cw.v[0][u]); L.ww[u] = set_half<H>(L.ww[u], cw.v[1][u]);
-      L.ep[u] = set_half<H>(L.ep[u], cw.v[2][u]); L.mu[u] = set_half<H>(L.mu[u], cw.v[3][u]);
+      L.uu[u] = set_half<H>(L.uu[u], coef_of<T>(cw, 0, u)); L.ww[u] = set_half<H>(L.ww[u], coef_of<T>(cw, 1, u));
+      L.ep[u] = set_half<H>(L.ep[u], coef_of<T>(cw, 2, u)); L.mu[u] = set_half<H>(L.mu[u], coef_of<T>(cw, 3, u));
       L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
       L.D[u] = set_half<H>(L.D[u], rrow == u ? d0 : (T)0);
     }
-    (void)PER;
     out_idx = (d.flags & BLK_LAST) ? d.out_idx : -1;
-    // copy k = (1 + gi) mod 4 has column 0 at hap_off + k*(copy_len + 1), so the byte
-    // of column (-1 - gi) is 4-aligned
-    const int k = (1 + gi) & 3;
-    const uint32_t col0 = d.hap_off + (uint32_t)(k * (copy_len + 1));
-    return reinterpret_cast<const uint32_t*>(A.hcodes + (col0 - 1u - (uint32_t)gi));
+    return wf_code_ptr(A, true, d, gi, copy_len);
   }
 #pragma unroll
   for (int u = 0; u < K; ++u) {
@@ -498,30 +525,20 @@ __device__ __forceinline__ unsigned long long wf_claim(const WfArgs2<T>& A, int 
 }
 
 // One warp streams through blocks [s, s+nblk) of one bin (ncols columns each). The stream's
-// block range lives in a per-warp shared-memory segment table (read at switch events only),
-// which keeps it out of the registers of the hot loop (212 instead of 218
-// registers). The table has room for a second segment: appending the next work item of the
-// same bin to a stream (one drain per stream instead of per item) was measured slower and
-// removed. Returns the next work item to run (~0: claim a new one).
+// first block s lives in a per-warp shared-memory slot (read at switch events only), which
+// keeps it out of the registers of the hot loop (212 instead of 218
+// registers).
 // kLong: the launch of the long-row bins (the only one with the ring rescale compiled in).
 template <typename T, bool kLong>
-__device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s,
-                                                        uint32_t xbuf_s, uint32_t seg_s,
-                                                        int lane,
-                                                        int64_t s, int nblk, int bin, bool trace = false) {
+__device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s, uint32_t xbuf_s,
+                                          uint32_t seg_s, int lane, int64_t s, int nblk, int bin,
+                                          bool trace = false) {
   const int ncols = bin * A.bucket;
-  // segments of the concatenated stream, kept in shared memory (warp-uniform, read at switch
-  // events only, so they do not occupy registers across the hot loop): logical blocks
-  // [curL, nblk) are physical [curS, ...), [prevL, curL) are physical [prevS, ...)
-  int64_t* seg = reinterpret_cast<int64_t*>(__cvta_shared_to_generic(seg_s));  // curS, prevS, curL, prevL
+  int64_t* seg = reinterpret_cast<int64_t*>(__cvta_shared_to_generic(seg_s));
   __syncwarp();
-  if (lane == 0) { seg[0] = s; seg[1] = s; seg[2] = 0; seg[3] = 0; }
+  if (lane == 0) seg[0] = s;
   __syncwarp();
-  const unsigned long long pending = ~0ull;
-  auto phys = [&](int b) -> int64_t {
-    const int64_t cL = seg[2];
-    return b >= cL ? seg[0] + (b - cL) : seg[1] + (b - seg[3]);
-  };
+  auto phys = [&](int b) -> int64_t { return seg[0] + b; };
   using V = typename WfT<T>::V;
   constexpr int K = WfT<T>::K;
   constexpr int PER = 16 / sizeof(T);
@@ -558,8 +575,23 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
   BlkDesc dnA, dnB;  // descriptors of the lane's next blocks (loaded one pass ahead)
   dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.n = 1; dnA.flags = 0;
   dnB = dnA;
-  if (2 * lane < nblk) dnA = A.blk[s + 2 * lane];
-  if (2 * lane + 1 < nblk) dnB = A.blk[s + 2 * lane + 1];
+  if (2 * lane < nblk) dnA = A.blk[phys(2 * lane)];
+  if (2 * lane + 1 < nblk) dnB = A.blk[phys(2 * lane + 1)];
+#if PHMM_CW_PREFETCH
+  // descriptors two passes ahead and the first two code words of the next block, so that a
+  // switch event finds its block's code words already in registers (no long-scoreboard stall
+  // on the first PRMT after a switch)
+  BlkDesc dnnA = dnA, dnnB = dnB;
+  if (2 * lane + 64 < nblk) dnnA = A.blk[phys(2 * lane + 64)];
+  if (2 * lane + 65 < nblk) dnnB = A.blk[phys(2 * lane + 65)];
+  uint32_t cwA0, cwA1, cwB0, cwB1;
+  {
+    const uint32_t* p0 = wf_code_ptr(A, 2 * lane < nblk, dnA, giA, copy_len);
+    const uint32_t* p1 = wf_code_ptr(A, 2 * lane + 1 < nblk, dnB, giB, copy_len);
+    cwA0 = __ldg(p0); cwA1 = __ldg(p0 + 1);
+    cwB0 = __ldg(p1); cwB1 = __ldg(p1 + 1);
+  }
+#endif
 #ifdef PHMM_DBG_TRACE
   int tstep = 0;
 #endif
@@ -664,12 +696,27 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
         if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
         pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
         pB = wf_load<1, T>(A, L, tabB_s, hB, dB, d0, outB, giB, copy_len);
+#if PHMM_CW_PREFETCH
+        wA_nx = cwA0; wA_nx2 = cwA1; pA += 2;
+        wB_nx = cwB0; wB_nx2 = cwB1; pB += 2;
+        dnA = dnnA;
+        dnB = dnnB;
+        {
+          const uint32_t* p0 = wf_code_ptr(A, bA + 64 < nblk, dnA, giA, copy_len);
+          const uint32_t* p1 = wf_code_ptr(A, bB + 64 < nblk, dnB, giB, copy_len);
+          cwA0 = __ldg(p0); cwA1 = __ldg(p0 + 1);
+          cwB0 = __ldg(p1); cwB1 = __ldg(p1 + 1);
+        }
+        if (bA + 128 < nblk) dnnA = A.blk[phys(bA + 128)];
+        if (bB + 128 < nblk) dnnB = A.blk[phys(bB + 128)];
+#else
         wA_nx = __ldg(pA); wA_nx2 = __ldg(pA + 1); pA += 2;
         wB_nx = __ldg(pB); wB_nx2 = __ldg(pB + 1); pB += 2;
         // prefetch the next pass's descriptors after this pass's loads are issued (a load
         // issued before the consumers of the previous prefetch would share its scoreboard)
         if (bA + 64 < nblk) dnA = A.blk[phys(bA + 64)];
         if (bB + 64 < nblk) dnB = A.blk[phys(bB + 64)];
+#endif
         if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
           T a, bb, c;
           rget<ring_packed<T, kLong>()>(ring_s, a, bb, c);
@@ -681,7 +728,6 @@ __device__ __forceinline__ unsigned long long wf_stream(const WfArgs2<T>& A, uin
       for (int k = 0; k < ngroups; ++k) group4();
     }
   }
-  return pending;
 }
 
 // The kernels are defined in wf.cu (their own translation unit, compiled with
@@ -695,7 +741,7 @@ template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_sme
   const size_t b = (size_t)2 * WF_NCODE * WfT<T>::KC * 32 * 16 +
                    (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) *
                        ring_slot_bytes<T, kLong>() +
-                   32;  // the stream's segment table (wf_stream)
+                   32;  // the stream's first block (wf_stream)
   return (b + 15) & ~(size_t)15;
 }
 template <typename T> cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm);
@@ -717,21 +763,17 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
   __syncwarp();
   const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
   const uint32_t xbuf_s = ring_s + (uint32_t)A.ring_len * ring_slot_bytes<T, kLong>();  // design A only
-  const uint32_t seg_s = (ptab_s + per_warp - 32u) & ~7u;   // the stream's segment table (last 32 B)
-  // work items of the launch, claimed from an atomic counter; a stream may append further
-  // items of its bin (wf_stream) and hands back the one it claimed but could not take
+  const uint32_t seg_s = (ptab_s + per_warp - 32u) & ~7u;   // the stream's first block (last 32 B)
+  // work items of the launch, claimed from an atomic counter
   const unsigned long long it1 = A.launch_items[1];
-  unsigned long long pending = ~0ull;
   while (true) {
-    const unsigned long long it = (pending != ~0ull) ? pending : wf_claim(A, lane);
-    pending = ~0ull;
+    const unsigned long long it = wf_claim(A, lane);
     if (it >= it1) break;
     int bin;
     int64_t s, e;
     wf_item(A, it, lane, bin, s, e);
     if (e <= s) continue;
-    pending = wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, seg_s, lane, s, (int)(e - s), bin,
-                                  it == A.launch_items[0]);
+    wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, seg_s, lane, s, (int)(e - s), bin, it == A.launch_items[0]);
     __syncwarp();
   }
 }
