@@ -173,6 +173,29 @@ phmm_status phmm_compute_batch_dev(phmm_ctx* ctx, const phmm_batch* b, double* d
  */
 phmm_status phmm_set_stream(phmm_ctx* ctx, void* cuda_stream);
 
+/*
+ * Asynchronous submission of host-buffer batches (for region-sized batches: a synchronous
+ * call costs ~0.6 ms whatever the batch size, PAPER.md's batches average 189 pairs,
+ * L24@575). phmm_submit checks the batch on the host (offsets, pair indices, sizes),
+ * copies it into the context's pinned queue and returns at once with a ticket; a worker
+ * thread of the context runs everything queued so far as ONE batch whenever it is idle
+ * (so batches submitted while a run is in flight are coalesced into the next run) and
+ * writes each batch's results to its own out_log10 / out_status, which must stay valid
+ * until phmm_wait returns for that ticket (the inputs are copied: they may be reused as
+ * soon as phmm_submit returns). Results are bitwise those of phmm_compute_batch on the same
+ * batch. phmm_wait blocks until the ticket's results are written and returns the batch's
+ * status: PHMM_OK, or the error that batch alone raises (a coalesced run that fails is
+ * re-run batch by batch; the outputs of a failed batch are untouched). A ticket can be
+ * waited for once. Other calls on the context wait while a run is in progress (the
+ * context serialises its work); phmm_destroy completes every submitted batch first.
+ * Returns PHMM_E_INVALID_ARG (NULL arguments, bad sizes or offsets, too many pairs
+ * queued), PHMM_E_INDEX, PHMM_E_OOM (pinned queue) from phmm_submit; PHMM_E_INVALID_ARG
+ * for an unknown or already-waited ticket from phmm_wait.
+ */
+phmm_status phmm_submit(phmm_ctx* ctx, const phmm_batch* b, double* out_log10, uint8_t* out_status,
+                        uint64_t* ticket);
+phmm_status phmm_wait(phmm_ctx* ctx, uint64_t ticket);
+
 /* Release the context and its device workspace. NULL-safe, idempotent per pointer. */
 void phmm_destroy(phmm_ctx* ctx);
 

@@ -8,6 +8,7 @@ namespace phmm {
 // ============================================================ prep kernels
 
 // Haplotype bases: validation only (the code regions are written by k_hap_codes_wf).
+// (Also used on the Smith-Waterman sequences.)
 __global__ void k_validate_haps(const uint8_t* __restrict__ hap, int64_t n, uint32_t* err) {
   uint32_t e = 0;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -15,31 +16,71 @@ __global__ void k_validate_haps(const uint8_t* __restrict__ hap, int64_t n, uint
   if (e) atomicOr(err, e);
 }
 
-// Read bases and qualities: validation only (the tables re-read them).
-__global__ void k_validate_reads(const uint8_t* __restrict__ rb, const uint8_t* __restrict__ q,
-                                 const uint8_t* __restrict__ qi, const uint8_t* __restrict__ qd,
-                                 const uint8_t* __restrict__ qg, int64_t n, uint32_t* err) {
+// One read base: alphabet, qualities <= 127, and the transitions out of M a distribution,
+// e(qi) + e(qd) <= 1 (reading R16; only qualities <= 3 can violate it).
+__device__ __forceinline__ uint32_t read_base_err(uint8_t b, uint8_t q, uint8_t qi, uint8_t qd, uint8_t qg) {
   uint32_t e = 0;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    if (base_code(rb[i]) == 0xffu) e |= ERR_BASE;
-    if ((q[i] | qi[i] | qd[i] | qg[i]) & 0x80u) e |= ERR_QUAL;
-    // the transitions out of M must be a distribution: e(qi) + e(qd) <= 1
-    // (reading R16); only qualities <= 3 can violate it
-    else if ((qi[i] <= 3 || qd[i] <= 3) && exp10(-(double)qi[i] / 10.0) + exp10(-(double)qd[i] / 10.0) > 1.0)
-      e |= ERR_QUAL;
-  }
-  if (e) atomicOr(err, e);
+  if (base_code(b) == 0xffu) e |= ERR_BASE;
+  if ((q | qi | qd | qg) & 0x80u) e |= ERR_QUAL;
+  else if ((qi <= 3 || qd <= 3) && exp10(-(double)qi / 10.0) + exp10(-(double)qd / 10.0) > 1.0) e |= ERR_QUAL;
+  return e;
 }
 
 // Offsets: start at 0, non-decreasing, end at total.
-__global__ void k_validate_offsets(const int64_t* __restrict__ off, int64_t n, int64_t total, uint32_t* err) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x) {
-    bool bad = false;
-    if (i == 0) bad = off[0] != 0;
-    else bad = off[i] < off[i - 1];
-    if (i == n) bad |= off[n] != total;
-    if (bad) atomicOr(err, ERR_ARG);
+__device__ __forceinline__ bool offset_bad(const int64_t* __restrict__ off, int64_t i, int64_t n, int64_t total) {
+  bool bad = (i == 0) ? off[0] != 0 : off[i] < off[i - 1];
+  if (i == n) bad |= off[n] != total;
+  return bad;
+}
+
+// The whole batch in one launch: every haplotype base, every read base with its four
+// qualities (4 bases per thread-step through 32-bit words where the five arrays share their
+// alignment), and both offset arrays. Errors are OR-ed into *err (one atomic per warp).
+__global__ void k_validate(const uint8_t* __restrict__ hap, int64_t n_hb, const uint8_t* __restrict__ rb,
+                           const uint8_t* __restrict__ q, const uint8_t* __restrict__ qi,
+                           const uint8_t* __restrict__ qd, const uint8_t* __restrict__ qg, int64_t n_rb,
+                           const int64_t* __restrict__ roff, int64_t n_reads, const int64_t* __restrict__ hoff,
+                           int64_t n_haps, uint32_t* err) {
+  uint32_t e = 0;
+  const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, nthr = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = tid; i < n_hb; i += nthr)
+    if (base_code(hap[i]) == 0xffu) e |= ERR_BASE;
+  // reads: a scalar head up to the first 4-aligned read byte, then words (when all five
+  // arrays are equally aligned), then a scalar tail
+  const uintptr_t mis = (uintptr_t)rb & 3;
+  const bool same = (((uintptr_t)q & 3) == mis) && (((uintptr_t)qi & 3) == mis) && (((uintptr_t)qd & 3) == mis) &&
+                    (((uintptr_t)qg & 3) == mis);
+  const int64_t head = same ? min(n_rb, (int64_t)((4 - mis) & 3)) : n_rb;
+  for (int64_t i = tid; i < head; i += nthr) e |= read_base_err(rb[i], q[i], qi[i], qd[i], qg[i]);
+  const int64_t nw = (n_rb - head) >> 2;
+  const uint32_t *rb4 = reinterpret_cast<const uint32_t*>(rb + head), *q4 = reinterpret_cast<const uint32_t*>(q + head),
+                 *i4 = reinterpret_cast<const uint32_t*>(qi + head), *d4 = reinterpret_cast<const uint32_t*>(qd + head),
+                 *g4 = reinterpret_cast<const uint32_t*>(qg + head);
+  for (int64_t w = tid; w < nw; w += nthr) {
+    const uint32_t b = rb4[w], a = q4[w], x = i4[w], y = d4[w], z = g4[w];
+    // fast path: every byte an uppercase base letter candidate and no quality byte >= 128 or <= 3
+    if (((a | x | y | z) & 0x80808080u) || __vcmpleu4(x, 0x03030303u) || __vcmpleu4(y, 0x03030303u)) {
+      for (int k = 0; k < 4; ++k)
+        e |= read_base_err((uint8_t)(b >> 8 * k), (uint8_t)(a >> 8 * k), (uint8_t)(x >> 8 * k),
+                           (uint8_t)(y >> 8 * k), (uint8_t)(z >> 8 * k));
+    } else {
+      for (int k = 0; k < 4; ++k)
+        if (base_code((uint8_t)(b >> 8 * k)) == 0xffu) e |= ERR_BASE;
+    }
   }
+  for (int64_t i = head + 4 * nw + tid; i < n_rb; i += nthr) e |= read_base_err(rb[i], q[i], qi[i], qd[i], qg[i]);
+  for (int64_t i = tid; i <= n_reads; i += nthr)
+    if (offset_bad(roff, i, n_reads, n_rb)) e |= ERR_ARG;
+  for (int64_t i = tid; i <= n_haps; i += nthr)
+    if (offset_bad(hoff, i, n_haps, n_hb)) e |= ERR_ARG;
+  e = __reduce_or_sync(0xffffffffu, e);
+  if (e && (threadIdx.x & 31) == 0) atomicOr(err, e);
+}
+
+// Offsets (the Smith-Waterman batch): start at 0, non-decreasing, end at total.
+__global__ void k_validate_offsets(const int64_t* __restrict__ off, int64_t n, int64_t total, uint32_t* err) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
+    if (offset_bad(off, i, n, total)) atomicOr(err, ERR_ARG);
 }
 
 // Per pair: validate indices/lengths, bin by column count, count blocks per bin.

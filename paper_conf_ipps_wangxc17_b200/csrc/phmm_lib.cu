@@ -14,6 +14,12 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <condition_variable>
+#include <map>
+#include <set>
+#include <mutex>
+#include <thread>
+#include <vector>
 #include <new>
 
 #include "../../include/phmm.h"
@@ -46,6 +52,8 @@ struct Buf {
   void* p = nullptr;
   size_t n = 0;
 };
+
+struct AsyncQueue;
 
 // device scalars written by the prep kernels, read back in one D2H copy
 struct Scalars {
@@ -85,6 +93,10 @@ struct phmm_ctx {
   int64_t sw_ops_cap = 0;         // last SW call: sum over tasks of M + N
   cudaEvent_t ev[kEvents] = {};
   Stager stage;                           // host variant: pinned staging of pageable buffers
+  std::map<uint64_t, int> occ;            // wavefront occupancy per (precision, launch class, warps, smem)
+  std::mutex run_mu;                      // one compute at a time (caller threads and the submit worker)
+  AsyncQueue* aq = nullptr;               // phmm_submit / phmm_wait (created on first submit)
+  size_t sw_smem_set = 0;                 // dynamic shared memory the SW fill kernel is allowed
   phmm_stats st{};
   PhaseMs acc{};                          // per-phase times summed over a call's chunks
   int launches = 0;
@@ -202,19 +214,27 @@ phmm_status run_validate(phmm_ctx* c, const DevBatch& d) {
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
-  if (d.n_hb > 0) {
-    k_validate_haps<<<grid_for(c, d.n_hb), kThreads, 0, s>>>(d.hap, d.n_hb, &scal->err);
-    LAUNCHED(c);
-  }
-  if (d.n_rb > 0) {
-    k_validate_reads<<<grid_for(c, d.n_rb), kThreads, 0, s>>>(d.rb, d.q, d.qi, d.qd, d.qg, d.n_rb, &scal->err);
-    LAUNCHED(c);
-  }
-  k_validate_offsets<<<grid_for(c, d.n_reads + 1), kThreads, 0, s>>>(d.roff, d.n_reads, d.n_rb, &scal->err);
-  LAUNCHED(c);
-  k_validate_offsets<<<grid_for(c, d.n_haps + 1), kThreads, 0, s>>>(d.hoff, d.n_haps, d.n_hb, &scal->err);
+  const int64_t work = std::max(std::max(d.n_hb, d.n_rb / 4), std::max(d.n_reads, d.n_haps) + 1);
+  k_validate<<<grid_for(c, work), kThreads, 0, s>>>(d.hap, d.n_hb, d.rb, d.q, d.qi, d.qd, d.qg, d.n_rb, d.roff,
+                                                    d.n_reads, d.hoff, d.n_haps, &scal->err);
   LAUNCHED(c);
   return PHMM_OK;
+}
+
+// Blocks per SM of a wavefront kernel configuration, cached per context (the occupancy
+// calculator costs microseconds per query, a small batch asks a few times per call).
+template <typename T>
+cudaError_t occupancy(phmm_ctx* c, bool long_rows, int warps, size_t smem, int* bps) {
+  const uint64_t key = ((uint64_t)smem << 16) | ((uint64_t)warps << 2) | ((uint64_t)long_rows << 1) |
+                       (uint64_t)(sizeof(T) == 8);
+  auto it = c->occ.find(key);
+  if (it != c->occ.end()) {
+    *bps = it->second;
+    return cudaSuccess;
+  }
+  cudaError_t e = wf_occupancy<T>(long_rows, warps, smem, bps);
+  if (e == cudaSuccess) c->occ[key] = *bps;
+  return e;
 }
 
 // Part 1 of a pass: bin the pairs, size the coefficient table (and, with
@@ -386,7 +406,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   auto P_of = [](int ncols) { return wf_pass_len(ncols); };
   const int p_max = P_of(pi.max_ncols);
   int bps_full = 0;
-  CUDA_TRY(wf_occupancy<T>(false, WF_WARPS, wf_warp_smem<T>(wf_pass_len(0) + 4) * WF_WARPS, &bps_full));
+  CUDA_TRY(occupancy<T>(c, false, WF_WARPS, wf_warp_smem<T>(wf_pass_len(0) + 4) * WF_WARPS, &bps_full));
   if (bps_full < 1) return PHMM_E_CUDA;
   const int64_t cta_budget = (int64_t)c->smem_per_sm / bps_full - c->smem_reserved;
   const int ring_full = (int)std::min<int64_t>(
@@ -411,7 +431,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
       const size_t sm = wf_warp_smem<T, true>(lb.ring_len) * w;
       if (sm > (size_t)c->smem_optin) continue;
       int b = 0;
-      CUDA_TRY(wf_occupancy<T>(true, w, sm, &b));
+      CUDA_TRY(occupancy<T>(c, true, w, sm, &b));
       if (b * w > best) { best = b * w; lb.warps = w; lb.bps = b; }
     }
     if (best < 1) return PHMM_E_INVALID_ARG;  // cannot happen for ncols <= kMaxHapLen + 8
@@ -834,188 +854,7 @@ void finish_stats(phmm_ctx* c) {
   }
 }
 
-}  // namespace
-
-extern "C" {
-
-int phmm_abi_version(void) { return PHMM_ABI_VERSION; }
-
-
-
-const char* phmm_status_string(phmm_status s) {
-  switch (s) {
-    case PHMM_OK: return "ok";
-    case PHMM_E_INVALID_ARG: return "invalid argument";
-    case PHMM_E_INVALID_BASE: return "invalid base (expected A, C, G, T or N)";
-    case PHMM_E_INVALID_QUAL: return "invalid quality (> 127)";
-    case PHMM_E_EMPTY_SEQ: return "empty read or haplotype";
-    case PHMM_E_INDEX: return "pair index out of range";
-    case PHMM_E_CUDA: return "CUDA error";
-    case PHMM_E_OOM: return "out of memory";
-  }
-  return "unknown status";
-}
-
-phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
-  if (!out) return PHMM_E_INVALID_ARG;
-  *out = nullptr;
-  phmm_config def{};
-  def.device = 0;
-  def.precision = PHMM_PREC_FP32_RESCUE;
-  def.cuda_stream = nullptr;
-  def.flags = 0;
-  def.col_bucket = 0;
-  if (!cfg) cfg = &def;
-  if (cfg->precision != PHMM_PREC_FP64 && cfg->precision != PHMM_PREC_FP32_RESCUE) return PHMM_E_INVALID_ARG;
-  if (cfg->col_bucket < 0 || cfg->col_bucket > 64) return PHMM_E_INVALID_ARG;
-  int ndev = 0;
-  if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
-    cudaGetLastError();
-    return PHMM_E_CUDA;
-  }
-  if (cfg->device < 0 || cfg->device >= ndev) return PHMM_E_INVALID_ARG;
-  phmm_ctx* c = new (std::nothrow) phmm_ctx();
-  if (!c) return PHMM_E_OOM;
-  c->device = cfg->device;
-  c->prec = cfg->precision;
-  c->flags = cfg->flags;
-  c->bucket = cfg->col_bucket > 0 ? cfg->col_bucket : 4;
-  auto fail = [&](phmm_status s) {
-    phmm_destroy(c);
-    return s;
-  };
-  if (cudaSetDevice(c->device) != cudaSuccess) return fail(PHMM_E_CUDA);
-  if (cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess ||
-      cudaDeviceGetAttribute(&c->smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device) !=
-          cudaSuccess ||
-      cudaDeviceGetAttribute(&c->smem_reserved, cudaDevAttrReservedSharedMemoryPerBlock, c->device) !=
-          cudaSuccess ||
-      cudaDeviceGetAttribute(&c->smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, c->device) != cudaSuccess)
-    return fail(PHMM_E_CUDA);
-  if (cfg->cuda_stream) {
-    c->stream = reinterpret_cast<cudaStream_t>(cfg->cuda_stream);
-  } else {
-    if (cudaStreamCreateWithFlags(&c->owned_stream, cudaStreamNonBlocking) != cudaSuccess) {
-      c->owned_stream = nullptr;
-      return fail(PHMM_E_CUDA);
-    }
-    c->stream = c->owned_stream;
-  }
-  if (cudaMallocHost(&c->host_scal, sizeof(Scalars)) != cudaSuccess) {
-    c->host_scal = nullptr;
-    return fail(PHMM_E_OOM);
-  }
-  if (cudaMallocHost(&c->host_sizes, 2 * sizeof(int64_t)) != cudaSuccess) {
-    c->host_sizes = nullptr;
-    return fail(PHMM_E_OOM);
-  }
-  for (int i = 0; i < kEvents; ++i)
-    if (cudaEventCreate(&c->ev[i]) != cudaSuccess) return fail(PHMM_E_CUDA);
-  {
-    int threads = (int)std::min(8u, std::max(1u, std::thread::hardware_concurrency() / 2));
-    if (const char* e = std::getenv("PHMM_STAGE_THREADS")) threads = std::max(1, std::min(64, std::atoi(e)));
-    if (c->stage.init(threads) != cudaSuccess) {
-      cudaGetLastError();
-      return fail(PHMM_E_OOM);
-    }
-  }
-  if (const char* e = std::getenv("PHMM_CHUNK_PAIRS")) c->chunk_pairs = std::max<int64_t>(64, std::atoll(e));
-  *out = c;
-  return PHMM_OK;
-}
-
-void phmm_destroy(phmm_ctx* c) {
-  if (!c) return;
-  cudaSetDevice(c->device);
-  if (c->stream) cudaStreamSynchronize(c->stream);
-  for (int i = 0; i < B_COUNT; ++i)
-    if (c->buf[i].p) cudaFree(c->buf[i].p);
-  for (int i = 0; i < kEvents; ++i)
-    if (c->ev[i]) cudaEventDestroy(c->ev[i]);
-  c->stage.release();
-  if (c->host_scal) cudaFreeHost(c->host_scal);
-  if (c->host_sizes) cudaFreeHost(c->host_sizes);
-  if (c->host_ranges) cudaFreeHost(c->host_ranges);
-  if (c->owned_stream) {
-    cudaStreamSynchronize(c->owned_stream);
-    cudaStreamDestroy(c->owned_stream);
-  }
-  cudaGetLastError();
-  delete c;
-}
-
-phmm_status phmm_get_stats(const phmm_ctx* c, phmm_stats* out) {
-  if (!c || !out) return PHMM_E_INVALID_ARG;
-  *out = c->st;
-  return PHMM_OK;
-}
-
-phmm_status phmm_set_stream(phmm_ctx* c, void* stream) {
-  if (!c) return PHMM_E_INVALID_ARG;
-  if (cudaSetDevice(c->device) != cudaSuccess) {
-    cudaGetLastError();
-    return PHMM_E_CUDA;
-  }
-  cudaStream_t s = stream ? reinterpret_cast<cudaStream_t>(stream) : c->owned_stream;
-  if (!s) {  // created on a caller's stream: make a private one for the NULL case
-    if (cudaStreamCreateWithFlags(&c->owned_stream, cudaStreamNonBlocking) != cudaSuccess) {
-      cudaGetLastError();
-      c->owned_stream = nullptr;
-      return PHMM_E_CUDA;
-    }
-    s = c->owned_stream;
-  }
-  c->stream = s;
-  return PHMM_OK;
-}
-
-phmm_status phmm_compute_batch_dev(phmm_ctx* c, const phmm_batch* b, double* dev_out, uint8_t* dev_status) {
-  if (!c) return PHMM_E_INVALID_ARG;
-  ST_TRY(check_batch_args(b));
-  if (b->n_pairs > 0 && !dev_out) return PHMM_E_INVALID_ARG;
-  if (cudaSetDevice(c->device) != cudaSuccess) {
-    cudaGetLastError();
-    return PHMM_E_CUDA;
-  }
-  c->launches = 0;
-  DevBatch d{b->read_bases, b->base_quals, b->ins_quals, b->del_quals, b->gcp_quals, b->hap_bases,
-             b->read_offsets, b->hap_offsets, b->pairs, b->n_reads, b->n_haps, b->n_pairs,
-             b->total_read_bases, b->total_hap_bases};
-  // results go to context scratch first and reach the caller's buffers only after the
-  // whole path (FP32 pass and FP64 rescue) succeeded: outputs stay untouched on error
-  double* out = nullptr;
-  uint8_t* status = nullptr;
-  if (b->n_pairs > 0) {
-    ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
-    if (dev_status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
-  }
-  ev_record(c, EV_START);
-  ev_record(c, EV_H2D);
-  phmm_status st = compute_dev(c, d, out, status);
-  if (st != PHMM_OK) {
-    cudaStreamSynchronize(c->stream);
-    cudaGetLastError();
-    return st;
-  }
-  if (b->n_pairs > 0) {
-    CUDA_TRY(cudaMemcpyAsync(dev_out, out, sizeof(double) * (size_t)b->n_pairs, cudaMemcpyDeviceToDevice,
-                             c->stream));
-    if (dev_status)
-      CUDA_TRY(cudaMemcpyAsync(dev_status, status, (size_t)b->n_pairs, cudaMemcpyDeviceToDevice, c->stream));
-  }
-  ev_record(c, EV_END);
-  if (cudaStreamSynchronize(c->stream) != cudaSuccess) {
-    cudaGetLastError();
-    return PHMM_E_CUDA;
-  }
-  finish_stats(c);
-  c->st.ms_h2d = 0.f;
-  c->st.ms_d2h = 0.f;
-  return PHMM_OK;
-}
-
-phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status) {
-  if (!c) return PHMM_E_INVALID_ARG;
+phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status) {
   ST_TRY(check_batch_args(b));
   if (b->n_pairs > 0 && !out_log10) return PHMM_E_INVALID_ARG;
   if (cudaSetDevice(c->device) != cudaSuccess) {
@@ -1082,9 +921,458 @@ phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log
   return PHMM_OK;
 }
 
+
+// ------------------------------------------------------------ phmm_submit / phmm_wait
+// Region-sized batches (~189 pairs in the paper, L24@575) cost ~0.6 ms per synchronous call
+// however small they are (launches and size read-backs), so the library offers a submission
+// queue: phmm_submit appends a batch to a pinned ARENA (inputs gathered back to back, offsets
+// and pair indices rebased) and returns a ticket at once; a worker thread takes the whole
+// arena whenever it is idle and runs it as ONE batch (compute_host), while later submissions
+// fill the other arena; then it copies each batch's results to its caller's buffers. Results
+// are bitwise those of separate calls (a pair's arithmetic never depends on its batch, R14).
+// If the coalesced run fails (an input-content error in one of the batches), every batch of
+// that run is re-run on its own, so each ticket gets its own status.
+struct AsyncJob {
+  uint64_t ticket;
+  int64_t p0, np, r0, nr, h0, nh, rb0, nrb, hb0, nhb;  // the batch's place in its arena
+  double* out;
+  uint8_t* status;
+};
+
+struct PinnedVec {  // growable page-locked byte buffer
+  uint8_t* p = nullptr;
+  size_t n = 0, cap = 0;
+  bool reserve(size_t want) {
+    if (want <= cap) return true;
+    size_t c2 = std::max(want, cap * 2 + ((size_t)1 << 20));
+    uint8_t* q = nullptr;
+    if (cudaHostAlloc(reinterpret_cast<void**>(&q), c2, cudaHostAllocPortable) != cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    if (n) std::memcpy(q, p, n);
+    if (p) cudaFreeHost(p);
+    p = q;
+    cap = c2;
+    return true;
+  }
+  void release() {
+    if (p) cudaFreeHost(p);
+    p = nullptr;
+    n = cap = 0;
+  }
+};
+
+struct Arena {
+  PinnedVec rb, q, qi, qd, qg, hb, roff, hoff, pairs, out, st;
+  std::vector<AsyncJob> jobs;
+  int64_t n_reads = 0, n_haps = 0, n_pairs = 0;
+  bool any_status = false;
+  void clear() {
+    for (PinnedVec* v : {&rb, &q, &qi, &qd, &qg, &hb, &roff, &hoff, &pairs, &out, &st}) v->n = 0;
+    jobs.clear();
+    n_reads = n_haps = n_pairs = 0;
+    any_status = false;
+  }
+  void release() {
+    for (PinnedVec* v : {&rb, &q, &qi, &qd, &qg, &hb, &roff, &hoff, &pairs, &out, &st}) v->release();
+  }
+};
+
+struct AsyncQueue {
+  std::mutex mu;
+  std::condition_variable cv, done_cv;
+  Arena arena[2];
+  int fill = 0;              // the arena submissions append to
+  bool stop = false, busy = false;
+  uint64_t next_ticket = 1;
+  std::map<uint64_t, phmm_status> done;  // finished tickets not yet waited for
+  std::set<uint64_t> outstanding;        // submitted tickets not yet waited for
+  std::thread worker;
+};
+
+void run_arena(phmm_ctx* c, Arena& A) {
+  std::vector<phmm_status> st(A.jobs.size(), PHMM_OK);
+  auto batch_of = [&](int64_t r0, int64_t nr, int64_t h0, int64_t nh, int64_t p0, int64_t np, int64_t rb0,
+                      int64_t hb0, std::vector<int64_t>* ro, std::vector<int64_t>* ho, std::vector<int32_t>* pr) {
+    phmm_batch b{};
+    const int64_t* aro = reinterpret_cast<const int64_t*>(A.roff.p);
+    const int64_t* aho = reinterpret_cast<const int64_t*>(A.hoff.p);
+    const int32_t* apr = reinterpret_cast<const int32_t*>(A.pairs.p);
+    ro->resize(nr + 1);
+    ho->resize(nh + 1);
+    pr->resize(2 * np);
+    for (int64_t i = 0; i <= nr; ++i) (*ro)[i] = aro[r0 + i] - rb0;
+    for (int64_t i = 0; i <= nh; ++i) (*ho)[i] = aho[h0 + i] - hb0;
+    for (int64_t i = 0; i < np; ++i) {
+      (*pr)[2 * i] = apr[2 * (p0 + i)] - (int32_t)r0;
+      (*pr)[2 * i + 1] = apr[2 * (p0 + i) + 1] - (int32_t)h0;
+    }
+    b.read_bases = A.rb.p + rb0; b.base_quals = A.q.p + rb0; b.ins_quals = A.qi.p + rb0;
+    b.del_quals = A.qd.p + rb0; b.gcp_quals = A.qg.p + rb0; b.hap_bases = A.hb.p + hb0;
+    b.read_offsets = ro->data(); b.hap_offsets = ho->data(); b.pairs = pr->data();
+    b.n_reads = nr; b.n_haps = nh; b.n_pairs = np;
+    b.total_read_bases = (*ro)[nr];
+    b.total_hap_bases = (*ho)[nh];
+    return b;
+  };
+  phmm_status all = PHMM_OK;
+  {
+    phmm_batch b{};
+    b.read_bases = A.rb.p; b.base_quals = A.q.p; b.ins_quals = A.qi.p; b.del_quals = A.qd.p; b.gcp_quals = A.qg.p;
+    b.read_offsets = reinterpret_cast<const int64_t*>(A.roff.p); b.n_reads = A.n_reads;
+    b.hap_bases = A.hb.p; b.hap_offsets = reinterpret_cast<const int64_t*>(A.hoff.p); b.n_haps = A.n_haps;
+    b.pairs = reinterpret_cast<const int32_t*>(A.pairs.p); b.n_pairs = A.n_pairs;
+    b.total_read_bases = (int64_t)A.rb.n; b.total_hap_bases = (int64_t)A.hb.n;
+    std::lock_guard<std::mutex> g(c->run_mu);
+    all = compute_host(c, &b, reinterpret_cast<double*>(A.out.p), A.any_status ? A.st.p : nullptr);
+  }
+  if (all != PHMM_OK) {  // attribute the failure: every batch of the run on its own
+    std::vector<int64_t> ro, ho;
+    std::vector<int32_t> pr;
+    for (size_t k = 0; k < A.jobs.size(); ++k) {
+      const AsyncJob& j = A.jobs[k];
+      phmm_batch b = batch_of(j.r0, j.nr, j.h0, j.nh, j.p0, j.np, j.rb0, j.hb0, &ro, &ho, &pr);
+      std::lock_guard<std::mutex> g(c->run_mu);
+      st[k] = compute_host(c, &b, reinterpret_cast<double*>(A.out.p) + j.p0, A.any_status ? A.st.p + j.p0 : nullptr);
+    }
+  }
+  for (size_t k = 0; k < A.jobs.size(); ++k) {
+    const AsyncJob& j = A.jobs[k];
+    if (st[k] != PHMM_OK || j.np == 0) continue;
+    std::memcpy(j.out, reinterpret_cast<double*>(A.out.p) + j.p0, sizeof(double) * (size_t)j.np);
+    if (j.status) std::memcpy(j.status, A.st.p + j.p0, (size_t)j.np);
+  }
+  AsyncQueue* q = c->aq;
+  std::lock_guard<std::mutex> g(q->mu);
+  for (size_t k = 0; k < A.jobs.size(); ++k) q->done[A.jobs[k].ticket] = st[k];
+  q->done_cv.notify_all();
+}
+
+void async_worker(phmm_ctx* c) {
+  AsyncQueue* q = c->aq;
+  cudaSetDevice(c->device);
+  while (true) {
+    int k;
+    {
+      std::unique_lock<std::mutex> lk(q->mu);
+      q->cv.wait(lk, [&] { return q->stop || !q->arena[q->fill].jobs.empty(); });
+      if (q->arena[q->fill].jobs.empty()) return;  // stop, nothing left
+      k = q->fill;
+      q->fill ^= 1;  // submissions go to the other arena while this one runs
+      q->busy = true;
+    }
+    run_arena(c, q->arena[k]);
+    std::lock_guard<std::mutex> g(q->mu);
+    q->arena[k].clear();
+    q->busy = false;
+    q->done_cv.notify_all();
+  }
+}
+
+void async_stop(phmm_ctx* c) {
+  AsyncQueue* q = c->aq;
+  if (!q) return;
+  {
+    std::lock_guard<std::mutex> g(q->mu);
+    q->stop = true;
+  }
+  q->cv.notify_all();
+  if (q->worker.joinable()) q->worker.join();
+  q->arena[0].release();
+  q->arena[1].release();
+  delete q;
+  c->aq = nullptr;
+}
+
+// host-side checks of a submitted batch (the device checks the contents when it runs)
+phmm_status submit_checks(const phmm_batch* b) {
+  ST_TRY(check_batch_args(b));
+  if (b->n_pairs == 0) return PHMM_OK;
+  const int64_t* ro = b->read_offsets;
+  const int64_t* ho = b->hap_offsets;
+  if (ro[0] != 0 || ho[0] != 0 || ro[b->n_reads] != b->total_read_bases || ho[b->n_haps] != b->total_hap_bases)
+    return PHMM_E_INVALID_ARG;
+  for (int64_t i = 0; i < b->n_reads; ++i)
+    if (ro[i + 1] < ro[i]) return PHMM_E_INVALID_ARG;
+  for (int64_t i = 0; i < b->n_haps; ++i)
+    if (ho[i + 1] < ho[i]) return PHMM_E_INVALID_ARG;
+  for (int64_t p = 0; p < b->n_pairs; ++p) {
+    const int32_t r = b->pairs[2 * p], h = b->pairs[2 * p + 1];
+    if (r < 0 || r >= b->n_reads || h < 0 || h >= b->n_haps) return PHMM_E_INDEX;
+  }
+  return PHMM_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int phmm_abi_version(void) { return PHMM_ABI_VERSION; }
+
+
+
+const char* phmm_status_string(phmm_status s) {
+  switch (s) {
+    case PHMM_OK: return "ok";
+    case PHMM_E_INVALID_ARG: return "invalid argument";
+    case PHMM_E_INVALID_BASE: return "invalid base (expected A, C, G, T or N)";
+    case PHMM_E_INVALID_QUAL: return "invalid quality (> 127)";
+    case PHMM_E_EMPTY_SEQ: return "empty read or haplotype";
+    case PHMM_E_INDEX: return "pair index out of range";
+    case PHMM_E_CUDA: return "CUDA error";
+    case PHMM_E_OOM: return "out of memory";
+  }
+  return "unknown status";
+}
+
+phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
+  if (!out) return PHMM_E_INVALID_ARG;
+  *out = nullptr;
+  phmm_config def{};
+  def.device = 0;
+  def.precision = PHMM_PREC_FP32_RESCUE;
+  def.cuda_stream = nullptr;
+  def.flags = 0;
+  def.col_bucket = 0;
+  if (!cfg) cfg = &def;
+  if (cfg->precision != PHMM_PREC_FP64 && cfg->precision != PHMM_PREC_FP32_RESCUE) return PHMM_E_INVALID_ARG;
+  if (cfg->col_bucket < 0 || cfg->col_bucket > 64) return PHMM_E_INVALID_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) return PHMM_E_INVALID_ARG;
+  phmm_ctx* c = new (std::nothrow) phmm_ctx();
+  if (!c) return PHMM_E_OOM;
+  c->device = cfg->device;
+  c->prec = cfg->precision;
+  c->flags = cfg->flags;
+  c->bucket = cfg->col_bucket > 0 ? cfg->col_bucket : 4;
+  auto fail = [&](phmm_status s) {
+    phmm_destroy(c);
+    return s;
+  };
+  if (cudaSetDevice(c->device) != cudaSuccess) return fail(PHMM_E_CUDA);
+  if (cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device) != cudaSuccess ||
+      cudaDeviceGetAttribute(&c->smem_per_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, c->device) !=
+          cudaSuccess ||
+      cudaDeviceGetAttribute(&c->smem_reserved, cudaDevAttrReservedSharedMemoryPerBlock, c->device) !=
+          cudaSuccess ||
+      cudaDeviceGetAttribute(&c->smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, c->device) != cudaSuccess)
+    return fail(PHMM_E_CUDA);
+  if (wf_set_max_smem(c->smem_optin) != cudaSuccess) return fail(PHMM_E_CUDA);
+  if (cfg->cuda_stream) {
+    c->stream = reinterpret_cast<cudaStream_t>(cfg->cuda_stream);
+  } else {
+    if (cudaStreamCreateWithFlags(&c->owned_stream, cudaStreamNonBlocking) != cudaSuccess) {
+      c->owned_stream = nullptr;
+      return fail(PHMM_E_CUDA);
+    }
+    c->stream = c->owned_stream;
+  }
+  if (cudaMallocHost(&c->host_scal, sizeof(Scalars)) != cudaSuccess) {
+    c->host_scal = nullptr;
+    return fail(PHMM_E_OOM);
+  }
+  if (cudaMallocHost(&c->host_sizes, 2 * sizeof(int64_t)) != cudaSuccess) {
+    c->host_sizes = nullptr;
+    return fail(PHMM_E_OOM);
+  }
+  for (int i = 0; i < kEvents; ++i)
+    if (cudaEventCreate(&c->ev[i]) != cudaSuccess) return fail(PHMM_E_CUDA);
+  {
+    int threads = (int)std::min(8u, std::max(1u, std::thread::hardware_concurrency() / 2));
+    if (const char* e = std::getenv("PHMM_STAGE_THREADS")) threads = std::max(1, std::min(64, std::atoi(e)));
+    if (c->stage.init(threads) != cudaSuccess) {
+      cudaGetLastError();
+      return fail(PHMM_E_OOM);
+    }
+  }
+  if (const char* e = std::getenv("PHMM_CHUNK_PAIRS")) c->chunk_pairs = std::max<int64_t>(64, std::atoll(e));
+  *out = c;
+  return PHMM_OK;
+}
+
+void phmm_destroy(phmm_ctx* c) {
+  if (!c) return;
+  async_stop(c);  // finishes every submitted batch first
+  cudaSetDevice(c->device);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  for (int i = 0; i < B_COUNT; ++i)
+    if (c->buf[i].p) cudaFree(c->buf[i].p);
+  for (int i = 0; i < kEvents; ++i)
+    if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  c->stage.release();
+  if (c->host_scal) cudaFreeHost(c->host_scal);
+  if (c->host_sizes) cudaFreeHost(c->host_sizes);
+  if (c->host_ranges) cudaFreeHost(c->host_ranges);
+  if (c->owned_stream) {
+    cudaStreamSynchronize(c->owned_stream);
+    cudaStreamDestroy(c->owned_stream);
+  }
+  cudaGetLastError();
+  delete c;
+}
+
+phmm_status phmm_get_stats(const phmm_ctx* c, phmm_stats* out) {
+  if (!c || !out) return PHMM_E_INVALID_ARG;
+  *out = c->st;
+  return PHMM_OK;
+}
+
+phmm_status phmm_set_stream(phmm_ctx* c, void* stream) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  std::lock_guard<std::mutex> g_(c->run_mu);
+  if (cudaSetDevice(c->device) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  cudaStream_t s = stream ? reinterpret_cast<cudaStream_t>(stream) : c->owned_stream;
+  if (!s) {  // created on a caller's stream: make a private one for the NULL case
+    if (cudaStreamCreateWithFlags(&c->owned_stream, cudaStreamNonBlocking) != cudaSuccess) {
+      cudaGetLastError();
+      c->owned_stream = nullptr;
+      return PHMM_E_CUDA;
+    }
+    s = c->owned_stream;
+  }
+  c->stream = s;
+  return PHMM_OK;
+}
+
+
+phmm_status phmm_submit(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status, uint64_t* ticket) {
+  if (!c || !ticket) return PHMM_E_INVALID_ARG;
+  ST_TRY(submit_checks(b));
+  if (b->n_pairs > 0 && !out_log10) return PHMM_E_INVALID_ARG;
+  if (!c->aq) {
+    c->aq = new (std::nothrow) AsyncQueue();
+    if (!c->aq) return PHMM_E_OOM;
+    c->aq->worker = std::thread(async_worker, c);
+  }
+  AsyncQueue* q = c->aq;
+  std::lock_guard<std::mutex> g(q->mu);
+  if (q->stop) return PHMM_E_INVALID_ARG;
+  Arena& A = q->arena[q->fill];
+  const int64_t np = b->n_pairs, nr = b->n_reads, nh = b->n_haps;
+  if (A.n_pairs + np > 0x7fffffffLL || A.n_reads + nr > 0x7fffffffLL || A.n_haps + nh > 0x7fffffffLL)
+    return PHMM_E_INVALID_ARG;  // wait for some tickets first
+  AsyncJob j{q->next_ticket, A.n_pairs, np, A.n_reads, nr, A.n_haps, nh, (int64_t)A.rb.n, b->total_read_bases,
+             (int64_t)A.hb.n, b->total_hap_bases, out_log10, out_status};
+  const size_t nrb = (size_t)b->total_read_bases, nhb = (size_t)b->total_hap_bases;
+  const bool first = A.jobs.empty();
+  // the arena's offset arrays hold n + 1 entries (a leading 0)
+  if (!A.rb.reserve(A.rb.n + nrb) || !A.q.reserve(A.q.n + nrb) || !A.qi.reserve(A.qi.n + nrb) ||
+      !A.qd.reserve(A.qd.n + nrb) || !A.qg.reserve(A.qg.n + nrb) || !A.hb.reserve(A.hb.n + nhb) ||
+      !A.roff.reserve(A.roff.n + 8 * (size_t)(nr + 1)) || !A.hoff.reserve(A.hoff.n + 8 * (size_t)(nh + 1)) ||
+      !A.pairs.reserve(A.pairs.n + 8 * (size_t)np) || !A.out.reserve(8 * (size_t)(A.n_pairs + np)) ||
+      !A.st.reserve((size_t)(A.n_pairs + np)))
+    return PHMM_E_OOM;
+  auto app = [](PinnedVec& v, const void* src, size_t n) {
+    if (n) std::memcpy(v.p + v.n, src, n);
+    v.n += n;
+  };
+  app(A.rb, b->read_bases, nrb); app(A.q, b->base_quals, nrb); app(A.qi, b->ins_quals, nrb);
+  app(A.qd, b->del_quals, nrb); app(A.qg, b->gcp_quals, nrb); app(A.hb, b->hap_bases, nhb);
+  if (first) {
+    const int64_t zero = 0;
+    app(A.roff, &zero, 8);
+    app(A.hoff, &zero, 8);
+  }
+  int64_t* ro = reinterpret_cast<int64_t*>(A.roff.p + A.roff.n);
+  for (int64_t i = 1; i <= nr; ++i) ro[i - 1] = b->read_offsets[i] + j.rb0;
+  A.roff.n += 8 * (size_t)nr;
+  int64_t* ho = reinterpret_cast<int64_t*>(A.hoff.p + A.hoff.n);
+  for (int64_t i = 1; i <= nh; ++i) ho[i - 1] = b->hap_offsets[i] + j.hb0;
+  A.hoff.n += 8 * (size_t)nh;
+  int32_t* pr = reinterpret_cast<int32_t*>(A.pairs.p + A.pairs.n);
+  for (int64_t p = 0; p < np; ++p) {
+    pr[2 * p] = b->pairs[2 * p] + (int32_t)j.r0;
+    pr[2 * p + 1] = b->pairs[2 * p + 1] + (int32_t)j.h0;
+  }
+  A.pairs.n += 8 * (size_t)np;
+  A.n_pairs += np;
+  A.n_reads += nr;
+  A.n_haps += nh;
+  A.any_status |= out_status != nullptr;
+  A.jobs.push_back(j);
+  q->outstanding.insert(j.ticket);
+  *ticket = q->next_ticket++;
+  q->cv.notify_one();
+  return PHMM_OK;
+}
+
+phmm_status phmm_wait(phmm_ctx* c, uint64_t ticket) {
+  if (!c || !c->aq) return PHMM_E_INVALID_ARG;
+  AsyncQueue* q = c->aq;
+  std::unique_lock<std::mutex> lk(q->mu);
+  if (!q->outstanding.count(ticket)) return PHMM_E_INVALID_ARG;  // unknown, or waited for before
+  q->done_cv.wait(lk, [&] { return q->done.count(ticket) > 0; });
+  auto it = q->done.find(ticket);
+  const phmm_status st = it->second;
+  q->done.erase(it);
+  q->outstanding.erase(ticket);
+  return st;
+}
+
+phmm_status phmm_compute_batch(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  std::lock_guard<std::mutex> g(c->run_mu);
+  return compute_host(c, b, out_log10, out_status);
+}
+
+phmm_status phmm_compute_batch_dev(phmm_ctx* c, const phmm_batch* b, double* dev_out, uint8_t* dev_status) {
+  if (!c) return PHMM_E_INVALID_ARG;
+  std::lock_guard<std::mutex> g(c->run_mu);
+  ST_TRY(check_batch_args(b));
+  if (b->n_pairs > 0 && !dev_out) return PHMM_E_INVALID_ARG;
+  if (cudaSetDevice(c->device) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  c->launches = 0;
+  DevBatch d{b->read_bases, b->base_quals, b->ins_quals, b->del_quals, b->gcp_quals, b->hap_bases,
+             b->read_offsets, b->hap_offsets, b->pairs, b->n_reads, b->n_haps, b->n_pairs,
+             b->total_read_bases, b->total_hap_bases};
+  // results go to context scratch first and reach the caller's buffers only after the
+  // whole path (FP32 pass and FP64 rescue) succeeded: outputs stay untouched on error
+  double* out = nullptr;
+  uint8_t* status = nullptr;
+  if (b->n_pairs > 0) {
+    ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
+    if (dev_status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
+  }
+  ev_record(c, EV_START);
+  ev_record(c, EV_H2D);
+  phmm_status st = compute_dev(c, d, out, status);
+  if (st != PHMM_OK) {
+    cudaStreamSynchronize(c->stream);
+    cudaGetLastError();
+    return st;
+  }
+  if (b->n_pairs > 0) {
+    CUDA_TRY(cudaMemcpyAsync(dev_out, out, sizeof(double) * (size_t)b->n_pairs, cudaMemcpyDeviceToDevice,
+                             c->stream));
+    if (dev_status)
+      CUDA_TRY(cudaMemcpyAsync(dev_status, status, (size_t)b->n_pairs, cudaMemcpyDeviceToDevice, c->stream));
+  }
+  ev_record(c, EV_END);
+  if (cudaStreamSynchronize(c->stream) != cudaSuccess) {
+    cudaGetLastError();
+    return PHMM_E_CUDA;
+  }
+  finish_stats(c);
+  c->st.ms_h2d = 0.f;
+  c->st.ms_d2h = 0.f;
+  return PHMM_OK;
+}
+
 phmm_status phmm_sw_align_batch_dev(phmm_ctx* c, const phmm_sw_batch* b, const phmm_sw_params* p, int32_t* dev_res,
                                     uint32_t* dev_ops) {
   if (!c) return PHMM_E_INVALID_ARG;
+  std::lock_guard<std::mutex> g_(c->run_mu);
   ST_TRY(sw_check_args(b, p));
   if (b->n_tasks > 0 && (!dev_res || !dev_ops)) return PHMM_E_INVALID_ARG;
   if (cudaSetDevice(c->device) != cudaSuccess) {
@@ -1116,6 +1404,7 @@ phmm_status phmm_sw_align_batch_dev(phmm_ctx* c, const phmm_sw_batch* b, const p
 phmm_status phmm_sw_align_batch(phmm_ctx* c, const phmm_sw_batch* b, const phmm_sw_params* p, int32_t* out_res,
                                 uint32_t* out_ops) {
   if (!c) return PHMM_E_INVALID_ARG;
+  std::lock_guard<std::mutex> g_(c->run_mu);
   ST_TRY(sw_check_args(b, p));
   if (b->n_tasks > 0 && (!out_res || !out_ops)) return PHMM_E_INVALID_ARG;
   if (cudaSetDevice(c->device) != cudaSuccess) {

@@ -172,6 +172,7 @@ static void make_haplotype(rng_t* r, const synth_spec* sp, const uint8_t* ref, i
       const int ln = (int)rng_int(r, 1, 5);
       if (rng_unif(r) < 0.5) {  /* insertion of ln random bases before position i */
         for (int k = 0; k < ln && o < n; ++k) out[o++] = BASES[rng_int(r, 0, 3)];
+        if (o >= n) break;
       } else {                  /* deletion of ln reference bases */
         i += ln;
         continue;

@@ -55,6 +55,9 @@ __device__ int g_trace_steps;
 #ifndef PHMM_F64_MINB
 #define PHMM_F64_MINB 2
 #endif
+#ifndef PHMM_COL_ORDER
+#define PHMM_COL_ORDER 0  // 1: wf_column variant (pre-emission sums of every row first)
+#endif
 #ifndef PHMM_CW_PREFETCH
 #define PHMM_CW_PREFETCH 0  // 1: code words of a lane's next block prefetched one pass ahead
 #endif
@@ -216,6 +219,28 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
                                           const typename WfT<T>::V upI) {
   using V = typename WfT<T>::V;
   constexpr int K = WfT<T>::K;
+#if PHMM_COL_ORDER == 1
+  // variant: all pre-emission sums first (old values only), then M, the I chain and D
+  V xs[K];
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    const V md = (u == 0) ? dgM : L.M[u - 1];
+    const V id = (u == 0) ? dgI : L.I[u - 1];
+    const V dd = (u == 0) ? dgD : L.D[u - 1];
+    xs[u] = fma2(L.ww[u], dd, fma2(L.uu[u], id, md));
+  }
+#pragma unroll
+  for (int u = 0; u < K; ++u) L.D[u] = fma2(L.mu[u], L.D[u], L.M[u]);
+  V m_up = upM, i_up = upI;
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    L.M[u] = pk(prA[u] * lo(xs[u]), prB[u] * hi(xs[u]));
+    const V ni = fma2(L.ep[u], i_up, m_up);
+    m_up = L.M[u];
+    i_up = ni;
+    L.I[u] = ni;
+  }
+#else
   // M and D: rows descending so that row u-1's old values are intact when row u reads them
 #pragma unroll
   for (int u = K - 1; u >= 0; --u) {
@@ -237,6 +262,7 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
     i_up = ni;
     L.I[u] = ni;
   }
+#endif
 }
 
 // ---- shared-memory accessors (inline PTX with "memory" clobbers: the ring and the prior
@@ -745,6 +771,7 @@ template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_sme
   return (b + 15) & ~(size_t)15;
 }
 template <typename T> cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm);
+cudaError_t wf_set_max_smem(int smem_optin);
 template <typename T>
 cudaError_t wf_launch(bool long_rows, unsigned grid, int warps, size_t smem, cudaStream_t stream,
                       const WfArgs2<T>& args);

@@ -11,20 +11,28 @@ static void* wf_kernel(bool long_rows) {
   return long_rows ? reinterpret_cast<void*>(k_wavefront<T, true>) : reinterpret_cast<void*>(k_wavefront<T, false>);
 }
 
+// Allow every wavefront kernel the device's opt-in maximum of dynamic shared memory once
+// (phmm_create), so that launches and occupancy queries need no per-call attribute change.
+cudaError_t wf_set_max_smem(int smem_optin) {
+  const void* fs[4] = {reinterpret_cast<const void*>(k_wavefront<float, false>),
+                       reinterpret_cast<const void*>(k_wavefront<float, true>),
+                       reinterpret_cast<const void*>(k_wavefront<double, false>),
+                       reinterpret_cast<const void*>(k_wavefront<double, true>)};
+  for (const void* f : fs) {
+    cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
 template <typename T>
 cudaError_t wf_occupancy(bool long_rows, int warps, size_t smem, int* blocks_per_sm) {
-  const void* f = wf_kernel<T>(long_rows);
-  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, f, warps * 32, smem);
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, wf_kernel<T>(long_rows), warps * 32, smem);
 }
 
 template <typename T>
 cudaError_t wf_launch(bool long_rows, unsigned grid, int warps, size_t smem, cudaStream_t stream,
                       const WfArgs2<T>& args) {
-  const void* f = wf_kernel<T>(long_rows);
-  cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
   if (long_rows) k_wavefront<T, true><<<grid, warps * 32, smem, stream>>>(args);
   else k_wavefront<T, false><<<grid, warps * 32, smem, stream>>>(args);
   return cudaGetLastError();

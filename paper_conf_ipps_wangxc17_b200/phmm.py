@@ -84,7 +84,7 @@ SW_OPS = "MID"
 
 # every symbol include/phmm.h declares (checked by tests/test_abi.py)
 EXPORTED_SYMBOLS = ("phmm_create", "phmm_compute_batch", "phmm_compute_batch_dev", "phmm_destroy",
-                    "phmm_status_string", "phmm_get_stats", "phmm_abi_version", "phmm_set_stream",
+                    "phmm_status_string", "phmm_get_stats", "phmm_abi_version", "phmm_set_stream", "phmm_submit", "phmm_wait",
                     "phmm_sw_align_batch", "phmm_sw_align_batch_dev")
 
 _lib = None
@@ -115,6 +115,10 @@ def load_library(path: str = LIB_PATH):
     L.phmm_abi_version.restype = ctypes.c_int
     L.phmm_set_stream.argtypes = [ctypes.c_void_p, ctypes.c_void_p]
     L.phmm_set_stream.restype = ctypes.c_int
+    L.phmm_submit.argtypes = [ctypes.c_void_p, ctypes.POINTER(_Batch), _f64p, _u8p, ctypes.POINTER(ctypes.c_uint64)]
+    L.phmm_submit.restype = ctypes.c_int
+    L.phmm_wait.argtypes = [ctypes.c_void_p, ctypes.c_uint64]
+    L.phmm_wait.restype = ctypes.c_int
     for f in (L.phmm_sw_align_batch, L.phmm_sw_align_batch_dev):
         f.argtypes = [ctypes.c_void_p, ctypes.POINTER(_SwBatch), ctypes.POINTER(_SwParams), ctypes.c_void_p,
                       ctypes.c_void_p]
@@ -236,6 +240,19 @@ def _check_out(t, dtype, n: int, dev, name: str) -> None:
                          f"{t.dtype}, {t.numel()} elements on {t.device} (contiguous={t.is_contiguous()})")
 
 
+class Ticket:
+    """A submitted batch (``phmm_submit``); ``wait()`` blocks in ``phmm_wait``."""
+
+    def __init__(self, ctx, ticket: int, out, status):
+        self.ctx, self.ticket, self.out, self.status = ctx, ticket, out, status
+
+    def wait(self):
+        rc = self.ctx._L.phmm_wait(self.ctx._h, self.ticket)
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_wait")
+        return self.out, self.status
+
+
 class PairHMM:
     """One libphmm context (``phmm_create``) bound to one CUDA device."""
 
@@ -283,6 +300,26 @@ class PairHMM:
         """Direct ``phmm_compute_batch`` with prepared pointers (bench e2e leg)."""
         return int(self._L.phmm_compute_batch(self._h, ctypes.byref(s), ctypes.cast(out_ptr, _f64p),
                                               ctypes.cast(status_ptr, _u8p) if status_ptr else None))
+
+    # ------------------------------------------------------------ submission queue
+    def submit(self, batch, out: Optional[np.ndarray] = None, status: Optional[np.ndarray] = None,
+               want_status: bool = True) -> "Ticket":
+        """``phmm_submit``: queue a host batch; returns a Ticket whose ``wait()`` (``phmm_wait``)
+        returns (out, status) once the library has written them. The batch's inputs are
+        copied by the call; ``out`` / ``status`` are kept alive by the ticket."""
+        s, keep = _host_struct(batch)
+        n = int(s.n_pairs)
+        if out is None:
+            out = np.empty(n, dtype=np.float64)
+        if status is None and want_status:
+            status = np.empty(n, dtype=np.uint8)
+        t = ctypes.c_uint64()
+        rc = self._L.phmm_submit(self._h, ctypes.byref(s), out.ctypes.data_as(_f64p),
+                                 status.ctypes.data_as(_u8p) if status is not None else None, ctypes.byref(t))
+        del keep
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_submit")
+        return Ticket(self, int(t.value), out, status)
 
     # ------------------------------------------------------------ device API
     def set_stream(self, stream) -> None:

@@ -115,3 +115,9 @@ def test_device_batch_checks_dtypes_and_sizes_on_cpu_tensors():
         bad.check()
     with pytest.raises(ValueError):
         phmm._check_out(torch.empty(3, dtype=torch.float32), torch.float64, 3, torch.device("cpu"), "out")
+
+
+def test_submit_and_wait_reject_null_without_gpu(lib):
+    t = ctypes.c_uint64()
+    assert lib.phmm_submit(None, None, None, None, ctypes.byref(t)) == -1
+    assert lib.phmm_wait(None, 1) == -1

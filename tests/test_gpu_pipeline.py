@@ -101,3 +101,36 @@ def test_device_call_chunking_is_bitwise(prec):
     finally:
         whole.close()
         chunked.close()
+
+
+def test_submit_queue_coalesces_regions_bitwise():
+    """phmm_submit / phmm_wait: 300 region-sized batches (C3 regions, ~240 pairs each)
+    submitted one by one are coalesced into few runs; every batch's results equal its own
+    synchronous call bit for bit. A batch with an invalid base fails alone (-2, outputs
+    untouched) while the batches coalesced with it succeed."""
+    ctx = phmm.PairHMM(precision="fp32")
+    try:
+        regions = [synth.config_batch("C3", n_regions=1, region_start=r) for r in range(300)]
+        bad_k = 137
+        bad = regions[bad_k].subset(np.arange(regions[bad_k].n_pairs))
+        bad.read_bases = bad.read_bases.copy()
+        bad.read_bases[5] = ord("Z")
+        tickets = []
+        for k, b in enumerate(regions):
+            src = bad if k == bad_k else b
+            out = np.full(src.n_pairs, 7.0)
+            tickets.append(ctx.submit(src, out=out))
+        for k, t in enumerate(tickets):
+            if k == bad_k:
+                with pytest.raises(phmm.PhmmError) as ei:
+                    t.wait()
+                assert ei.value.code == -2 and np.all(t.out == 7.0)
+            else:
+                got, st = t.wait()
+                ref, rst = ctx.compute_batch(regions[k])
+                assert np.array_equal(got, ref) and np.array_equal(st, rst), k
+        # a ticket can be waited for once
+        with pytest.raises(phmm.PhmmError):
+            tickets[0].wait()
+    finally:
+        ctx.close()

@@ -47,3 +47,21 @@ def test_alphabet_and_quality_range():
     assert set(np.unique(b.read_bases)) <= set(b"ACGTN")
     assert set(np.unique(b.hap_bases)) <= set(b"ACGTN")
     assert b.base_quals.max() <= 127
+
+
+def test_generator_heap_is_intact_after_many_regions():
+    """Regression: an insertion that filled a haplotype to its target length was followed by
+    one more write (one byte past the end); glibc caught the corrupted heap only at exit.
+    Generate 2,048 regions of every config in a fresh process and require a clean exit."""
+    import subprocess
+    import sys
+
+    code = ("import sys; sys.path.insert(0, %r)\n"
+            "from paper_conf_ipps_wangxc17_b200 import synth\n"
+            "for c in ('C2', 'C3', 'C4', 'C5'):\n"
+            "    bs = [synth.config_batch(c, n_regions=1, region_start=r) for r in range(512)]\n"
+            "    w = synth.config_batch(c, n_regions=2048)\n"
+            "print('ok')\n") % __import__("os").path.dirname(__import__("os").path.dirname(__file__))
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600,
+                       env=dict(__import__("os").environ, MALLOC_CHECK_="3"))
+    assert r.returncode == 0 and r.stdout.strip() == "ok", r.stderr[-2000:]
