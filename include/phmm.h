@@ -177,7 +177,7 @@ phmm_status phmm_set_stream(phmm_ctx* ctx, void* cuda_stream);
  * Asynchronous submission of host-buffer batches (for region-sized batches: a synchronous
  * call costs ~0.6 ms whatever the batch size, PAPER.md's batches average 189 pairs,
  * L24@575). phmm_submit checks the batch on the host (offsets, pair indices, sizes),
- * copies it into the context's pinned queue and returns at once with a ticket; a worker
+ * copies it into the context's host queue and returns at once with a ticket; a worker
  * thread of the context runs everything queued so far as ONE batch whenever it is idle
  * (so batches submitted while a run is in flight are coalesced into the next run) and
  * writes each batch's results to its own out_log10 / out_status, which must stay valid
@@ -189,7 +189,7 @@ phmm_status phmm_set_stream(phmm_ctx* ctx, void* cuda_stream);
  * waited for once. Other calls on the context wait while a run is in progress (the
  * context serialises its work); phmm_destroy completes every submitted batch first.
  * Returns PHMM_E_INVALID_ARG (NULL arguments, bad sizes or offsets, too many pairs
- * queued), PHMM_E_INDEX, PHMM_E_OOM (pinned queue) from phmm_submit; PHMM_E_INVALID_ARG
+ * queued), PHMM_E_INDEX, PHMM_E_OOM (host queue) from phmm_submit; PHMM_E_INVALID_ARG
  * for an unknown or already-waited ticket from phmm_wait.
  */
 phmm_status phmm_submit(phmm_ctx* ctx, const phmm_batch* b, double* out_log10, uint8_t* out_status,

@@ -22,6 +22,8 @@
 #include <vector>
 #include <new>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/phmm.h"
 #include "phmm_device.cuh"
 #include "host_stage.h"
@@ -54,6 +56,14 @@ struct Buf {
 };
 
 struct AsyncQueue;
+
+// NVTX range around a host phase of the path (a no-op unless a profiler is attached):
+// "phmm:validate", "phmm:fp32_pass", "phmm:rescue", "phmm:fp64_pass", "phmm:chunk",
+// "phmm:h2d", "phmm:d2h", "phmm:submit_run" show up on an Nsight timeline.
+struct Nvtx {
+  explicit Nvtx(const char* name) { nvtxRangePushA(name); }
+  ~Nvtx() { nvtxRangePop(); }
+};
 
 // device scalars written by the prep kernels, read back in one D2H copy
 struct Scalars {
@@ -210,6 +220,7 @@ struct PassInfo {
 
 // Validation of the whole batch. Errors land in scal->err (read back by pass_prepare).
 phmm_status run_validate(phmm_ctx* c, const DevBatch& d) {
+  Nvtx nvtx_("phmm:validate");
   cudaStream_t s = c->stream;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
@@ -516,6 +527,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
 // (as pair index + rbase) and counted in *n_rescue. Returns the haplotype code regions it built.
 phmm_status fp32_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status, int32_t* rlist,
                       int64_t rbase, int64_t* n_rescue, PassInfo* pi, uint8_t** hc, int64_t* total_hc, bool timed) {
+  Nvtx nvtx_("phmm:fp32_pass");
   cudaStream_t s = c->stream;
   int64_t total_tab = 0;
   ST_TRY((pass_prepare<float>(c, d, nullptr, d.n_pairs, pi, &total_tab, total_hc)));
@@ -540,6 +552,7 @@ phmm_status fp32_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* 
 // code regions of d (nullptr: build them here).
 phmm_status rescue_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status, const int32_t* rlist,
                         int64_t nr, const uint8_t* hc, int64_t total_hc, bool timed) {
+  Nvtx nvtx_("phmm:rescue");
   cudaStream_t s = c->stream;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
@@ -592,6 +605,7 @@ void acc_phases(phmm_ctx* c) {
 // underflowing pairs (or the FP64 pass), results into out / status (context scratch).
 // Accumulates the call's statistics; ends synchronised.
 phmm_status compute_one(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* dev_status) {
+  Nvtx nvtx_("phmm:chunk");
   cudaStream_t s = c->stream;
   PassInfo pi;
   int64_t total_tab = 0, total_hc = 0;
@@ -892,15 +906,18 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
   Stager& S = c->stage;
   S.staged_bytes = 0;
   ev_record(c, EV_START);
-  CUDA_TRY(S.h2d(roff, b->read_offsets, sizeof(int64_t) * (b->n_reads + 1), s));
-  CUDA_TRY(S.h2d(hoff, b->hap_offsets, sizeof(int64_t) * (b->n_haps + 1), s));
-  CUDA_TRY(S.h2d(pairs, b->pairs, sizeof(int32_t) * 2 * b->n_pairs, s));
-  CUDA_TRY(S.h2d(hap, b->hap_bases, nh, s));
-  CUDA_TRY(S.h2d(rb, b->read_bases, nr, s));
-  CUDA_TRY(S.h2d(q, b->base_quals, nr, s));
-  CUDA_TRY(S.h2d(qi, b->ins_quals, nr, s));
-  CUDA_TRY(S.h2d(qd, b->del_quals, nr, s));
-  CUDA_TRY(S.h2d(qg, b->gcp_quals, nr, s));
+  {
+    Nvtx nv("phmm:h2d");
+    CUDA_TRY(S.h2d(roff, b->read_offsets, sizeof(int64_t) * (b->n_reads + 1), s));
+    CUDA_TRY(S.h2d(hoff, b->hap_offsets, sizeof(int64_t) * (b->n_haps + 1), s));
+    CUDA_TRY(S.h2d(pairs, b->pairs, sizeof(int32_t) * 2 * b->n_pairs, s));
+    CUDA_TRY(S.h2d(hap, b->hap_bases, nh, s));
+    CUDA_TRY(S.h2d(rb, b->read_bases, nr, s));
+    CUDA_TRY(S.h2d(q, b->base_quals, nr, s));
+    CUDA_TRY(S.h2d(qi, b->ins_quals, nr, s));
+    CUDA_TRY(S.h2d(qd, b->del_quals, nr, s));
+    CUDA_TRY(S.h2d(qg, b->gcp_quals, nr, s));
+  }
   ev_record(c, EV_H2D);
   DevBatch d{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs, (int64_t)nr, (int64_t)nh};
   phmm_status st = compute_dev(c, d, out, status);
@@ -910,8 +927,11 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
     return st;
   }
   ev_record(c, EV_D2H);
-  CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s));
-  if (out_status) CUDA_TRY(S.d2h(out_status, status, b->n_pairs, s));
+  {
+    Nvtx nv("phmm:d2h");
+    CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s));
+    if (out_status) CUDA_TRY(S.d2h(out_status, status, b->n_pairs, s));
+  }
   ev_record(c, EV_END);
   CUDA_TRY(cudaStreamSynchronize(s));
   finish_stats(c);
@@ -925,7 +945,7 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
 // ------------------------------------------------------------ phmm_submit / phmm_wait
 // Region-sized batches (~189 pairs in the paper, L24@575) cost ~0.6 ms per synchronous call
 // however small they are (launches and size read-backs), so the library offers a submission
-// queue: phmm_submit appends a batch to a pinned ARENA (inputs gathered back to back, offsets
+// queue: phmm_submit appends a batch to a host ARENA (inputs gathered back to back, offsets
 // and pair indices rebased) and returns a ticket at once; a worker thread takes the whole
 // arena whenever it is idle and runs it as ONE batch (compute_host), while later submissions
 // fill the other arena; then it copies each batch's results to its caller's buffers. Results
@@ -939,43 +959,41 @@ struct AsyncJob {
   uint8_t* status;
 };
 
-struct PinnedVec {  // growable page-locked byte buffer
+// Growable host byte buffer of an arena. Plain (pageable) memory: growing it costs a
+// realloc, not a page-locking allocation (which takes milliseconds and serialises with the
+// driver); compute_host stages it to the device through the context's pinned ring.
+struct HostVec {
   uint8_t* p = nullptr;
   size_t n = 0, cap = 0;
   bool reserve(size_t want) {
     if (want <= cap) return true;
-    size_t c2 = std::max(want, cap * 2 + ((size_t)1 << 20));
-    uint8_t* q = nullptr;
-    if (cudaHostAlloc(reinterpret_cast<void**>(&q), c2, cudaHostAllocPortable) != cudaSuccess) {
-      cudaGetLastError();
-      return false;
-    }
-    if (n) std::memcpy(q, p, n);
-    if (p) cudaFreeHost(p);
-    p = q;
+    const size_t c2 = std::max(want, cap * 2 + ((size_t)1 << 20));
+    void* q = std::realloc(p, c2);
+    if (!q) return false;
+    p = static_cast<uint8_t*>(q);
     cap = c2;
     return true;
   }
   void release() {
-    if (p) cudaFreeHost(p);
+    std::free(p);
     p = nullptr;
     n = cap = 0;
   }
 };
 
 struct Arena {
-  PinnedVec rb, q, qi, qd, qg, hb, roff, hoff, pairs, out, st;
+  HostVec rb, q, qi, qd, qg, hb, roff, hoff, pairs, out, st;
   std::vector<AsyncJob> jobs;
   int64_t n_reads = 0, n_haps = 0, n_pairs = 0;
   bool any_status = false;
   void clear() {
-    for (PinnedVec* v : {&rb, &q, &qi, &qd, &qg, &hb, &roff, &hoff, &pairs, &out, &st}) v->n = 0;
+    for (HostVec* v : {&rb, &q, &qi, &qd, &qg, &hb, &roff, &hoff, &pairs, &out, &st}) v->n = 0;
     jobs.clear();
     n_reads = n_haps = n_pairs = 0;
     any_status = false;
   }
   void release() {
-    for (PinnedVec* v : {&rb, &q, &qi, &qd, &qg, &hb, &roff, &hoff, &pairs, &out, &st}) v->release();
+    for (HostVec* v : {&rb, &q, &qi, &qd, &qg, &hb, &roff, &hoff, &pairs, &out, &st}) v->release();
   }
 };
 
@@ -992,6 +1010,7 @@ struct AsyncQueue {
 };
 
 void run_arena(phmm_ctx* c, Arena& A) {
+  Nvtx nvtx_("phmm:submit_run");
   std::vector<phmm_status> st(A.jobs.size(), PHMM_OK);
   auto batch_of = [&](int64_t r0, int64_t nr, int64_t h0, int64_t nh, int64_t p0, int64_t np, int64_t rb0,
                       int64_t hb0, std::vector<int64_t>* ro, std::vector<int64_t>* ho, std::vector<int32_t>* pr) {
@@ -1270,7 +1289,7 @@ phmm_status phmm_submit(phmm_ctx* c, const phmm_batch* b, double* out_log10, uin
       !A.pairs.reserve(A.pairs.n + 8 * (size_t)np) || !A.out.reserve(8 * (size_t)(A.n_pairs + np)) ||
       !A.st.reserve((size_t)(A.n_pairs + np)))
     return PHMM_E_OOM;
-  auto app = [](PinnedVec& v, const void* src, size_t n) {
+  auto app = [](HostVec& v, const void* src, size_t n) {
     if (n) std::memcpy(v.p + v.n, src, n);
     v.n += n;
   };

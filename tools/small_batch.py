@@ -46,7 +46,10 @@ def main():
     for b in regions:
         ctx.compute_batch(b)
     t_host = time.perf_counter() - t0
-    # one submission per region (phmm_submit), then wait for all
+    # one submission per region (phmm_submit), then wait for all (after one untimed round
+    # that sizes the queue's host buffers)
+    for t in [ctx.submit(b) for b in regions]:
+        t.wait()
     t0 = time.perf_counter()
     tickets = [ctx.submit(b) for b in regions] if not os.environ.get("NO_SUBMIT") else []
     for t in tickets:
