@@ -414,10 +414,10 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
 
   // launch classes: bins whose ring fits at full occupancy, then (if any) the longer bins
   const int slot = (int)ring_slot_bytes<T>();
-  auto P_of = [](int ncols) { return wf_pass_len(ncols); };
+  auto P_of = [](int ncols) { return wf_pass_len<T>(ncols); };
   const int p_max = P_of(pi.max_ncols);
   int bps_full = 0;
-  CUDA_TRY(occupancy<T>(c, false, WF_WARPS, wf_warp_smem<T>(wf_pass_len(0) + 4) * WF_WARPS, &bps_full));
+  CUDA_TRY(occupancy<T>(c, false, WF_WARPS, wf_warp_smem<T>(wf_pass_len<T>(0) + 4) * WF_WARPS, &bps_full));
   if (bps_full < 1) return PHMM_E_CUDA;
   const int64_t cta_budget = (int64_t)c->smem_per_sm / bps_full - c->smem_reserved;
   const int ring_full = (int)std::min<int64_t>(

@@ -55,6 +55,9 @@ __device__ int g_trace_steps;
 #ifndef PHMM_F64_MINB
 #define PHMM_F64_MINB 2
 #endif
+#ifndef PHMM_STAGED_SWITCH
+#define PHMM_STAGED_SWITCH 1  // 1: staged switch events in the FP32 pass (next block's table by cp.async, coefficients committed 4 steps later)
+#endif
 #ifndef PHMM_COL_ORDER
 #define PHMM_COL_ORDER 0  // 1: wf_column variant (pre-emission sums of every row first)
 #endif
@@ -85,6 +88,15 @@ constexpr int WF_TAIL_SPLIT = PHMM_TAIL_SPLIT;  // short items are 1/WF_TAIL_SPL
 constexpr int WF_LPT = PHMM_LPT;  // 1: longest-row bins first inside a launch
 constexpr int WF_TAIL_DIV = PHMM_TAIL_DIV;  // last 1/WF_TAIL_DIV of a launch's blocks in short work items (0: none)
 constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
+// Staged switch (PHMM_STAGED_SWITCH, FP32 pass): a lane starts its next block wf_sh
+// columns earlier (PAD: the code regions have 16 PAD columns in front), issues the block's
+// table as cp.async copies at its switch event and commits the coefficients 4 steps later,
+// before the first column whose result is used, so no instruction waits on the table loads;
+// a pass is wf_sh steps longer. (The FP64 pass keeps loading at the switch: its 32-byte ring
+// slots leave no shared memory for the staging slots at full occupancy.)
+template <typename T> __host__ __device__ constexpr int wf_sh() {
+  return (PHMM_STAGED_SWITCH && sizeof(T) == 4) ? 4 : 0;
+}
 constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
 constexpr int WF_KC32 = PHMM_F32_K / 4;  // 16-byte chunks per row set of the FP32 pass (K floats)
 constexpr int WF_KC64 = PHMM_F64_K / 2;  // ... of the FP64 pass (K doubles)
@@ -340,14 +352,19 @@ __device__ __forceinline__ void sts16(uint32_t a, const uint4 v) {
 // get 64 more steps, so that virtual lane 63 has finished its whole row when virtual lane
 // 0 of the next pass starts: the ring rescale then sees the full ring row.
 constexpr int WF_RESCALE_COLS = 768;
+template <typename T = float>
 __host__ __device__ inline int wf_pass_len(int ncols) {
-  if (ncols >= WF_RESCALE_COLS) return ncols + WF_G + 64;
-  return (ncols + WF_G > WF_MIN_P) ? ncols + WF_G : WF_MIN_P;
+  constexpr int SH = wf_sh<T>();
+  if (ncols >= WF_RESCALE_COLS) return ncols + WF_G + 64 + SH;
+  return (ncols + WF_G + SH > WF_MIN_P) ? ncols + WF_G + SH : WF_MIN_P;
 }
 // Haplotype code regions: 4 shifted copies per haplotype so that every lane reads its
-// codes as aligned 32-bit words, 4 columns at a time.
+// codes as aligned 32-bit words, 4 columns at a time (sized for the longer of the two
+// passes' P: the FP64 rescue reads the FP32 pass's regions).
 __host__ __device__ inline int wf_hc_copy_len(int ncols) {
-  return ((int)WF_HC_FRONT + wf_pass_len(ncols) + 24 + 3) & ~3;  // + prefetch distance
+  const int P = wf_pass_len<float>(ncols) > wf_pass_len<double>(ncols) ? wf_pass_len<float>(ncols)
+                                                                        : wf_pass_len<double>(ncols);
+  return ((int)WF_HC_FRONT + P + 24 + 3) & ~3;  // + prefetch distance
 }
 
 // Value u of coefficient field f of a TBlock<T> held as 16-byte words w[f * KC + chunk]
@@ -415,6 +432,82 @@ __device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>&
   }
   out_idx = -1;
   return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
+}
+
+// ---- staged switch (PHMM_STAGED_SWITCH): per-warp staging slots, 8 per warp (lane % 8) x 2
+// halves, each [4*KC coefficient words][flags word]
+template <typename T> __host__ __device__ constexpr uint32_t wf_stage_slot() {
+  return 16u * (WF_NCOEF * WfT<T>::KC + 1);
+}
+__device__ __forceinline__ void cp_async16(uint32_t s, const void* g) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" :: "r"(s), "l"(g) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+__device__ __forceinline__ void sts32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" :: "r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint4 lds128(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a)
+               : "memory");
+  return v;
+}
+constexpr uint32_t WF_STG_NONE = 0xffffu;  // staged flags: no block
+// staging bytes of one warp: the 4 lanes of a switch group x 2 halves (a group commits before
+// the next one switches)
+template <typename T> __host__ __device__ constexpr uint32_t wf_stage_bytes() {
+  return wf_sh<T>() > 0 ? 8u * wf_stage_slot<T>() : 0u;
+}
+
+// Switch event of half H (staged): the block's priors go straight into the lane's prior
+// table and its coefficients into the staging slot, both by cp.async (no register waits on
+// them); the R-row position (or "no block") as the slot's flags. The table rows A..N are not
+// read again before column 0, wf_sh + 1 + gi steps later. Returns the code pointer of the
+// lane's first step (column -1 - gi - wf_sh: one word of PAD).
+template <int H, typename T>
+__device__ __forceinline__ const uint32_t* wf_stage(const WfArgs2<T>& A, uint32_t tab_s, uint32_t stg_s, bool have,
+                                                    const BlkDesc& d, int& out_idx, int gi, int copy_len) {
+  constexpr int KC = WfT<T>::KC;
+  if (have) {
+    const uint4* s4 = reinterpret_cast<const uint4*>(A.tab + d.tab_blk);
+#pragma unroll
+    for (int k = 0; k < 5 * KC; ++k) cp_async16(tab_s + 512u * k, s4 + WF_NCOEF * KC + k);
+#pragma unroll
+    for (int k = 0; k < WF_NCOEF * KC; ++k) cp_async16(stg_s + 16u * k, s4 + k);
+    sts32(stg_s + 16u * WF_NCOEF * KC, (uint32_t)((d.flags >> WF_RROW_SHIFT) & 15));
+    out_idx = (d.flags & BLK_LAST) ? d.out_idx : -1;
+    return wf_code_ptr(A, true, d, gi, copy_len) - wf_sh<T>() / 4;
+  }
+  sts32(stg_s + 16u * WF_NCOEF * KC, WF_STG_NONE);
+  out_idx = -1;
+  return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
+}
+
+// Commit of half H, 4 steps after its switch event: the staged coefficients into the lane's
+// registers, M = I = 0 and D = the virtual row 0 on the R row.
+template <int H, typename T>
+__device__ __forceinline__ void wf_commit(Lane<T>& L, uint32_t stg_s, T d0) {
+  constexpr int K = WfT<T>::K;
+  constexpr int KC = WfT<T>::KC;
+  cp_async_wait_all();
+  const uint32_t fl = lds32(stg_s + 16u * WF_NCOEF * KC);
+  const bool have = fl != WF_STG_NONE;
+  uint4 cw[WF_NCOEF * KC];
+#pragma unroll
+  for (int k = 0; k < WF_NCOEF * KC; ++k) cw[k] = have ? lds128(stg_s + 16u * k) : make_uint4(0u, 0u, 0u, 0u);
+  const int rrow = have ? (int)fl : -1;
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    L.uu[u] = set_half<H>(L.uu[u], coef_of<T>(cw, 0, u)); L.ww[u] = set_half<H>(L.ww[u], coef_of<T>(cw, 1, u));
+    L.ep[u] = set_half<H>(L.ep[u], coef_of<T>(cw, 2, u)); L.mu[u] = set_half<H>(L.mu[u], coef_of<T>(cw, 3, u));
+    L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
+    L.D[u] = set_half<H>(L.D[u], rrow == u ? d0 : (T)0);
+  }
 }
 
 #ifndef PHMM_RS_TARGET
@@ -556,9 +649,9 @@ __device__ __forceinline__ unsigned long long wf_claim(const WfArgs2<T>& A, int 
 // registers).
 // kLong: the launch of the long-row bins (the only one with the ring rescale compiled in).
 template <typename T, bool kLong>
-__device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_s, uint32_t xbuf_s,
-                                          uint32_t seg_s, int lane, int64_t s, int nblk, int bin,
-                                          bool trace = false) {
+__device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_base_s,
+                                          uint32_t xbuf_s, uint32_t seg_s, uint32_t stg_s, int lane, int64_t s,
+                                          int nblk, int bin, bool trace = false) {
   const int ncols = bin * A.bucket;
   int64_t* seg = reinterpret_cast<int64_t*>(__cvta_shared_to_generic(seg_s));
   __syncwarp();
@@ -572,10 +665,14 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   constexpr int NGRP = 64 / G;       // switch events per pass
   constexpr int LPG = G / 2;         // physical lanes per group
   constexpr uint32_t RS = ring_slot_bytes<T, kLong>();
+  // ring slot of column c = ring_s + RS * (c + 1); staged switches also read SH slots in
+  // front (never written: zero) for the PAD columns before a block
+  constexpr int SH = wf_sh<T>();
+  const uint32_t ring_s = ring_base_s + RS * (uint32_t)SH;
   const int grp = lane / LPG;
   const int giA = 2 * (lane % LPG), giB = giA + 1;  // position of each half inside its group
   const T d0 = (T)ldexp(1.0, WfT<T>::kScaleExp) / (T)ncols;  // virtual row 0
-  const int P = wf_pass_len(ncols);                           // multiple of 4 (ncols is)
+  const int P = wf_pass_len<T>(ncols);                        // multiple of 4 (ncols is)
   int npass = (nblk + 63) >> 6;
   const int copy_len = wf_hc_copy_len(ncols);
   Lane<T> L;
@@ -595,6 +692,9 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   const uint32_t tabB_s = ptab_s + 16u * (WF_NCODE * WfT<T>::KC * 32 + lane);   // half B
   const int src = (lane + 31) & 31;
   const bool is0 = lane == 0, is31 = lane == 31;
+  const uint32_t stgA_s = stg_s + wf_stage_slot<T>() * (uint32_t)(2 * (lane & 3));  // staged switch only
+  const uint32_t stgB_s = stgA_s + wf_stage_slot<T>();
+  (void)stgA_s; (void)stgB_s;
   int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
   int c31B = -(1 << 20);  // (uniform) column of virtual lane 63 (lane 31, half B)
   T rvM = 0, rvI = 0, rvD = 0;  // lane 31: ring slot for virtual lane 0's next column
@@ -700,6 +800,50 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     step(0); step(1); step(2); step(3);
   };
 
+  if constexpr (SH > 0) {
+  // Staged switch events: group e switches at pass step 8e (its lanes start column
+  // -1 - gi - SH), issuing the next block's table by cp.async, and commits the coefficients
+  // and the initial state at pass step 8e + 4, before any column whose result is used (the
+  // first is column -1 of gi = 0, at that step). Events every 4 steps: 2e switches group e,
+  // 2e + 1 commits it; the last segment runs the rest of the pass.
+  for (int q = 0; q <= npass; ++q) {
+#pragma unroll 1
+    for (int e2 = 0; e2 < 2 * NGRP; ++e2) {
+      const int e = e2 >> 1;
+      if (e2 == 0) {
+        c0 = -1 - SH;  // virtual lane 0 starts its pass
+        if constexpr (rescale) {
+          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && ncols >= WF_RESCALE_COLS;
+          wf_ring_rescale<T, ring_packed<T, kLong>()>((uint64_t)ring_s, ncols, lane, cont,
+                                                      A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
+        }
+      }
+      if (e2 == 2 * NGRP - 2) c31B = -1 - (G - 1) - SH;  // virtual lane 63
+      if (grp == e) {
+        if (!(e2 & 1)) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3
+          const int bA = q * 64 + 2 * lane, bB = bA + 1;
+          const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
+          const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
+          if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S row: the last-row M+I sum (L20@2262)
+          if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
+          pA = wf_stage<0, T>(A, tabA_s, stgA_s, hA, dA, outA, giA, copy_len);
+          pB = wf_stage<1, T>(A, tabB_s, stgB_s, hB, dB, outB, giB, copy_len);
+          // the first code word of a block (columns -1-gi-4 .. -2-gi) is PAD
+          wA_nx = kPadW; wA_nx2 = __ldg(pA + 1); pA += 2;
+          wB_nx = kPadW; wB_nx2 = __ldg(pB + 1); pB += 2;
+          if (bA + 64 < nblk) dnA = A.blk[phys(bA + 64)];
+          if (bB + 64 < nblk) dnB = A.blk[phys(bB + 64)];
+        } else {  // commit of the group that switched 4 steps ago
+          wf_commit<0, T>(L, stgA_s, d0);
+          wf_commit<1, T>(L, stgB_s, d0);
+        }
+      }
+      const int ngroups = (e2 < 2 * NGRP - 1) ? 1 : (q < npass ? (P - (2 * NGRP - 1) * 4) / 4 : 0);
+#pragma unroll 1
+      for (int k = 0; k < ngroups; ++k) group4();
+    }
+  }
+  } else {
   for (int q = 0; q <= npass; ++q) {
 #pragma unroll 1
     for (int e = 0; e < NGRP; ++e) {
@@ -754,6 +898,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
       for (int k = 0; k < ngroups; ++k) group4();
     }
   }
+  }
 }
 
 // The kernels are defined in wf.cu (their own translation unit, compiled with
@@ -762,11 +907,11 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 // phmm_lib.cu reaches them through these host functions.
 // shared memory of one warp: its prior tables and its ring
 template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_smem(int ring_len) {
-  // prior tables, ring, and (design-A ablation only) the exchange line buffer; a multiple of
-  // 16 bytes so that every warp's tables stay 16-byte aligned
-  const size_t b = (size_t)2 * WF_NCODE * WfT<T>::KC * 32 * 16 +
-                   (size_t)(ring_len + (PHMM_XCHG_SMEM ? 32 : 0)) *
-                       ring_slot_bytes<T, kLong>() +
+  // prior tables, (staged switch only) the staging slots, the ring (+ wf_sh front slots),
+  // (design-A ablation only) the exchange line buffer; a multiple of 16 bytes so that every
+  // warp's tables stay 16-byte aligned
+  const size_t b = (size_t)2 * WF_NCODE * WfT<T>::KC * 32 * 16 + (size_t)wf_stage_bytes<T>() +
+                   (size_t)(ring_len + wf_sh<T>() + (PHMM_XCHG_SMEM ? 32 : 0)) * ring_slot_bytes<T, kLong>() +
                    32;  // the stream's first block (wf_stream)
   return (b + 15) & ~(size_t)15;
 }
@@ -788,8 +933,8 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
   unsigned char* base = smem_raw + (size_t)wib * per_warp;
   for (uint32_t i = 4 * lane; i < per_warp; i += 128) *reinterpret_cast<uint32_t*>(base + i) = 0u;
   __syncwarp();
-  const uint32_t ptab_s = smem_addr(base), ring_s = ptab_s + kTabBytes;
-  const uint32_t xbuf_s = ring_s + (uint32_t)A.ring_len * ring_slot_bytes<T, kLong>();  // design A only
+  const uint32_t ptab_s = smem_addr(base), stg_s = ptab_s + kTabBytes, ring_s = stg_s + wf_stage_bytes<T>();
+  const uint32_t xbuf_s = ring_s + (uint32_t)(A.ring_len + wf_sh<T>()) * ring_slot_bytes<T, kLong>();  // design A only
   const uint32_t seg_s = (ptab_s + per_warp - 32u) & ~7u;   // the stream's first block (last 32 B)
   // work items of the launch, claimed from an atomic counter
   const unsigned long long it1 = A.launch_items[1];
@@ -800,7 +945,8 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
     int64_t s, e;
     wf_item(A, it, lane, bin, s, e);
     if (e <= s) continue;
-    wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, seg_s, lane, s, (int)(e - s), bin, it == A.launch_items[0]);
+    wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, seg_s, stg_s, lane, s, (int)(e - s), bin,
+                        it == A.launch_items[0]);
     __syncwarp();
   }
 }
