@@ -94,8 +94,11 @@ constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >=
 // before the first column whose result is used, so no instruction waits on the table loads;
 // a pass is wf_sh steps longer. (The FP64 pass keeps loading at the switch: its 32-byte ring
 // slots leave no shared memory for the staging slots at full occupancy.)
+#ifndef PHMM_STAGED_SWITCH64
+#define PHMM_STAGED_SWITCH64 1  // 1: staged switch events in the FP64 pass too (with packed 24-byte ring slots)
+#endif
 template <typename T> __host__ __device__ constexpr int wf_sh() {
-  return (PHMM_STAGED_SWITCH && sizeof(T) == 4) ? 4 : 0;
+  return (sizeof(T) == 4 ? PHMM_STAGED_SWITCH : PHMM_STAGED_SWITCH64) ? 4 : 0;
 }
 constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
 constexpr int WF_KC32 = PHMM_F32_K / 4;  // 16-byte chunks per row set of the FP32 pass (K floats)
@@ -301,7 +304,7 @@ __device__ __forceinline__ void ring_get3(uint32_t a, double& x, double& y, doub
 // FP64 long-row kernel, where the ring limits occupancy (C4 rescue: 3 -> 4 warps per SM;
 // packing the FP32 long-row ring measured slower)
 template <typename T, bool kLong = false> __host__ __device__ constexpr bool ring_packed() {
-  return kLong && sizeof(T) == 8;
+  return (kLong || PHMM_STAGED_SWITCH64) && sizeof(T) == 8;
 }
 template <typename T, bool kLong = false> __host__ __device__ constexpr uint32_t ring_slot_bytes() {
   return ring_packed<T, kLong>() ? 3u * (uint32_t)sizeof(T) : (sizeof(T) == 4 ? 16u : 32u);
