@@ -58,12 +58,6 @@ __device__ int g_trace_steps;
 #ifndef PHMM_STAGED_SWITCH
 #define PHMM_STAGED_SWITCH 1  // 1: staged switch events in the FP32 pass (next block's table by cp.async, coefficients committed 4 steps later)
 #endif
-#ifndef PHMM_COL_ORDER
-#define PHMM_COL_ORDER 0  // 1: wf_column variant (pre-emission sums of every row first)
-#endif
-#ifndef PHMM_CW_PREFETCH
-#define PHMM_CW_PREFETCH 0  // 1: code words of a lane's next block prefetched one pass ahead
-#endif
 #ifndef PHMM_XCHG_SMEM
 #define PHMM_XCHG_SMEM 0  // 1: design-A ablation build (row exchange through shared memory)
 #endif
@@ -88,12 +82,13 @@ constexpr int WF_TAIL_SPLIT = PHMM_TAIL_SPLIT;  // short items are 1/WF_TAIL_SPL
 constexpr int WF_LPT = PHMM_LPT;  // 1: longest-row bins first inside a launch
 constexpr int WF_TAIL_DIV = PHMM_TAIL_DIV;  // last 1/WF_TAIL_DIV of a launch's blocks in short work items (0: none)
 constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
-// Staged switch (PHMM_STAGED_SWITCH, FP32 pass): a lane starts its next block wf_sh
-// columns earlier (PAD: the code regions have 16 PAD columns in front), issues the block's
-// table as cp.async copies at its switch event and commits the coefficients 4 steps later,
-// before the first column whose result is used, so no instruction waits on the table loads;
-// a pass is wf_sh steps longer. (The FP64 pass keeps loading at the switch: its 32-byte ring
-// slots leave no shared memory for the staging slots at full occupancy.)
+// Staged switch (PHMM_STAGED_SWITCH: FP32 pass, PHMM_STAGED_SWITCH64: FP64 pass): a lane
+// starts its next block wf_sh = 4 columns earlier (PAD: the code regions have 16 PAD columns
+// in front), issues the block's table as cp.async copies at its switch event and commits the
+// coefficients 4 steps later, before the first column whose result is used, so no
+// instruction waits on the table loads; a pass is 4 steps longer. The FP64
+// pass packs its ring slots into 24 bytes to pay for the staging slots and stay at 8 warps
+// per SM.
 #ifndef PHMM_STAGED_SWITCH64
 #define PHMM_STAGED_SWITCH64 1  // 1: staged switch events in the FP64 pass too (with packed 24-byte ring slots)
 #endif
@@ -234,28 +229,6 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
                                           const typename WfT<T>::V upI) {
   using V = typename WfT<T>::V;
   constexpr int K = WfT<T>::K;
-#if PHMM_COL_ORDER == 1
-  // variant: all pre-emission sums first (old values only), then M, the I chain and D
-  V xs[K];
-#pragma unroll
-  for (int u = 0; u < K; ++u) {
-    const V md = (u == 0) ? dgM : L.M[u - 1];
-    const V id = (u == 0) ? dgI : L.I[u - 1];
-    const V dd = (u == 0) ? dgD : L.D[u - 1];
-    xs[u] = fma2(L.ww[u], dd, fma2(L.uu[u], id, md));
-  }
-#pragma unroll
-  for (int u = 0; u < K; ++u) L.D[u] = fma2(L.mu[u], L.D[u], L.M[u]);
-  V m_up = upM, i_up = upI;
-#pragma unroll
-  for (int u = 0; u < K; ++u) {
-    L.M[u] = pk(prA[u] * lo(xs[u]), prB[u] * hi(xs[u]));
-    const V ni = fma2(L.ep[u], i_up, m_up);
-    m_up = L.M[u];
-    i_up = ni;
-    L.I[u] = ni;
-  }
-#else
   // M and D: rows descending so that row u-1's old values are intact when row u reads them
 #pragma unroll
   for (int u = K - 1; u >= 0; --u) {
@@ -277,7 +250,6 @@ __device__ __forceinline__ void wf_column(Lane<T>& L, const T (&prA)[WfT<T>::K],
     i_up = ni;
     L.I[u] = ni;
   }
-#endif
 }
 
 // ---- shared-memory accessors (inline PTX with "memory" clobbers: the ring and the prior
@@ -706,21 +678,6 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   dnB = dnA;
   if (2 * lane < nblk) dnA = A.blk[phys(2 * lane)];
   if (2 * lane + 1 < nblk) dnB = A.blk[phys(2 * lane + 1)];
-#if PHMM_CW_PREFETCH
-  // descriptors two passes ahead and the first two code words of the next block, so that a
-  // switch event finds its block's code words already in registers (no long-scoreboard stall
-  // on the first PRMT after a switch)
-  BlkDesc dnnA = dnA, dnnB = dnB;
-  if (2 * lane + 64 < nblk) dnnA = A.blk[phys(2 * lane + 64)];
-  if (2 * lane + 65 < nblk) dnnB = A.blk[phys(2 * lane + 65)];
-  uint32_t cwA0, cwA1, cwB0, cwB1;
-  {
-    const uint32_t* p0 = wf_code_ptr(A, 2 * lane < nblk, dnA, giA, copy_len);
-    const uint32_t* p1 = wf_code_ptr(A, 2 * lane + 1 < nblk, dnB, giB, copy_len);
-    cwA0 = __ldg(p0); cwA1 = __ldg(p0 + 1);
-    cwB0 = __ldg(p1); cwB1 = __ldg(p1 + 1);
-  }
-#endif
 #ifdef PHMM_DBG_TRACE
   int tstep = 0;
 #endif
@@ -869,27 +826,12 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
         if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
         pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
         pB = wf_load<1, T>(A, L, tabB_s, hB, dB, d0, outB, giB, copy_len);
-#if PHMM_CW_PREFETCH
-        wA_nx = cwA0; wA_nx2 = cwA1; pA += 2;
-        wB_nx = cwB0; wB_nx2 = cwB1; pB += 2;
-        dnA = dnnA;
-        dnB = dnnB;
-        {
-          const uint32_t* p0 = wf_code_ptr(A, bA + 64 < nblk, dnA, giA, copy_len);
-          const uint32_t* p1 = wf_code_ptr(A, bB + 64 < nblk, dnB, giB, copy_len);
-          cwA0 = __ldg(p0); cwA1 = __ldg(p0 + 1);
-          cwB0 = __ldg(p1); cwB1 = __ldg(p1 + 1);
-        }
-        if (bA + 128 < nblk) dnnA = A.blk[phys(bA + 128)];
-        if (bB + 128 < nblk) dnnB = A.blk[phys(bB + 128)];
-#else
         wA_nx = __ldg(pA); wA_nx2 = __ldg(pA + 1); pA += 2;
         wB_nx = __ldg(pB); wB_nx2 = __ldg(pB + 1); pB += 2;
         // prefetch the next pass's descriptors after this pass's loads are issued (a load
         // issued before the consumers of the previous prefetch would share its scoreboard)
         if (bA + 64 < nblk) dnA = A.blk[phys(bA + 64)];
         if (bB + 64 < nblk) dnB = A.blk[phys(bB + 64)];
-#endif
         if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
           T a, bb, c;
           rget<ring_packed<T, kLong>()>(ring_s, a, bb, c);
