@@ -55,9 +55,6 @@ __device__ int g_trace_steps;
 #ifndef PHMM_F64_MINB
 #define PHMM_F64_MINB 2
 #endif
-#ifndef PHMM_STAGED_SWITCH
-#define PHMM_STAGED_SWITCH 1  // 1: staged switch events in the FP32 pass (next block's table by cp.async, coefficients committed 4 steps later)
-#endif
 #ifndef PHMM_XCHG_SMEM
 #define PHMM_XCHG_SMEM 0  // 1: design-A ablation build (row exchange through shared memory)
 #endif
@@ -82,19 +79,13 @@ constexpr int WF_TAIL_SPLIT = PHMM_TAIL_SPLIT;  // short items are 1/WF_TAIL_SPL
 constexpr int WF_LPT = PHMM_LPT;  // 1: longest-row bins first inside a launch
 constexpr int WF_TAIL_DIV = PHMM_TAIL_DIV;  // last 1/WF_TAIL_DIV of a launch's blocks in short work items (0: none)
 constexpr int WF_MIN_P = 72;      // ring delay: virtual lane 63 -> 0 needs P >= 72
-// Staged switch (PHMM_STAGED_SWITCH: FP32 pass, PHMM_STAGED_SWITCH64: FP64 pass): a lane
-// starts its next block wf_sh = 4 columns earlier (PAD: the code regions have 16 PAD columns
-// in front), issues the block's table as cp.async copies at its switch event and commits the
-// coefficients 4 steps later, before the first column whose result is used, so no
-// instruction waits on the table loads; a pass is 4 steps longer. The FP64
-// pass packs its ring slots into 24 bytes to pay for the staging slots and stay at 8 warps
-// per SM.
-#ifndef PHMM_STAGED_SWITCH64
-#define PHMM_STAGED_SWITCH64 1  // 1: staged switch events in the FP64 pass too (with packed 24-byte ring slots)
-#endif
-template <typename T> __host__ __device__ constexpr int wf_sh() {
-  return (sizeof(T) == 4 ? PHMM_STAGED_SWITCH : PHMM_STAGED_SWITCH64) ? 4 : 0;
-}
+// Staged switch events (both passes): a lane starts its next block wf_sh = 4 columns
+// earlier (PAD: the code regions have 16 PAD columns in front), issues the block's table as
+// cp.async copies at its switch event and commits the coefficients 4 steps later, before the
+// first column whose result is used, so no instruction waits on the table loads; a pass is
+// 4 steps longer. The FP64 pass packs its ring slots into 24 bytes to pay
+// for the staging slots and stay at 8 warps per SM.
+template <typename T> __host__ __device__ constexpr int wf_sh() { return 4; }
 constexpr int64_t WF_HC_FRONT = 16;  // PAD codes before every haplotype's code array
 constexpr int WF_KC32 = PHMM_F32_K / 4;  // 16-byte chunks per row set of the FP32 pass (K floats)
 constexpr int WF_KC64 = PHMM_F64_K / 2;  // ... of the FP64 pass (K doubles)
@@ -276,7 +267,7 @@ __device__ __forceinline__ void ring_get3(uint32_t a, double& x, double& y, doub
 // FP64 long-row kernel, where the ring limits occupancy (C4 rescue: 3 -> 4 warps per SM;
 // packing the FP32 long-row ring measured slower)
 template <typename T, bool kLong = false> __host__ __device__ constexpr bool ring_packed() {
-  return (kLong || PHMM_STAGED_SWITCH64) && sizeof(T) == 8;
+  return sizeof(T) == 8;  // FP64: 24-byte slots pay for the staging slots (8 warps per SM)
 }
 template <typename T, bool kLong = false> __host__ __device__ constexpr uint32_t ring_slot_bytes() {
   return ring_packed<T, kLong>() ? 3u * (uint32_t)sizeof(T) : (sizeof(T) == 4 ? 16u : 32u);
@@ -371,46 +362,8 @@ __device__ __forceinline__ const uint32_t* wf_code_ptr(const WfArgs2<T>& A, bool
   return reinterpret_cast<const uint32_t*>(A.hcodes + (col0 - 1u - (uint32_t)gi));
 }
 
-// Load a block (or nothing) into half H of a lane. Returns the 32-bit-aligned code
-// pointer for the lane's first step (column -1 - gi).
-template <int H, typename T>
-__device__ __forceinline__ const uint32_t* wf_load(const WfArgs2<T>& A, Lane<T>& L, uint32_t tab_s, bool have,
-                                                   const BlkDesc& d, T d0, int& out_idx, int gi, int copy_len) {
-  constexpr int K = WfT<T>::K;
-  if (have) {
-    const uint4* __restrict__ s4 = reinterpret_cast<const uint4*>(A.tab + d.tab_blk);
-    constexpr int KC = WfT<T>::KC;
-    // the 4 coefficient fields as 16-byte words, unpacked value by value (no type punning)
-    uint4 cw[WF_NCOEF * KC];
-#pragma unroll
-    for (int k = 0; k < WF_NCOEF * KC; ++k) cw[k] = __ldg(s4 + k);
-#pragma unroll
-    for (int k = 0; k < 5 * KC; ++k)  // prior[code][chunk]
-      sts16(tab_s + 512u * k, __ldg(s4 + WF_NCOEF * KC + k));
-    const int rrow = (d.flags >> WF_RROW_SHIFT) & 15;
-#pragma unroll
-    for (int u = 0; u < K; ++u) {
-      L.uu[u] = set_half<H>(L.uu[u], coef_of<T>(cw, 0, u)); L.ww[u] = set_half<H>(L.ww[u], coef_of<T>(cw, 1, u));
-      L.ep[u] = set_half<H>(L.ep[u], coef_of<T>(cw, 2, u)); L.mu[u] = set_half<H>(L.mu[u], coef_of<T>(cw, 3, u));
-      L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
-      L.D[u] = set_half<H>(L.D[u], rrow == u ? d0 : (T)0);
-    }
-    out_idx = (d.flags & BLK_LAST) ? d.out_idx : -1;
-    return wf_code_ptr(A, true, d, gi, copy_len);
-  }
-#pragma unroll
-  for (int u = 0; u < K; ++u) {
-    L.uu[u] = set_half<H>(L.uu[u], (T)0); L.ww[u] = set_half<H>(L.ww[u], (T)0);
-    L.ep[u] = set_half<H>(L.ep[u], (T)0); L.mu[u] = set_half<H>(L.mu[u], (T)0);
-    L.M[u] = set_half<H>(L.M[u], (T)0); L.I[u] = set_half<H>(L.I[u], (T)0);
-    L.D[u] = set_half<H>(L.D[u], (T)0);
-  }
-  out_idx = -1;
-  return reinterpret_cast<const uint32_t*>(A.hcodes + A.pad_idx);
-}
-
-// ---- staged switch (PHMM_STAGED_SWITCH): per-warp staging slots, 8 per warp (lane % 8) x 2
-// halves, each [4*KC coefficient words][flags word]
+// ---- staged switch: per-warp staging slots, the 4 lanes of a switch group x 2 halves,
+// each [4*KC coefficient words][flags word]
 template <typename T> __host__ __device__ constexpr uint32_t wf_stage_slot() {
   return 16u * (WF_NCOEF * WfT<T>::KC + 1);
 }
@@ -436,7 +389,7 @@ constexpr uint32_t WF_STG_NONE = 0xffffu;  // staged flags: no block
 // staging bytes of one warp: the 4 lanes of a switch group x 2 halves (a group commits before
 // the next one switches)
 template <typename T> __host__ __device__ constexpr uint32_t wf_stage_bytes() {
-  return wf_sh<T>() > 0 ? 8u * wf_stage_slot<T>() : 0u;
+  return 8u * wf_stage_slot<T>();
 }
 
 // Switch event of half H (staged): the block's priors go straight into the lane's prior
@@ -666,8 +619,8 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   const uint32_t tabA_s = ptab_s + 16u * lane;                              // [code][chunk][lane] 16 B
   const uint32_t tabB_s = ptab_s + 16u * (WF_NCODE * WfT<T>::KC * 32 + lane);   // half B
   const int src = (lane + 31) & 31;
-  const bool is0 = lane == 0, is31 = lane == 31;
-  const uint32_t stgA_s = stg_s + wf_stage_slot<T>() * (uint32_t)(2 * (lane & 3));  // staged switch only
+  const bool is31 = lane == 31;
+  const uint32_t stgA_s = stg_s + wf_stage_slot<T>() * (uint32_t)(2 * (lane & 3));
   const uint32_t stgB_s = stgA_s + wf_stage_slot<T>();
   (void)stgA_s; (void)stgB_s;
   int c0 = -(1 << 20);    // (uniform) column of virtual lane 0 (lane 0, half A)
@@ -760,7 +713,6 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     step(0); step(1); step(2); step(3);
   };
 
-  if constexpr (SH > 0) {
   // Staged switch events: group e switches at pass step 8e (its lanes start column
   // -1 - gi - SH), issuing the next block's table by cp.async, and commits the coefficients
   // and the initial state at pass step 8e + 4, before any column whose result is used (the
@@ -803,47 +755,6 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
       for (int k = 0; k < ngroups; ++k) group4();
     }
   }
-  } else {
-  for (int q = 0; q <= npass; ++q) {
-#pragma unroll 1
-    for (int e = 0; e < NGRP; ++e) {
-      if (e == 0) {
-        c0 = -1;  // virtual lane 0 starts its pass: column -1 next
-        if constexpr (rescale) {
-          // lane 0's block of this pass continues the pair of virtual lane 63's last block?
-          // (rows shorter than WF_RESCALE_COLS have no complete ring row at the pass start)
-          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && ncols >= WF_RESCALE_COLS;
-          wf_ring_rescale<T, ring_packed<T, kLong>()>((uint64_t)ring_s, ncols, lane, cont,
-                                                      A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
-        }
-      }
-      if (e == NGRP - 1) c31B = -1 - (G - 1);  // virtual lane 63
-      if (grp == e) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3, both halves
-        const int bA = q * 64 + 2 * lane, bB = bA + 1;
-        const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
-        const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
-        if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S row: the last-row M+I sum (L20@2262)
-        if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
-        pA = wf_load<0, T>(A, L, tabA_s, hA, dA, d0, outA, giA, copy_len);
-        pB = wf_load<1, T>(A, L, tabB_s, hB, dB, d0, outB, giB, copy_len);
-        wA_nx = __ldg(pA); wA_nx2 = __ldg(pA + 1); pA += 2;
-        wB_nx = __ldg(pB); wB_nx2 = __ldg(pB + 1); pB += 2;
-        // prefetch the next pass's descriptors after this pass's loads are issued (a load
-        // issued before the consumers of the previous prefetch would share its scoreboard)
-        if (bA + 64 < nblk) dnA = A.blk[phys(bA + 64)];
-        if (bB + 64 < nblk) dnB = A.blk[phys(bB + 64)];
-        if (is0) {  // virtual lane 0: its column -1 needs the boundary slot of the ring
-          T a, bb, c;
-          rget<ring_packed<T, kLong>()>(ring_s, a, bb, c);
-          upM = set_half<0>(upM, a); upI = set_half<0>(upI, bb); upD = set_half<0>(upD, c);
-        }
-      }
-      const int ngroups = (e < NGRP - 1) ? G / 4 : (q < npass ? (P - (NGRP - 1) * G) / 4 : 0);
-#pragma unroll 1
-      for (int k = 0; k < ngroups; ++k) group4();
-    }
-  }
-  }
 }
 
 // The kernels are defined in wf.cu (their own translation unit, compiled with
@@ -852,7 +763,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 // phmm_lib.cu reaches them through these host functions.
 // shared memory of one warp: its prior tables and its ring
 template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_smem(int ring_len) {
-  // prior tables, (staged switch only) the staging slots, the ring (+ wf_sh front slots),
+  // prior tables, the staging slots, the ring (+ wf_sh front slots),
   // (design-A ablation only) the exchange line buffer; a multiple of 16 bytes so that every
   // warp's tables stay 16-byte aligned
   const size_t b = (size_t)2 * WF_NCODE * WfT<T>::KC * 32 * 16 + (size_t)wf_stage_bytes<T>() +

@@ -4,9 +4,13 @@ virtual lanes are packed into physical lanes / register halves:
 
 * a warp streams through the blocks of one length bin; pass q gives block 64q+v to
   virtual lane v (K rows each, the Z/R/read/S pad-row layout of DESIGN.md §4.2);
-* virtual lane v computes column x of its block at step T_q + 1 + v + x; a pass is
-  P = max(ncols + G, 72) steps; virtual lanes switch blocks in groups of G = 8 at the
-  events T_q + 8e (e = 0..7), taking column -1 - (v mod 8) next;
+* virtual lane v computes column x of its block at step T_q + 1 + SH + v + x; a pass is
+  P = max(ncols + G + SH, 72) steps; virtual lanes switch blocks in groups of G = 8 at the
+  events T_q + 8e (e = 0..7), taking column -1 - (v mod 8) - SH next (SH = 4 PAD columns,
+  the staged switch of DESIGN.md §4.4): the switch writes the finished pair's result and
+  points the lane at its new block's codes and priors, and 4 steps later the group COMMITS
+  the new block's coefficients and initial state (M = I = 0, D = the virtual row 0 on the
+  R row) -- until then the lane computes PAD columns with its old coefficients and state;
 * columns outside a block read the PAD code (prior 0) -- no per-lane branch;
 * virtual lane v takes the row above from v-1's last row one step later; v = 0 from
   a ring indexed by column + 1 (slot 0 = boundary column) written by v = 63 of the
@@ -23,10 +27,13 @@ RESCALE_COLS = 768  # long rows: passes 64 steps longer, ring rescale on (DESIGN
 RS_TARGET, RS_TRIG, RS_CAP = 112, 104, 126  # ring rescale: below 2^RS_TRIG -> ~2^RS_TARGET, saturating at 2^RS_CAP
 
 
+SH = 4  # PAD columns a lane runs before its block (staged switch)
+
+
 def pass_len(ncols):
     if ncols >= RESCALE_COLS:
-        return ncols + G + 64
-    return max(ncols + G, MINP)
+        return ncols + G + 64 + SH
+    return max(ncols + G + SH, MINP)
 E = np.float32
 
 
@@ -187,7 +194,8 @@ def run_stream(blocks, ncols, K, rescale=True):
                     pr_ = blocks[b]["pair"]
                     sat = ring_scale(sh)
                     exps[pr_] = exps.get(pr_, 0) + (-(1 << 24) if sat else sh)
-            for v in range(8 * e, 8 * e + 8):
+            staged = {}
+            for v in range(8 * e, 8 * e + 8):  # switch
                 gi = v % G
                 b = q * 64 + v
                 if out[v] >= 0:
@@ -196,23 +204,28 @@ def run_stream(blocks, ncols, K, rescale=True):
                 if q < npass and b < nblk:
                     blk = blocks[b]
                     for u in range(K):
-                        r = blk["rows"][u]
-                        for fi in range(4):
-                            co[fi, v, u] = r[fi]
                         for cc in range(5):
-                            pri[v, cc, u] = r[4][cc]
-                        M[v, u] = 0; I[v, u] = 0
-                        D[v, u] = d0 if blk["rrow"] == u else E(0)
+                            pri[v, cc, u] = blk["rows"][u][4][cc]
                     codes[v], offs[v] = blk["codes"]
                     if blk["last"]:
                         out[v] = blk["pair"]
+                    staged[v] = blk
                 else:
-                    co[:, v, :] = 0; pri[v] = 0; M[v] = 0; I[v] = 0; D[v] = 0
                     codes[v] = pad; offs[v] = 0
-                col[v] = -1 - gi
-                if v == 0:
-                    up[0] = ring[0]
-            nsteps = G if e < 7 else (P - 7 * G if q < npass else 0)
+                    staged[v] = None
+                col[v] = -1 - gi - SH
+            for k in range(4):
+                step()
+            for v, blk in staged.items():  # commit, 4 steps after the switch
+                if blk is None:
+                    co[:, v, :] = 0; M[v] = 0; I[v] = 0; D[v] = 0
+                    continue
+                for u in range(K):
+                    for fi in range(4):
+                        co[fi, v, u] = blk["rows"][u][fi]
+                    M[v, u] = 0; I[v, u] = 0
+                    D[v, u] = d0 if blk["rrow"] == u else E(0)
+            nsteps = 4 if e < 7 else (P - 7 * G - 4 if q < npass else 0)
             for k in range(nsteps):
                 step()
     return res, exps
