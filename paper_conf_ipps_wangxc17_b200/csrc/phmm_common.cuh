@@ -43,6 +43,7 @@ constexpr int kMinCols = 40;        // ring delay needs ncols > 32
 constexpr int kMaxHapLen = 4094;    // FP32/FP64 ring in shared memory
 constexpr int kMaxReadLen = 1 << 20;  // longest read a pair may use (include/phmm.h)
 constexpr int kMaxBins = 4200;      // ncols / bucket <= kMaxBins
+constexpr int kNcolsComplement = 1 << 20;  // > any column count: min(ncols) travels as max(this - ncols)
 
 // error flag bits (device) -> phmm_status
 enum : uint32_t {

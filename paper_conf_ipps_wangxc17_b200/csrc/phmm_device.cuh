@@ -95,7 +95,8 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
                             const int64_t* __restrict__ hoff, int64_t n_haps, int bucket,
                             int32_t* __restrict__ pair_bin, int32_t* __restrict__ pair_nb,
                             unsigned long long* __restrict__ bin_blocks, unsigned long long* __restrict__ bin_pairs,
-                            int* __restrict__ max_ncols, unsigned long long* __restrict__ cells,
+                            int* __restrict__ max_ncols, int* __restrict__ min_ncols_c,
+                            unsigned long long* __restrict__ cells,
                             unsigned long long* __restrict__ padded_cells, unsigned long long* __restrict__ total_blocks,
                             uint32_t* err) {
   const int64_t n = n_list_dev ? *n_list_dev : n_pairs;
@@ -103,7 +104,7 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   uint32_t e = 0;
   unsigned long long my_cells = 0, my_padded = 0, my_blocks = 0;
-  int my_max = 0;
+  int my_max = 0, my_minc = 0;  // my_minc = kNcolsComplement - smallest column count
   for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < n; base += stride) {
     const int64_t k = base + lane;
     int bin = -1, nb = 0;
@@ -123,6 +124,7 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
           bin = bin_of_ncols(nc, bucket);
           nb = nblocks_of<K>((int)m);
           my_max = max(my_max, nc);
+          my_minc = max(my_minc, kNcolsComplement - nc);
           my_cells += (unsigned long long)(m * nh);
           my_padded += (unsigned long long)nb * K * nc;
           my_blocks += (unsigned long long)nb;
@@ -147,6 +149,7 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
     my_padded += __shfl_xor_sync(0xffffffffu, my_padded, o);
     my_blocks += __shfl_xor_sync(0xffffffffu, my_blocks, o);
     my_max = max(my_max, __shfl_xor_sync(0xffffffffu, my_max, o));
+    my_minc = max(my_minc, __shfl_xor_sync(0xffffffffu, my_minc, o));
     e |= __shfl_xor_sync(0xffffffffu, e, o);
   }
   if (lane == 0) {
@@ -154,6 +157,7 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
     if (my_padded) atomicAdd(padded_cells, my_padded);
     if (my_blocks) atomicAdd(total_blocks, my_blocks);
     if (my_max) atomicMax(max_ncols, my_max);
+    if (my_minc) atomicMax(min_ncols_c, my_minc);
     if (e) atomicOr(err, e);
   }
 }

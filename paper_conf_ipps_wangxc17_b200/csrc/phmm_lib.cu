@@ -69,6 +69,7 @@ struct Nvtx {
 struct Scalars {
   uint32_t err;
   int32_t max_ncols;
+  int32_t min_ncols_c;  // kMinColsComplement - smallest column count (0-initialised max)
   unsigned long long cells;
   unsigned long long padded_cells;
   unsigned long long total_blocks;
@@ -215,7 +216,7 @@ struct DevBatch {
 
 struct PassInfo {
   unsigned long long cells = 0, padded_cells = 0, total_blocks = 0;
-  int max_ncols = 0;
+  int max_ncols = 0, min_ncols = 0;
 };
 
 // Validation of the whole batch. Errors land in scal->err (read back by pass_prepare).
@@ -273,7 +274,8 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
 
   k_pair_bins<K><<<grid_for(c, n), kThreads, 0, s>>>(
       d.pairs, list, nullptr, n, d.roff, d.n_reads, d.hoff, d.n_haps, c->bucket, pair_bin, pair_nb, bins,
-      bins + nb1, &scal->max_ncols, &scal->cells, &scal->padded_cells, &scal->total_blocks, &scal->err);
+      bins + nb1, &scal->max_ncols, &scal->min_ncols_c, &scal->cells, &scal->padded_cells, &scal->total_blocks,
+      &scal->err);
   LAUNCHED(c);
 
   // table items and their block offsets (exclusive scan over n_items + 1)
@@ -352,6 +354,7 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   pi->padded_cells = c->host_scal->padded_cells;
   pi->total_blocks = c->host_scal->total_blocks;
   pi->max_ncols = c->host_scal->max_ncols;
+  pi->min_ncols = kNcolsComplement - c->host_scal->min_ncols_c;
   // block descriptors address tables and code regions with 32-bit offsets
   if (hsz[0] > 0xffffffffLL || pi->total_blocks > 0x7fffffffULL) return PHMM_E_INVALID_ARG;
   *total_tab_out = hsz[0];
@@ -478,17 +481,23 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   int end_bit = 1;
   while ((1 << end_bit) <= kMaxBins + 1) ++end_bit;
   size_t sort_bytes = 0, scan_bytes = 0;
-  CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+  // one length bin (every pair the same column count, e.g. C2): the stable sort is the identity
+  const bool one_bin = pi.min_ncols == pi.max_ncols;
+  const int32_t* sorted = one_bin ? vals : vals + n;
+  if (!one_bin)
+    CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
   CUDA_TRY(cub::DeviceScan::ExclusiveSum(nullptr, scan_bytes, nbs, blk_off, n + 1, s));
   unsigned char* tmp;
   ST_TRY(ws(c, B_SORT_TMP, std::max(sort_bytes, scan_bytes), &tmp));
-  CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
-  c->launches += 2;
-  k_sorted_nb<<<grid_for(c, n), kThreads, 0, s>>>(vals + n, pair_nb, n, nbs);
+  if (!one_bin) {
+    CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+    c->launches += 2;
+  }
+  k_sorted_nb<<<grid_for(c, n), kThreads, 0, s>>>(sorted, pair_nb, n, nbs);
   LAUNCHED(c);
   CUDA_TRY(cub::DeviceScan::ExclusiveSum(tmp, scan_bytes, nbs, blk_off, n + 1, s));
   ++c->launches;
-  k_alloc_blocks_wf<K><<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, pair_item, vals + n, n, pair_nb, blk_off,
+  k_alloc_blocks_wf<K><<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, pair_item, sorted, n, pair_nb, blk_off,
                                                            d.roff, d.hoff, hc_off, item_off, blk);
   LAUNCHED(c);
 

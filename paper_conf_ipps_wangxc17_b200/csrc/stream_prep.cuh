@@ -88,6 +88,12 @@ __global__ void k_hap_ncols(const int64_t* __restrict__ hoff, int64_t n_haps, in
 //   D^ = M^(left) + mu D^(left),  I^ = M^(up) + ep' I^(up),
 //   M^ = T[code] * (M^(diag) + u I^(diag) + w D^(diag)).
 constexpr int kTabThreads = 256;
+// a / b in the table's precision: FP32 tables use the 2-ulp hardware division (7 divisions per
+// row dominate the kernel; 2 ulp per coefficient is far inside the FP32 pass's 1e-3 log10
+// tolerance), FP64 tables the correctly rounded one
+__device__ __forceinline__ float tdiv(float a, float b) { return __fdividef(a, b); }
+__device__ __forceinline__ double tdiv(double a, double b) { return a / b; }
+
 template <typename T>
 __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
     const int32_t* __restrict__ item_read, int64_t n_items, const int64_t* __restrict__ item_tab_off,
@@ -133,14 +139,14 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
       if (i == 0) {
         a = de1;
       } else if (real) {
-        const T k = (i < m) ? fmin((T)1, err[qi[x + 1] & 127] / ed) : (T)1;
+        const T k = (i < m) ? fmin((T)1, tdiv(err[qi[x + 1] & 127], ed)) : (T)1;
         a = k * ed;
         d = k;
       }
       T ap = __shfl_up_sync(0xffffffffu, a, 1);
       if (lane == 0) ap = ca;
       // b = a_{i-1} / delta_i (b_1 = 1)
-      const T b = (real && i >= 2) ? ap / ei : (T)1;
+      const T b = (real && i >= 2) ? tdiv(ap, ei) : (T)1;
       T bp = __shfl_up_sync(0xffffffffu, b, 1), dp = __shfl_up_sync(0xffffffffu, d, 1);
       if (lane == 0) { bp = cb; dp = cd; }
       ca = __shfl_sync(0xffffffffu, a, 31);
@@ -156,22 +162,22 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
       } else if (real) {
         const T al = (T)1 - fmin(ei + ed, (T)1);  // > 0.0065 after validation (R16)
         const T be = (T)1 - eg;
-        const T g = be * ap / al;
-        uu = g / bp;
-        ww = g / dp;
-        ep = eg * b / bp;
+        const T g = tdiv(be * ap, al);
+        uu = tdiv(g, bp);
+        ww = tdiv(g, dp);
+        ep = tdiv(eg * b, bp);
         mu = eg;
-        const T t = a * al / ap;
-        const T pm = t * ((T)1 - eb), px = t * (eb / (T)3);
+        const T t = tdiv(a * al, ap);
+        const T pm = t * ((T)1 - eb), px = t * tdiv(eb, (T)3);
         p5[0] = (base_c == 'A' || base_c == 'N') ? pm : px;
         p5[1] = (base_c == 'C' || base_c == 'N') ? pm : px;
         p5[2] = (base_c == 'G' || base_c == 'N') ? pm : px;
         p5[3] = (base_c == 'T' || base_c == 'N') ? pm : px;
         p5[4] = pm;  // haplotype 'N' matches everything
       } else {  // S: M^ = (M + I)(m, j-1), D^ = running sum (the L20@2262 termination)
-        uu = ap / bp;
+        uu = tdiv(ap, bp);
         mu = 1;
-        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = (T)1 / ap;
+        p5[0] = p5[1] = p5[2] = p5[3] = p5[4] = tdiv((T)1, ap);
       }
       TBlock<T>& B = Tb[row / K];
       const int t = row % K;

@@ -339,7 +339,7 @@ def _bench_kernel(lib: str, workload: str = "C2") -> dict:
     return json.loads(res.stdout.strip().splitlines()[-1])
 
 
-def main(out_path: str = os.path.join(ROOT, "profiles", "r01_shuffle_study.json")) -> dict:
+def main(out_path: str = os.path.join(ROOT, "profiles", "r02_shuffle_study.json")) -> dict:
     """Run the microbenchmarks, bench design B (libphmm.so) and design A
     (libphmm_xsmem.so) on C2, and instantiate Eq. 7-8 for both."""
     import torch
@@ -356,9 +356,12 @@ def main(out_path: str = os.path.join(ROOT, "profiles", "r01_shuffle_study.json"
         ptx = os.path.join(_PKG, "ptxas_info.txt") if tag.startswith("B") else lib + ".ptxas.txt"
         mangled = WF32_SYMBOL
         regs = _ptxas_regs(ptx, mangled) or 0
-        ncols = 304  # C2: N = 300 -> ncols 304, P = 312, ring 316 slots of 16 B
-        # wf_warp_smem<float>: prior tables + ring (+ design A's line buffer) + segment table
-        smem_block = 4 * ((2 * 6 * 2 * 32 * 16 + (316 + (32 if tag.startswith("A") else 0)) * 16 + 32 + 15) & ~15)
+        # C2: N = 300 -> ncols 304, P = 304 + 8 + 4 = 316 (staged switch), ring 320 + 4 slots of 16 B
+        ncols = 304
+        # wf_warp_smem<float>: prior tables + staging slots (8 x 144 B) + ring (+ design A's line
+        # buffer) + the stream's first block
+        smem_block = 4 * ((2 * 6 * 2 * 32 * 16 + 8 * 144 + (324 + (32 if tag.startswith("A") else 0)) * 16 + 32 + 15)
+                          & ~15)
         designs[tag] = {"lib": os.path.relpath(lib, ROOT), "kernel_gcups": r["achieved"], "frac": r["frac"],
                         "wavefront_ms": r["wavefront_ms"], "step_gcups": b["value"], "regs_per_thread": regs,
                         "smem_per_block": smem_block, "ncols": ncols,
