@@ -356,12 +356,22 @@ def main():
 
     from paper_conf_ipps_wangxc17_b200 import parallel, phmm, synth
 
+    # PHMM_BENCH_BACKEND=gloo (tests only): ranks may share a GPU and the result gather goes
+    # through host memory -- exercises the N > 1 path on a one-GPU box; NCCL is the product path
+    backend = os.environ.get("PHMM_BENCH_BACKEND", "nccl")
+    if backend not in ("nccl", "gloo"):
+        raise SystemExit(f"PHMM_BENCH_BACKEND must be nccl or gloo, not {backend!r}")
+    local = local % max(1, torch.cuda.device_count()) if backend == "gloo" else local
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     gloo = None
     if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
-        gloo = dist.new_group(backend="gloo")  # host-side reductions / the e2e legs' host gather
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+            gloo = dist.new_group(backend="gloo")  # host-side reductions / the e2e legs' host gather
+        else:
+            dist.init_process_group("gloo")
+            gloo = dist.group.WORLD
 
     scaling = args.scaling or ("strong" if args.workload == "C5" else "weak")
     n_regions = args.regions or DEFAULT_REGIONS[args.workload]
@@ -393,7 +403,7 @@ def main():
         ctx.compute_batch_dev(db, out=out, status=status)
         if ws > 1:
             with torch.cuda.stream(stream):
-                gathered[0] = parallel.gather_slots(slot, ws)
+                gathered[0] = parallel.gather_slots(slot if backend == "nccl" else slot.cpu(), ws)
 
     for _ in range(max(args.warmup, 0)):
         step()
