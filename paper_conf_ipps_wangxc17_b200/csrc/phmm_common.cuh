@@ -67,7 +67,7 @@ struct BlkDesc {
   uint32_t tab_blk;   // block index in the coefficient table
   uint32_t hap_off;   // offset of the haplotype in the code array
   int32_t out_idx;    // output slot of the pair (valid on its last block)
-  uint16_t n;         // haplotype length N
+  uint16_t pad;       // unused (keeps the descriptor 16 bytes)
   uint16_t flags;     // bit0: last block of its pair, bit1: first block of its pair
 };
 static_assert(sizeof(BlkDesc) == 16, "BlkDesc must be 16 bytes");

@@ -47,6 +47,7 @@ enum BufId {
   B_CH_ROFF, B_CH_HOFF, B_CH_PAIRS,            // chunked device call: one chunk's offsets / rebased pairs
   B_DEDUP,                                       // rescue pass: head flags + their scan (one table per read)
   B_CH_RANGES,                                   // chunked device call: read / haplotype index range per chunk
+  B_UNDERFLOW,                                   // pairs of the call whose FP64 sum underflowed
   B_COUNT
 };
 
@@ -113,6 +114,8 @@ struct phmm_ctx {
   int launches = 0;
   int64_t chunk_pairs = kDevChunkPairs;   // PHMM_CHUNK_PAIRS=n overrides (tests)
   uint32_t* host_ranges = nullptr;        // pinned: per-chunk index ranges of a chunked call
+  unsigned long long* host_underflow = nullptr;  // pinned: the call's FP64 underflow count (read at its end)
+  bool timing_deferred = false;           // one-chunk call: phase times read after the final sync
   int64_t host_ranges_n = 0;
 };
 
@@ -578,15 +581,13 @@ phmm_status rescue_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   double* out64;
   ST_TRY(ws(c, B_OUT64, (size_t)nr, &out64));
   ST_TRY((pass_run<double>(c, d, rlist, nr, pr, tab_r, hc, total_hc, out64, false)));
-  CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
+  unsigned long long* uf;
+  ST_TRY(ws(c, B_UNDERFLOW, 1, &uf));
   k_finalize_fp64<<<grid_for(c, nr), kThreads, 0, s>>>(out64, rlist, nullptr, nr, d.pairs, d.hoff, c->bucket, dev_out,
-                                                       dev_status, dev_status != nullptr, 1, &scal->n_underflow);
+                                                       dev_status, dev_status != nullptr, 1, uf);
   LAUNCHED(c);
   c->st.padded_cells += (int64_t)pr.padded_cells;
   if (timed) ev_record(c, EV_RESC1);
-  CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
-  CUDA_TRY(cudaStreamSynchronize(s));
-  c->st.n_fp64_underflow += (int64_t)c->host_scal->n_underflow;
   return PHMM_OK;
 }
 
@@ -629,16 +630,13 @@ phmm_status compute_one(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     ST_TRY(ws(c, B_OUT64, (size_t)d.n_pairs, &out64));
     ev_record(c, EV_PREP);
     ST_TRY((pass_run<double>(c, d, nullptr, d.n_pairs, pi, total_tab, hc, total_hc, out64, true)));
-    CUDA_TRY(cudaMemsetAsync(&scal->n_underflow, 0, sizeof(unsigned long long), s));
+    unsigned long long* uf;
+    ST_TRY(ws(c, B_UNDERFLOW, 1, &uf));
     k_finalize_fp64<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out64, nullptr, nullptr, d.n_pairs, d.pairs,
                                                                   d.hoff, c->bucket, dev_out,
-                                                                  dev_status, dev_status != nullptr, 0,
-                                                                  &scal->n_underflow);
+                                                                  dev_status, dev_status != nullptr, 0, uf);
     LAUNCHED(c);
     ev_record(c, EV_FIN);
-    CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
-    CUDA_TRY(cudaStreamSynchronize(s));
-    c->st.n_fp64_underflow += (int64_t)c->host_scal->n_underflow;
     c->st.cells += (int64_t)pi.cells;
     c->st.padded_cells += (int64_t)pi.padded_cells;
   } else {
@@ -654,7 +652,7 @@ phmm_status compute_one(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     if (nr > 0) ST_TRY(rescue_pass(c, d, dev_out, dev_status, rlist, nr, hc, total_hc, true));
     else ev_record(c, EV_RESC1);
   }
-  acc_phases(c);
+  if (!c->timing_deferred) acc_phases(c);
   ++c->st.n_chunks;
   return PHMM_OK;
 }
@@ -670,9 +668,15 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   c->st = phmm_stats{};
   c->acc = PhaseMs{};
   c->st.n_pairs = d.n_pairs;
+  c->timing_deferred = false;
   if (d.n_pairs == 0) return PHMM_OK;
   ST_TRY(run_validate(c, d));
+  unsigned long long* uf;
+  ST_TRY(ws(c, B_UNDERFLOW, 1, &uf));
+  CUDA_TRY(cudaMemsetAsync(uf, 0, sizeof(unsigned long long), s));
   const int64_t cp = c->chunk_pairs;
+  // one chunk: the phase times and the underflow count are read after the call's final sync
+  c->timing_deferred = d.n_pairs <= cp;
   if (d.n_pairs <= cp) return compute_one(c, d, dev_out, dev_status);
   // chunk k = pairs [k*cp, min((k+1)*cp, n)); its read / haplotype index ranges in one pass
   const int64_t nch = (d.n_pairs + cp - 1) / cp;
@@ -862,7 +866,22 @@ phmm_status check_batch_args(const phmm_batch* b) {
   return PHMM_OK;
 }
 
+// Enqueue the read-back of the call's FP64 underflow count (before the call's final sync).
+phmm_status enqueue_underflow_readback(phmm_ctx* c) {
+  if (c->st.n_pairs == 0) return PHMM_OK;
+  unsigned long long* uf;
+  ST_TRY(ws(c, B_UNDERFLOW, 1, &uf));
+  CUDA_TRY(cudaMemcpyAsync(c->host_underflow, uf, sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
+  return PHMM_OK;
+}
+
+// After the call's final sync: the statistics read at the end.
 void finish_stats(phmm_ctx* c) {
+  if (c->st.n_pairs > 0) c->st.n_fp64_underflow = (int64_t)*c->host_underflow;
+  if (c->timing_deferred) {
+    acc_phases(c);
+    c->timing_deferred = false;
+  }
   c->st.kernel_launches = c->launches;
   if (c->flags & PHMM_FLAG_TIMING) {
     cudaEventSynchronize(c->ev[EV_END]);
@@ -935,6 +954,7 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
     cudaGetLastError();
     return st;
   }
+  ST_TRY(enqueue_underflow_readback(c));
   ev_record(c, EV_D2H);
   {
     Nvtx nv("phmm:d2h");
@@ -1208,6 +1228,11 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
     c->host_sizes = nullptr;
     return fail(PHMM_E_OOM);
   }
+  if (cudaMallocHost(&c->host_underflow, sizeof(unsigned long long)) != cudaSuccess) {
+    c->host_underflow = nullptr;
+    return fail(PHMM_E_OOM);
+  }
+  *c->host_underflow = 0;
   for (int i = 0; i < kEvents; ++i)
     if (cudaEventCreate(&c->ev[i]) != cudaSuccess) return fail(PHMM_E_CUDA);
   {
@@ -1236,6 +1261,7 @@ void phmm_destroy(phmm_ctx* c) {
   if (c->host_scal) cudaFreeHost(c->host_scal);
   if (c->host_sizes) cudaFreeHost(c->host_sizes);
   if (c->host_ranges) cudaFreeHost(c->host_ranges);
+  if (c->host_underflow) cudaFreeHost(c->host_underflow);
   if (c->owned_stream) {
     cudaStreamSynchronize(c->owned_stream);
     cudaStreamDestroy(c->owned_stream);
@@ -1386,6 +1412,7 @@ phmm_status phmm_compute_batch_dev(phmm_ctx* c, const phmm_batch* b, double* dev
     if (dev_status)
       CUDA_TRY(cudaMemcpyAsync(dev_status, status, (size_t)b->n_pairs, cudaMemcpyDeviceToDevice, c->stream));
   }
+  ST_TRY(enqueue_underflow_readback(c));
   ev_record(c, EV_END);
   if (cudaStreamSynchronize(c->stream) != cudaSuccess) {
     cudaGetLastError();

@@ -207,10 +207,12 @@ __global__ void k_sorted_nb(const int32_t* __restrict__ sorted_idx, const int32_
   if (blockIdx.x == 0 && threadIdx.x == 0) nb_sorted[n] = 0;
 }
 
-// Block descriptors: one warp per 32 sorted entries, the lanes of the warp write one
-// pair's descriptors together (coalesced 16-byte stores). Entry k of the pass is pair
-// list[k] (or k when list == nullptr); its table item is pair_item[k] (or its read),
-// its output slot k (list) or the pair id.
+// Block descriptors: one warp per 32 sorted entries, whose blocks are one contiguous range
+// (blk_off is an exclusive scan in sorted order); the lanes write that range as consecutive
+// 16-byte descriptors (coalesced), each finding its entry by a binary search over the 32
+// entries' first blocks held in the lanes. Entry k of the pass is pair list[k] (or k when
+// list == nullptr); its table item is pair_item[k] (or its read), its output slot k (list) or
+// the pair id.
 template <int K>
 __global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32_t* __restrict__ list,
                                   const int32_t* __restrict__ pair_item, const int32_t* __restrict__ sorted_idx,
@@ -222,40 +224,49 @@ __global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < n; base += stride) {
     const int64_t i = base + lane;
-    int nb = 0, m = 0, nh = 0;
-    int64_t g0 = 0, slot = 0;
+    int nb = 0, f = 0;
+    int64_t g0 = INT64_MAX, slot = 0;
     uint32_t tab0 = 0, hap = 0;
     if (i < n) {
       const int64_t k = sorted_idx[i];
       const int64_t p = list ? list[k] : k;
       nb = pair_nb[k];
       const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
-      m = (int)(roff[r + 1] - roff[r]);
-      nh = (int)(hoff[h + 1] - hoff[h]);
+      const int m = (int)(roff[r + 1] - roff[r]);
+      f = nb * K - (m + 2);  // R row index within the pair's rows (f >= 1 Z rows before it)
       g0 = blk_off[i];
       tab0 = (uint32_t)item_tab_off[pair_item ? pair_item[k] : r];
       hap = (uint32_t)(hc_off[h] + WF_HC_FRONT);
       slot = list ? k : p;
     }
     const int cnt = (int)min((int64_t)32, n - base);
-    for (int src = 0; src < cnt; ++src) {
-      const int nb_s = __shfl_sync(0xffffffffu, nb, src);
-      const int m_s = __shfl_sync(0xffffffffu, m, src);
-      const int nh_s = __shfl_sync(0xffffffffu, nh, src);
-      const int64_t g0_s = __shfl_sync(0xffffffffu, g0, src);
-      const int64_t slot_s = __shfl_sync(0xffffffffu, slot, src);
-      const uint32_t tab_s = __shfl_sync(0xffffffffu, tab0, src);
-      const uint32_t hap_s = __shfl_sync(0xffffffffu, hap, src);
-      const int f = nb_s * K - (m_s + 2);  // R row index within the pair's rows (f >= 1 Z rows before it)
-      for (int j = lane; j < nb_s; j += 32) {
+    const int64_t first = __shfl_sync(0xffffffffu, g0, 0);
+    const int64_t last = __shfl_sync(0xffffffffu, g0, cnt - 1) + __shfl_sync(0xffffffffu, nb, cnt - 1);
+    for (int64_t pos = first + lane; pos - lane < last; pos += 32) {
+      // owner entry: the last of the (ascending) first blocks <= pos
+      int e = 0;
+#pragma unroll
+      for (int st = 16; st > 0; st >>= 1) {
+        const int cand = e + st;
+        const int64_t gc = __shfl_sync(0xffffffffu, g0, cand & 31);
+        if (cand < cnt && gc <= pos) e = cand;
+      }
+      const int64_t g0e = __shfl_sync(0xffffffffu, g0, e);
+      const int nbe = __shfl_sync(0xffffffffu, nb, e);
+      const int fe = __shfl_sync(0xffffffffu, f, e);
+      const int64_t slote = __shfl_sync(0xffffffffu, slot, e);
+      const uint32_t tabe = __shfl_sync(0xffffffffu, tab0, e);
+      const uint32_t hape = __shfl_sync(0xffffffffu, hap, e);
+      if (pos < last) {
+        const int j = (int)(pos - g0e);
         BlkDesc d;
-        d.tab_blk = tab_s + j;
-        d.hap_off = hap_s;
-        d.out_idx = (int32_t)slot_s;
-        d.n = (uint16_t)nh_s;
-        const int rrow = (f / K == j) ? (f % K) : WF_RROW_NONE;
-        d.flags = (uint16_t)((j == nb_s - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) | (rrow << WF_RROW_SHIFT));
-        blk[g0_s + j] = d;
+        d.tab_blk = tabe + j;
+        d.hap_off = hape;
+        d.out_idx = (int32_t)slote;
+        d.pad = 0;
+        const int rrow = (fe / K == j) ? (fe % K) : WF_RROW_NONE;
+        d.flags = (uint16_t)((j == nbe - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) | (rrow << WF_RROW_SHIFT));
+        blk[pos] = d;
       }
     }
   }

@@ -627,7 +627,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   int c31B = -(1 << 20);  // (uniform) column of virtual lane 63 (lane 31, half B)
   T rvM = 0, rvI = 0, rvD = 0;  // lane 31: ring slot for virtual lane 0's next column
   BlkDesc dnA, dnB;  // descriptors of the lane's next blocks (loaded one pass ahead)
-  dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.n = 1; dnA.flags = 0;
+  dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.pad = 0; dnA.flags = 0;
   dnB = dnA;
   if (2 * lane < nblk) dnA = A.blk[phys(2 * lane)];
   if (2 * lane + 1 < nblk) dnB = A.blk[phys(2 * lane + 1)];

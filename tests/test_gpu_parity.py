@@ -141,6 +141,7 @@ def test_fp64_underflow_gives_minus_inf(ctx32):
     got, st = ctx32.compute_batch(b)
     assert oracle.batch_log10(b)[0] < -2000
     assert np.isneginf(got[0]) and st[0] == 2
+    assert ctx32.stats()["n_fp64_underflow"] == 1 and ctx32.stats()["n_rescued"] == 1
 
 
 def test_order_and_batch_invariance_bitwise(ctx32):
