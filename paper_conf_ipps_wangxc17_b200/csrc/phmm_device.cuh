@@ -309,15 +309,6 @@ __global__ void k_rescue_items_dedup(const uint32_t* __restrict__ sorted_read, c
   }
 }
 
-// item list of the rescue pass: one table item per rescued pair (its read)
-__global__ void k_rescue_items(const int32_t* __restrict__ pairs, const int32_t* __restrict__ list,
-                               int64_t n, int32_t* __restrict__ item_read,
-                               int32_t* __restrict__ pair_item) {
-  for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
-    item_read[k] = pairs[2 * (int64_t)list[k]];
-    pair_item[k] = (int32_t)k;
-  }
-}
 
 // exclusive scan of bins + work items (single block; nbins <= kMaxBins)
 // Work items of each bin (the length-binned scheduler). A launch runs the

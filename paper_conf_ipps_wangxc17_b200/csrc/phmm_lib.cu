@@ -288,36 +288,31 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
     int32_t* pair_item;
     ST_TRY(ws(c, B_ITEM_READ, (size_t)n, &item_read));
     ST_TRY(ws(c, B_PAIR_ITEM, (size_t)n, &pair_item));
-    if (WF_RESCUE_DEDUP) {
-      // one table per distinct read of the listed pairs (the rescued pairs of a read share it):
-      // radix sort of the read ids, head flags, inclusive scan -> item of every listed pair
-      uint32_t* keys;
-      int32_t *vals, *head, *incl;
-      ST_TRY(ws(c, B_SKEYS, (size_t)2 * n, &keys));
-      ST_TRY(ws(c, B_SVALS, (size_t)2 * n, &vals));
-      ST_TRY(ws(c, B_DEDUP, (size_t)2 * n, &head));
-      incl = head + n;
-      k_rescue_read_keys<<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, n, keys, vals);
-      LAUNCHED(c);
-      int end_bit = 1;
-      while (end_bit < 32 && (1ll << end_bit) <= d.n_reads) ++end_bit;
-      size_t sb = 0, cb = 0;
-      CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sb, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
-      CUDA_TRY(cub::DeviceScan::InclusiveSum(nullptr, cb, head, incl, n, s));
-      unsigned char* tmp;
-      ST_TRY(ws(c, B_SORT_TMP, std::max(sb, cb), &tmp));
-      CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sb, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
-      k_rescue_head_flags<<<grid_for(c, n), kThreads, 0, s>>>(keys + n, n, head);
-      LAUNCHED(c);
-      CUDA_TRY(cub::DeviceScan::InclusiveSum(tmp, cb, head, incl, n, s));
-      k_rescue_items_dedup<<<grid_for(c, n), kThreads, 0, s>>>(keys + n, vals + n, head, incl, n, item_read,
-                                                               pair_item);
-      LAUNCHED(c);
-      c->launches += 2;
-    } else {
-      k_rescue_items<<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, n, item_read, pair_item);
-      LAUNCHED(c);
-    }
+    // one table per distinct read of the listed pairs (the rescued pairs of a read share it):
+    // radix sort of the read ids, head flags, inclusive scan -> item of every listed pair
+    uint32_t* keys;
+    int32_t *vals, *head, *incl;
+    ST_TRY(ws(c, B_SKEYS, (size_t)2 * n, &keys));
+    ST_TRY(ws(c, B_SVALS, (size_t)2 * n, &vals));
+    ST_TRY(ws(c, B_DEDUP, (size_t)2 * n, &head));
+    incl = head + n;
+    k_rescue_read_keys<<<grid_for(c, n), kThreads, 0, s>>>(d.pairs, list, n, keys, vals);
+    LAUNCHED(c);
+    int end_bit = 1;
+    while (end_bit < 32 && (1ll << end_bit) <= d.n_reads) ++end_bit;
+    size_t sb = 0, cb = 0;
+    CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sb, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+    CUDA_TRY(cub::DeviceScan::InclusiveSum(nullptr, cb, head, incl, n, s));
+    unsigned char* tmp;
+    ST_TRY(ws(c, B_SORT_TMP, std::max(sb, cb), &tmp));
+    CUDA_TRY(cub::DeviceRadixSort::SortPairs(tmp, sb, keys, keys + n, vals, vals + n, n, 0, end_bit, s));
+    k_rescue_head_flags<<<grid_for(c, n), kThreads, 0, s>>>(keys + n, n, head);
+    LAUNCHED(c);
+    CUDA_TRY(cub::DeviceScan::InclusiveSum(tmp, cb, head, incl, n, s));
+    k_rescue_items_dedup<<<grid_for(c, n), kThreads, 0, s>>>(keys + n, vals + n, head, incl, n, item_read,
+                                                             pair_item);
+    LAUNCHED(c);
+    c->launches += 2;
   }
   int64_t *item_nb, *item_off;
   ST_TRY(ws(c, B_ITEM_NB, (size_t)n_items + 1, &item_nb));

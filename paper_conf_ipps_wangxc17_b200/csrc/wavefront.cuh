@@ -447,10 +447,6 @@ __device__ __forceinline__ void wf_commit(Lane<T>& L, uint32_t stg_s, T d0) {
 #ifndef PHMM_RS_CAP
 #define PHMM_RS_CAP 126  // saturation of the scaled ring row (a saturated pair goes to the FP64 rescue)
 #endif
-#ifndef PHMM_RESCUE_DEDUP
-#define PHMM_RESCUE_DEDUP 1  // rescue pass: one FP64 table per distinct read, not per rescued pair
-#endif
-constexpr bool WF_RESCUE_DEDUP = PHMM_RESCUE_DEDUP;
 // Ring rescale helpers, used once per rescaled pass by the non-inlined
 // wf_ring_rescale, so they do not perturb the register allocation of the hot loop.
 // Max of the ring row (slots [0, ncols], every value incl. the FP32 slot padding, which is

@@ -478,3 +478,29 @@ def test_dev_variant_follows_torch_stream_and_leaves_outputs_on_error(ctx32):
             ctx32.compute_batch_dev(db, out=torch.empty(b.n_pairs, dtype=torch.float32, device="cuda:0"))
         with pytest.raises(ValueError):
             ctx32.compute_batch_dev(db, out=torch.empty(b.n_pairs - 1, dtype=torch.float64, device="cuda:0"))
+
+
+def test_full_c5_one_gpu_sampled(ctx32):
+    """BASELINE configs[4] at its stated size on one B200: 2^26 pairs (262,144 regions, 3.28e12
+    cells) in one device call, which runs as 8 chunks of 2^23 pairs. A seeded sample of pairs
+    plus rescued pairs against the oracle (1e-3), every result finite or -inf with a status,
+    and the chunked call's cell count equal to the job's."""
+    import torch
+
+    b = synth.config_batch("C5")
+    assert b.n_pairs == 1 << 26
+    db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+    out, st = ctx32.compute_batch_dev(db)
+    torch.cuda.synchronize()
+    stats = ctx32.stats()
+    assert stats["n_chunks"] == 8 and stats["cells"] == b.cells()
+    out = out.cpu().numpy()
+    st = st.cpu().numpy()
+    del db
+    torch.cuda.empty_cache()
+    assert np.all(np.isfinite(out) | np.isneginf(out)) and set(np.unique(st)) <= {0, 1, 2}
+    assert stats["n_rescued"] == int(np.sum(st >= 1))
+    rng = np.random.default_rng(55)
+    sample = np.unique(np.concatenate([rng.choice(b.n_pairs, 4000, replace=False),
+                                       rng.permutation(np.nonzero(st != 0)[0])[:1000]]))
+    _check(out[sample], oracle.batch_log10(b, pair_idx=sample), "fp32")
