@@ -504,3 +504,58 @@ def test_full_c5_one_gpu_sampled(ctx32):
     sample = np.unique(np.concatenate([rng.choice(b.n_pairs, 4000, replace=False),
                                        rng.permutation(np.nonzero(st != 0)[0])[:1000]]))
     _check(out[sample], oracle.batch_log10(b, pair_idx=sample), "fp32")
+
+
+@pytest.mark.parametrize("seed", [71, 72, 73, 74])
+def test_full_quality_ranges(ctx32, ctx64, seed):
+    """Base qualities over the whole accepted range Q0-127, indel qualities Q4-127 (R16 keeps
+    e(qi) + e(qd) <= 1), gap continuation Q1-127, 10 % 'N' bases, ragged lengths incl. m > N:
+    FP32 + rescue within 1e-3, FP64 within 1e-9 relative, -inf exactly where the oracle's is."""
+    b = synth.random_pairs_batch(seed, 300, m_range=(1, 150), n_range=(1, 220), qual_range=(0, 127),
+                                 indel_qual_range=(4, 127), gcp_range=(1, 127), n_frac=0.1)
+    ref = oracle.batch_log10(b)
+    # Q127 mismatches take P below the FP64 pass's range (scale 2^1020, DESIGN.md R7): the scaled
+    # FP64 sum is subnormal below log10 P = -614.7 (status 2, imprecise by design, not compared)
+    # and 0 below ~ -630 (-inf, status 2)
+    cmp = ref > -614
+    low = ref < -640
+    for ctx, mode in ((ctx32, "fp32"), (ctx64, "fp64")):
+        got, st = ctx.compute_batch(b)
+        _check(got[cmp], ref[cmp], mode)
+        assert np.all(np.isneginf(got[low])) and np.all(st[low] == 2)
+        assert np.all(st[~cmp] == 2)
+
+
+def test_device_call_argument_errors(ctx32):
+    """The device-buffer call rejects inconsistent sizes and offsets with PHMM_E_INVALID_ARG
+    (offsets not starting at 0, decreasing, or not ending at the total) and out-of-range pair
+    indices with PHMM_E_INDEX, leaving the outputs untouched."""
+    import torch
+
+    b = synth.random_pairs_batch(5, 30)
+    cases = []
+    ro = b.read_offsets.copy(); ro[3], ro[4] = ro[4], ro[3]       # decreasing
+    cases.append(("read_offsets", ro, -1))
+    ho = b.hap_offsets.copy(); ho[0] = 1                          # does not start at 0
+    cases.append(("hap_offsets", ho, -1))
+    pr = b.pairs.copy(); pr[4, 1] = -1                            # negative haplotype index
+    cases.append(("pairs", pr, -5))
+    for field, arr, code in cases:
+        bb = synth.Batch(**{**{k: getattr(b, k) for k in ("read_bases", "base_quals", "ins_quals", "del_quals",
+                                                         "gcp_quals", "read_offsets", "hap_bases",
+                                                         "hap_offsets", "pairs")}, field: arr})
+        db = phmm.DeviceBatch.from_host(bb, device="cuda:0")
+        o = torch.full((b.n_pairs,), 3.0, dtype=torch.float64, device="cuda:0")
+        with pytest.raises(phmm.PhmmError) as ei:
+            ctx32.compute_batch_dev(db, out=o)
+        assert ei.value.code == code, (field, ei.value.code)
+        assert bool(torch.all(o == 3.0))
+    # a total that disagrees with the offsets (the host variant checks it on the host)
+    import ctypes
+
+    st, keep = phmm._host_struct(b)
+    st.total_read_bases -= 1
+    out = np.full(b.n_pairs, 3.0)
+    rc = ctx32._L.phmm_compute_batch(ctx32._h, ctypes.byref(st), out.ctypes.data_as(phmm._f64p), None)
+    assert rc == -1 and np.all(out == 3.0)
+    del keep
