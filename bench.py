@@ -512,6 +512,15 @@ def main():
     extra = None
     if ws == 1 and not args.no_extra and not args.profile_steps and args.workload == "C2" and args.regions is None:
         extra = {"C3": run_extra(ctx, "C3", DEFAULT_REGIONS["C3"], args, stream, flush)}
+        # the FP64 path (PHMM_PREC_FP64, BASELINE configs[0]'s precision) on the whole of C2,
+        # against the FP64 pipe roofline (64 FP64 lanes per SM, 8 ops per cell)
+        ctx64 = phmm.PairHMM(device=local, precision="fp64", stream=stream.cuda_stream, timing=True)
+        x = run_extra(ctx64, "C2", DEFAULT_REGIONS["C2"], args, stream, flush)
+        ctx64.close()
+        peak64 = nsm * FP64_LANES_PER_SM * sm_max * 1e6 / FP32_OPS_PER_CELL / 1e9
+        x.update({"precision": "fp64 (every pair)", "kernel": "k_wavefront<double>",
+                  "kernel_frac_fp64_roofline": x["kernel_gcups"] / peak64, "fp64_roofline_gcups": peak64})
+        extra["C2_fp64"] = x
 
     if rank == 0:
         split = (f"strong: the fixed {n_regions}-region job split over {ws} rank(s) by cells (whole regions)"
