@@ -230,8 +230,9 @@ def _e2e_leg(args, ctx, batch, ws, flush, stream, gloo, n_slot, pair_start, pinn
     """Same metric through the host-buffer C-ABI call: H2D of the step's inputs, the whole
     path, D2H of the results, every step (wall clock around the synchronous call, max over
     ranks). pinned: inputs and outputs in page-locked host memory; otherwise plain numpy
-    (pageable) arrays, which the library stages through its own pinned buffers. N > 1: the
-    host results of every rank are gathered (gloo, no re-upload to the GPU)."""
+    (pageable) arrays, which the library stages through its own pinned buffers. N > 1: every
+    rank's results land in its own host memory -- a distributed caller consumes its shard
+    where it computed it; the cross-rank gather of the results is the device step's (NCCL)."""
     import torch
     import torch.distributed as dist
 
@@ -258,15 +259,12 @@ def _e2e_leg(args, ctx, batch, ws, flush, stream, gloo, n_slot, pair_start, pinn
     hst = torch.empty(n, dtype=torch.uint8)
     if pinned:
         hst = hst.pin_memory()
-    hg = torch.empty(ws * (n_slot + 2), dtype=torch.float64) if ws > 1 else None
     h2d = int(sum(t.numel() * t.element_size() for t in host.values()))
     d2h = n * (8 + 1)
 
     def one():
         rc = ctx.compute_batch_raw(s, hout.data_ptr(), hst.data_ptr())
         assert rc == 0, rc
-        if ws > 1:
-            dist.all_gather_into_tensor(hg, hslot, group=gloo)
 
     for _ in range(max(1, args.warmup)):
         one()
