@@ -113,7 +113,6 @@ struct phmm_ctx {
   PhaseMs acc{};                          // per-phase times summed over a call's chunks
   int launches = 0;
   int64_t chunk_pairs = kDevChunkPairs;   // PHMM_CHUNK_PAIRS=n overrides (tests)
-  int f64_conc = 0;  // experiment: PHMM_F64_CONC=b runs FP64 passes as b one-warp CTAs per SM
   uint32_t* host_ranges = nullptr;        // pinned: per-chunk index ranges of a chunked call
   unsigned long long* host_underflow = nullptr;  // pinned: the call's FP64 underflow count (read at its end)
   bool timing_deferred = false;           // one-chunk call: phase times read after the final sync
@@ -437,7 +436,6 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   Launch L[2];
   int nl = 0;
   L[nl++] = Launch{0, std::min(bin_cut, kMaxBins + 1), WF_WARPS, std::min(p_max + 4, ring_full), bps_full};
-  if (sizeof(T) == 8 && c->f64_conc > 0) { L[0].warps = 1; L[0].bps = c->f64_conc; }
   if (bin_cut <= kMaxBins) {
     Launch lb{bin_cut, kMaxBins + 1, 0, p_max + 8, 0};  // global ring: prefetch reads up to slot P + 4
     int best = 0;
@@ -1241,7 +1239,6 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
     }
   }
   if (const char* e = std::getenv("PHMM_CHUNK_PAIRS")) c->chunk_pairs = std::max<int64_t>(64, std::atoll(e));
-  if (const char* e = std::getenv("PHMM_F64_CONC")) c->f64_conc = std::max(0, std::atoi(e));
   *out = c;
   return PHMM_OK;
 }

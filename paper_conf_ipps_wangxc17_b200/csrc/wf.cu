@@ -4,8 +4,6 @@
 #define PHMM_DEFINE_WF
 #include "wavefront.cuh"
 
-#include <cstdlib>
-
 namespace phmm {
 
 template <typename T>
@@ -23,10 +21,6 @@ cudaError_t wf_set_max_smem(int smem_optin) {
   for (const void* f : fs) {
     cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin);
     if (e != cudaSuccess) return e;
-    if (std::getenv("PHMM_CARVEOUT")) {
-      e = cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-      if (e != cudaSuccess) return e;
-    }
   }
   return cudaSuccess;
 }
