@@ -33,9 +33,28 @@ __device__ __forceinline__ bool offset_bad(const int64_t* __restrict__ off, int6
   return bad;
 }
 
+// Four base letters in a 32-bit word, each one of A C G T N (SIMD byte compares).
+__device__ __forceinline__ bool bases_ok4(uint32_t w) {
+  const uint32_t m = __vcmpeq4(w, 0x41414141u) | __vcmpeq4(w, 0x43434343u) | __vcmpeq4(w, 0x47474747u) |
+                     __vcmpeq4(w, 0x54545454u) | __vcmpeq4(w, 0x4e4e4e4eu);
+  return m == 0xffffffffu;
+}
+
+// 4 read bases with their four qualities (one 32-bit word of each array).
+__device__ __forceinline__ uint32_t read_word_err(uint32_t b, uint32_t a, uint32_t x, uint32_t y, uint32_t z) {
+  // fast path: every byte a base letter, no quality byte >= 128, no indel quality <= 3
+  if (!((a | x | y | z) & 0x80808080u) && !__vcmpleu4(x, 0x03030303u) && !__vcmpleu4(y, 0x03030303u))
+    return bases_ok4(b) ? 0u : ERR_BASE;
+  uint32_t e = 0;
+  for (int k = 0; k < 4; ++k)
+    e |= read_base_err((uint8_t)(b >> 8 * k), (uint8_t)(a >> 8 * k), (uint8_t)(x >> 8 * k), (uint8_t)(y >> 8 * k),
+                       (uint8_t)(z >> 8 * k));
+  return e;
+}
+
 // The whole batch in one launch: every haplotype base, every read base with its four
-// qualities (4 bases per thread-step through 32-bit words where the five arrays share their
-// alignment), and both offset arrays. Errors are OR-ed into *err (one atomic per warp).
+// qualities (16 bases per thread-step through 16-byte vectors where the five arrays share
+// their alignment), and both offset arrays. Errors are OR-ed into *err (one atomic per warp).
 __global__ void k_validate(const uint8_t* __restrict__ hap, int64_t n_hb, const uint8_t* __restrict__ rb,
                            const uint8_t* __restrict__ q, const uint8_t* __restrict__ qi,
                            const uint8_t* __restrict__ qd, const uint8_t* __restrict__ qg, int64_t n_rb,
@@ -43,32 +62,51 @@ __global__ void k_validate(const uint8_t* __restrict__ hap, int64_t n_hb, const 
                            int64_t n_haps, uint32_t* err) {
   uint32_t e = 0;
   const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, nthr = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t i = tid; i < n_hb; i += nthr)
-    if (base_code(hap[i]) == 0xffu) e |= ERR_BASE;
-  // reads: a scalar head up to the first 4-aligned read byte, then words (when all five
-  // arrays are equally aligned), then a scalar tail
-  const uintptr_t mis = (uintptr_t)rb & 3;
-  const bool same = (((uintptr_t)q & 3) == mis) && (((uintptr_t)qi & 3) == mis) && (((uintptr_t)qd & 3) == mis) &&
-                    (((uintptr_t)qg & 3) == mis);
-  const int64_t head = same ? min(n_rb, (int64_t)((4 - mis) & 3)) : n_rb;
-  for (int64_t i = tid; i < head; i += nthr) e |= read_base_err(rb[i], q[i], qi[i], qd[i], qg[i]);
-  const int64_t nw = (n_rb - head) >> 2;
-  const uint32_t *rb4 = reinterpret_cast<const uint32_t*>(rb + head), *q4 = reinterpret_cast<const uint32_t*>(q + head),
-                 *i4 = reinterpret_cast<const uint32_t*>(qi + head), *d4 = reinterpret_cast<const uint32_t*>(qd + head),
-                 *g4 = reinterpret_cast<const uint32_t*>(qg + head);
-  for (int64_t w = tid; w < nw; w += nthr) {
-    const uint32_t b = rb4[w], a = q4[w], x = i4[w], y = d4[w], z = g4[w];
-    // fast path: every byte an uppercase base letter candidate and no quality byte >= 128 or <= 3
-    if (((a | x | y | z) & 0x80808080u) || __vcmpleu4(x, 0x03030303u) || __vcmpleu4(y, 0x03030303u)) {
-      for (int k = 0; k < 4; ++k)
-        e |= read_base_err((uint8_t)(b >> 8 * k), (uint8_t)(a >> 8 * k), (uint8_t)(x >> 8 * k),
-                           (uint8_t)(y >> 8 * k), (uint8_t)(z >> 8 * k));
-    } else {
-      for (int k = 0; k < 4; ++k)
-        if (base_code((uint8_t)(b >> 8 * k)) == 0xffu) e |= ERR_BASE;
+  // haplotypes: a scalar head up to 16-byte alignment, 16-byte vectors, a scalar tail
+  {
+    const int64_t head = min(n_hb, (int64_t)((16 - ((uintptr_t)hap & 15)) & 15));
+    for (int64_t i = tid; i < head; i += nthr)
+      if (base_code(hap[i]) == 0xffu) e |= ERR_BASE;
+    const int64_t nv = (n_hb - head) >> 4;
+    const uint4* h16 = reinterpret_cast<const uint4*>(hap + head);
+    for (int64_t v = tid; v < nv; v += nthr) {
+      const uint4 w = h16[v];
+      if (!(bases_ok4(w.x) && bases_ok4(w.y) && bases_ok4(w.z) && bases_ok4(w.w))) e |= ERR_BASE;
     }
+    for (int64_t i = head + 16 * nv + tid; i < n_hb; i += nthr)
+      if (base_code(hap[i]) == 0xffu) e |= ERR_BASE;
   }
-  for (int64_t i = head + 4 * nw + tid; i < n_rb; i += nthr) e |= read_base_err(rb[i], q[i], qi[i], qd[i], qg[i]);
+  // reads: the same, as 16-byte vectors of all five arrays when they share their alignment
+  // (else 4-byte words when they share it mod 4, else bytes)
+  auto same_mod = [&](uintptr_t m) {
+    const uintptr_t r = (uintptr_t)rb & m;
+    return (((uintptr_t)q & m) == r) && (((uintptr_t)qi & m) == r) && (((uintptr_t)qd & m) == r) &&
+           (((uintptr_t)qg & m) == r);
+  };
+  const int vec = same_mod(15) ? 16 : (same_mod(3) ? 4 : 1);
+  const int64_t head = vec == 1 ? n_rb : min(n_rb, (int64_t)((vec - ((uintptr_t)rb & (vec - 1))) & (vec - 1)));
+  for (int64_t i = tid; i < head; i += nthr) e |= read_base_err(rb[i], q[i], qi[i], qd[i], qg[i]);
+  int64_t done = head;
+  if (vec == 16) {
+    const int64_t nv = (n_rb - head) >> 4;
+    const uint4 *b16 = reinterpret_cast<const uint4*>(rb + head), *q16 = reinterpret_cast<const uint4*>(q + head),
+                *i16 = reinterpret_cast<const uint4*>(qi + head), *d16 = reinterpret_cast<const uint4*>(qd + head),
+                *g16 = reinterpret_cast<const uint4*>(qg + head);
+    for (int64_t v = tid; v < nv; v += nthr) {
+      const uint4 b = b16[v], a = q16[v], x = i16[v], y = d16[v], z = g16[v];
+      e |= read_word_err(b.x, a.x, x.x, y.x, z.x) | read_word_err(b.y, a.y, x.y, y.y, z.y) |
+           read_word_err(b.z, a.z, x.z, y.z, z.z) | read_word_err(b.w, a.w, x.w, y.w, z.w);
+    }
+    done = head + 16 * nv;
+  } else if (vec == 4) {
+    const int64_t nw = (n_rb - head) >> 2;
+    const uint32_t *b4 = reinterpret_cast<const uint32_t*>(rb + head), *q4 = reinterpret_cast<const uint32_t*>(q + head),
+                   *i4 = reinterpret_cast<const uint32_t*>(qi + head), *d4 = reinterpret_cast<const uint32_t*>(qd + head),
+                   *g4 = reinterpret_cast<const uint32_t*>(qg + head);
+    for (int64_t w = tid; w < nw; w += nthr) e |= read_word_err(b4[w], q4[w], i4[w], d4[w], g4[w]);
+    done = head + 4 * nw;
+  }
+  for (int64_t i = done + tid; i < n_rb; i += nthr) e |= read_base_err(rb[i], q[i], qi[i], qd[i], qg[i]);
   for (int64_t i = tid; i <= n_reads; i += nthr)
     if (offset_bad(roff, i, n_reads, n_rb)) e |= ERR_ARG;
   for (int64_t i = tid; i <= n_haps; i += nthr)
@@ -85,9 +123,14 @@ __global__ void k_validate_offsets(const int64_t* __restrict__ off, int64_t n, i
 
 // Per pair: validate indices/lengths, bin by column count, count blocks per bin.
 // pair_list == nullptr -> pairs 0..n-1, else the listed pair ids (rescue pass).
-// Counters are aggregated per warp (match_any + reduce) before one atomic per
-// distinct bin and per warp: with one length bin every pair would otherwise hit
-// the same address.
+// Counters are aggregated per warp (match_any + reduce), then per CTA in a shared-memory
+// histogram, which is flushed with one global atomic per non-empty bin and CTA: with one
+// length bin (C2) every warp would otherwise hit the same global address (32 K same-address
+// atomics per 2^20 pairs, 63 us; profiles/r02_timeline_C2.json). 32-bit shared counters:
+// the launch gives every CTA at most kPairBinsPerCta pairs of at most 2^18 blocks each
+// (nblocks_of<4>(kMaxReadLen)), so a CTA's count stays below 2^30.
+constexpr int64_t kPairBinsPerCta = 4096;
+constexpr int kPairBinsU = 4;  // pairs per lane per trip
 template <int K>
 __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __restrict__ pair_list,
                             const int64_t* __restrict__ n_list_dev, int64_t n_pairs,
@@ -99,50 +142,83 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
                             unsigned long long* __restrict__ cells,
                             unsigned long long* __restrict__ padded_cells, unsigned long long* __restrict__ total_blocks,
                             uint32_t* err) {
+  __shared__ uint32_t s_blk[kMaxBins + 1], s_cnt[kMaxBins + 1];
+  for (int i = threadIdx.x; i <= kMaxBins; i += blockDim.x) s_blk[i] = s_cnt[i] = 0u;
+  __syncthreads();
   const int64_t n = n_list_dev ? *n_list_dev : n_pairs;
   const int lane = threadIdx.x & 31;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   uint32_t e = 0;
   unsigned long long my_cells = 0, my_padded = 0, my_blocks = 0;
   int my_max = 0, my_minc = 0;  // my_minc = kNcolsComplement - smallest column count
-  for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < n; base += stride) {
-    const int64_t k = base + lane;
-    int bin = -1, nb = 0;
-    if (k < n) {
-      const int64_t p = pair_list ? pair_list[k] : k;
-      const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
-      if (r < 0 || r >= n_reads || h < 0 || h >= n_haps) {
-        e |= ERR_INDEX;
-      } else {
-        const int64_t m = roff[r + 1] - roff[r], nh = hoff[h + 1] - hoff[h];
-        if (m < 1 || nh < 1) {
-          e |= ERR_EMPTY;
-        } else if (nh > kMaxHapLen || m > kMaxReadLen) {
-          e |= ERR_ARG;
-        } else {
-          const int nc = ncols_of((int)nh, bucket);
-          bin = bin_of_ncols(nc, bucket);
-          nb = nblocks_of<K>((int)m);
-          my_max = max(my_max, nc);
-          my_minc = max(my_minc, kNcolsComplement - nc);
-          my_cells += (unsigned long long)(m * nh);
-          my_padded += (unsigned long long)nb * K * nc;
-          my_blocks += (unsigned long long)nb;
-        }
+  // kPairBinsU pairs per lane per trip, their loads issued together (the kernel is bound by
+  // the latency of the pairs -> offsets gather chain, not by bandwidth)
+  constexpr int U = kPairBinsU;
+  for (int64_t base = ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll) * U; base < n; base += stride * U) {
+    int32_t r[U], h[U];
+    int64_t r0[U], r1[U], h0[U], h1[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t k = base + 32 * u + lane;
+      r[u] = h[u] = -1;
+      if (k < n) {
+        const int64_t p = pair_list ? pair_list[k] : k;
+        r[u] = pairs[2 * p];
+        h[u] = pairs[2 * p + 1];
       }
-      pair_bin[k] = bin;
-      pair_nb[k] = nb;
     }
-    const unsigned act = __ballot_sync(0xffffffffu, bin >= 0);
-    if (bin >= 0) {
-      const unsigned peers = __match_any_sync(act, bin);
-      const unsigned sum_nb = __reduce_add_sync(peers, (unsigned)nb);
-      if (lane == __ffs(peers) - 1) {
-        atomicAdd(&bin_blocks[bin], (unsigned long long)sum_nb);
-        atomicAdd(&bin_pairs[bin], (unsigned long long)__popc(peers));
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool ok = r[u] >= 0 && r[u] < n_reads && h[u] >= 0 && h[u] < n_haps;
+      r0[u] = ok ? roff[r[u]] : 0;
+      r1[u] = ok ? roff[r[u] + 1] : 0;
+      h0[u] = ok ? hoff[h[u]] : 0;
+      h1[u] = ok ? hoff[h[u] + 1] : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int64_t k = base + 32 * u + lane;
+      int bin = -1, nb = 0;
+      if (k < n) {
+        if (r[u] < 0 || r[u] >= n_reads || h[u] < 0 || h[u] >= n_haps) {
+          e |= ERR_INDEX;
+        } else {
+          const int64_t m = r1[u] - r0[u], nh = h1[u] - h0[u];
+          if (m < 1 || nh < 1) {
+            e |= ERR_EMPTY;
+          } else if (nh > kMaxHapLen || m > kMaxReadLen) {
+            e |= ERR_ARG;
+          } else {
+            const int nc = ncols_of((int)nh, bucket);
+            bin = bin_of_ncols(nc, bucket);
+            nb = nblocks_of<K>((int)m);
+            my_max = max(my_max, nc);
+            my_minc = max(my_minc, kNcolsComplement - nc);
+            my_cells += (unsigned long long)(m * nh);
+            my_padded += (unsigned long long)nb * K * nc;
+            my_blocks += (unsigned long long)nb;
+          }
+        }
+        pair_bin[k] = bin;
+        pair_nb[k] = nb;
+      }
+      const unsigned act = __ballot_sync(0xffffffffu, bin >= 0);
+      if (bin >= 0) {
+        const unsigned peers = __match_any_sync(act, bin);
+        const unsigned sum_nb = __reduce_add_sync(peers, (unsigned)nb);
+        if (lane == __ffs(peers) - 1) {
+          atomicAdd(&s_blk[bin], sum_nb);
+          atomicAdd(&s_cnt[bin], (uint32_t)__popc(peers));
+        }
       }
     }
   }
+  __syncthreads();
+  for (int i = threadIdx.x; i <= kMaxBins; i += blockDim.x)
+    if (s_cnt[i]) {
+      atomicAdd(&bin_blocks[i], (unsigned long long)s_blk[i]);
+      atomicAdd(&bin_pairs[i], (unsigned long long)s_cnt[i]);
+    }
   // one atomic per warp for the scalars
   for (int o = 16; o > 0; o >>= 1) {
     my_cells += __shfl_xor_sync(0xffffffffu, my_cells, o);
@@ -350,65 +426,87 @@ __global__ void __launch_bounds__(1024) k_scan_bins(const unsigned long long* __
                                                     unsigned long long* __restrict__ item_start,
                                                     unsigned long long* __restrict__ bin_nbig,
                                                     unsigned long long* __restrict__ launch_items) {
-  __shared__ unsigned long long sh[1024];
-  // pass 1: first block of every bin (serial-by-tile scan: nbins is a few thousand at most)
-  unsigned long long carry = 0, tot;
-  for (int base = 0; base < nbins; base += 1024) {
-    const int i = base + threadIdx.x;
-    const unsigned long long vb = (i < nbins) ? bin_blocks[i] : 0ull;
-    const unsigned long long ex = block_scan_1024(vb, sh, &tot);
-    if (i < nbins) bin_start[i] = carry + ex;
-    carry += tot;
+  // every thread owns kPer consecutive bins (serial within the thread, one block scan over
+  // the 1024 thread sums per pass); the prefixes are kept in shared memory for the lookups
+  // of a neighbouring bin
+  constexpr int kPer = (kMaxBins + 1 + 1023) / 1024;
+  __shared__ unsigned long long sh[64];
+  __shared__ unsigned long long spre[kPer * 1024 + 1];
+  const int i0 = threadIdx.x * kPer;
+  unsigned long long vb[kPer], loc = 0, tot;
+#pragma unroll
+  for (int r = 0; r < kPer; ++r) {
+    vb[r] = (i0 + r < nbins) ? bin_blocks[i0 + r] : 0ull;
+    loc += vb[r];
   }
-  if (threadIdx.x == 0) bin_start[nbins] = carry;
+  // pass 1: first block of every bin
+  unsigned long long acc = block_scan_1024(loc, sh, &tot);
+  unsigned long long bs[kPer];
+#pragma unroll
+  for (int r = 0; r < kPer; ++r) {
+    bs[r] = acc;
+    acc += vb[r];
+    if (i0 + r < nbins) {
+      bin_start[i0 + r] = bs[r];
+      spre[i0 + r] = bs[r];
+    }
+  }
+  const unsigned long long Ball = tot;
+  if (threadIdx.x == 0) {
+    bin_start[nbins] = Ball;
+    spre[nbins] = Ball;
+  }
   __syncthreads();
   const int c = cut < 0 ? 0 : (cut > nbins ? nbins : cut);
-  const unsigned long long B0 = bin_start[c], Ball = carry;
+  const unsigned long long B0 = spre[c];
   const unsigned long long L0 = B0, L1 = Ball - B0;  // blocks of the two launches
   const unsigned long long thr0 = tail_div > 0 ? L0 - L0 / tail_div : L0;
   const unsigned long long thr1 = tail_div > 0 ? L1 - L1 / tail_div : L1;
-  // pass 2: items per bin (item_start: exclusive prefix in bin order for now)
-  carry = 0;
-  for (int base = 0; base < nbins; base += 1024) {
-    const int i = base + threadIdx.x;
-    unsigned long long vi = 0;
+  // pass 2: items per bin (exclusive prefix in ascending bin order)
+  unsigned long long vi[kPer];
+  loc = 0;
+#pragma unroll
+  for (int r = 0; r < kPer; ++r) {
+    const int i = i0 + r;
+    vi[r] = 0;
     if (i < nbins) {
-      const unsigned long long vb = bin_blocks[i];
       const bool l0 = i < c;
       // position of the bin's first block in its launch's order (ascending or, lpt, descending bins)
-      const unsigned long long pos = lpt ? (l0 ? B0 : Ball) - bin_start[i + 1] : bin_start[i] - (l0 ? 0ull : B0);
+      const unsigned long long pos = lpt ? (l0 ? B0 : Ball) - spre[i + 1] : bs[r] - (l0 ? 0ull : B0);
       const unsigned long long thr = l0 ? thr0 : thr1;
-      const unsigned long long big = thr <= pos ? 0ull : (thr - pos < vb ? thr - pos : vb);
-      const unsigned long long nbig = (big == vb) ? (vb + chunk - 1) / chunk : big / chunk;
-      const unsigned long long used = nbig * chunk < vb ? nbig * chunk : vb;
-      vi = nbig + (vb - used + chunk_s - 1) / chunk_s;
+      const unsigned long long big = thr <= pos ? 0ull : (thr - pos < vb[r] ? thr - pos : vb[r]);
+      const unsigned long long nbig = (big == vb[r]) ? (vb[r] + chunk - 1) / chunk : big / chunk;
+      const unsigned long long used = nbig * chunk < vb[r] ? nbig * chunk : vb[r];
+      vi[r] = nbig + (vb[r] - used + chunk_s - 1) / chunk_s;
       bin_nbig[i] = nbig;
     }
-    const unsigned long long ex = block_scan_1024(vi, sh, &tot);
-    if (i < nbins) item_start[i] = carry + ex;
-    carry += tot;
+    loc += vi[r];
   }
-  if (threadIdx.x == 0) item_start[nbins] = carry;
+  unsigned long long Iall;
+  acc = block_scan_1024(loc, sh, &Iall);  // (ends with a barrier: spre is free again)
+  unsigned long long is[kPer];
+#pragma unroll
+  for (int r = 0; r < kPer; ++r) {
+    is[r] = acc;
+    acc += vi[r];
+    if (i0 + r < nbins) spre[i0 + r] = is[r];
+  }
+  if (threadIdx.x == 0) {
+    spre[nbins] = Iall;
+    item_start[nbins] = Iall;
+  }
   __syncthreads();
-  const unsigned long long I0 = item_start[c], Iall = carry;
+  const unsigned long long I0 = spre[c];
   if (threadIdx.x == 0) {
     launch_items[0] = 0; launch_items[1] = I0; launch_items[2] = I0; launch_items[3] = Iall;
   }
-  if (lpt) {  // descending bins inside each launch: item_start[i] = launch base + items of the bins above i
-    constexpr int kPer = (kMaxBins + 1 + 1023) / 1024;
-    unsigned long long v[kPer];
 #pragma unroll
-    for (int r = 0; r < kPer; ++r) {  // read every old value before any is overwritten
-      const int i = threadIdx.x + 1024 * r;
-      const unsigned long long nxt = (i + 1 < nbins) ? item_start[i + 1] : Iall;
-      v[r] = (i < c) ? I0 - nxt : I0 + (Iall - nxt);
-    }
-    __syncthreads();
-#pragma unroll
-    for (int r = 0; r < kPer; ++r) {
-      const int i = threadIdx.x + 1024 * r;
-      if (i < nbins) item_start[i] = v[r];
-    }
+  for (int r = 0; r < kPer; ++r) {
+    const int i = i0 + r;
+    if (i >= nbins) break;
+    // lpt: descending bins inside each launch, item_start[i] = launch base + items of the bins above i
+    const unsigned long long nxt = spre[i + 1];
+    item_start[i] = !lpt ? is[r] : (i < c) ? I0 - nxt : I0 + (Iall - nxt);
   }
 }
 

@@ -275,7 +275,9 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   // per-pass scalars (err is kept: it accumulates validation errors)
   CUDA_TRY(cudaMemsetAsync(&scal->max_ncols, 0, offsetof(Scalars, n_rescue) - offsetof(Scalars, max_ncols), s));
 
-  k_pair_bins<K><<<grid_for(c, n), kThreads, 0, s>>>(
+  const int pb_grid = (int)std::max<int64_t>(grid_for(c, (n + kPairBinsU - 1) / kPairBinsU),
+                                              (n + kPairBinsPerCta - 1) / kPairBinsPerCta);
+  k_pair_bins<K><<<pb_grid, kThreads, 0, s>>>(
       d.pairs, list, nullptr, n, d.roff, d.n_reads, d.hoff, d.n_haps, c->bucket, pair_bin, pair_nb, bins,
       bins + nb1, &scal->max_ncols, &scal->min_ncols_c, &scal->cells, &scal->padded_cells, &scal->total_blocks,
       &scal->err);

@@ -39,21 +39,34 @@ __global__ void __launch_bounds__(kHcThreads) k_hap_codes_wf(const uint8_t* __re
     if (n < 1 || n > kMaxHapLen) continue;
     const int len = wf_hc_copy_len(ncols_of(n, bucket));  // multiple of 4, region start 4-aligned
     __syncwarp();
-    for (int b = lane; b < len + 4; b += 32) {  // byte b of copy 0 = column b - WF_HC_FRONT
-      const int c = b - (int)WF_HC_FRONT;
-      uint32_t v = WF_PAD;
-      if (c >= 0 && c < n) {
-        switch (hap[h0 + c]) {
-          case 'A': v = 0; break;
-          case 'C': v = 1; break;
-          case 'G': v = 2; break;
-          case 'T': v = 3; break;
-          default: v = 4; break;  // 'N' (invalid bytes were rejected by validation)
-        }
-      } else if (c == n) {
-        v = 4;
+    // byte b of copy 0 = column b - WF_HC_FRONT; 4 bytes per lane per trip, their loads
+    // issued before any is used (the loop is bound by load latency, one haplotype per warp)
+    for (int b0 = 0; b0 < len + 4; b0 += 128) {
+      uint8_t x[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int c = b0 + 32 * j + lane - (int)WF_HC_FRONT;
+        x[j] = (c >= 0 && c < n) ? hap[h0 + c] : (uint8_t)0;
       }
-      buf[b] = (uint8_t)(v * WF_CB);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int b = b0 + 32 * j + lane;
+        const int c = b - (int)WF_HC_FRONT;
+        if (b >= len + 4) break;
+        uint32_t v = WF_PAD;
+        if (c >= 0 && c < n) {
+          switch (x[j]) {
+            case 'A': v = 0; break;
+            case 'C': v = 1; break;
+            case 'G': v = 2; break;
+            case 'T': v = 3; break;
+            default: v = 4; break;  // 'N' (invalid bytes were rejected by validation)
+          }
+        } else if (c == n) {
+          v = 4;
+        }
+        buf[b] = (uint8_t)(v * WF_CB);
+      }
     }
     __syncwarp();
     uint32_t* dst = reinterpret_cast<uint32_t*>(codes + hc_off[h]);
