@@ -37,12 +37,6 @@
 
 namespace phmm {
 
-#if defined(PHMM_DBG_TRACE) && defined(PHMM_DEFINE_WF)
-// debug builds only: per-step last-row state (FP32 pass) of the warp that runs work item 0
-__device__ float g_trace[4096 * 32 * 2 * 3];
-__device__ int g_trace_steps;
-#endif
-
 #ifndef PHMM_F32_K
 #define PHMM_F32_K 8  // rows per half in the FP32 pass (8 or 4)
 #endif
@@ -575,7 +569,7 @@ __device__ __forceinline__ unsigned long long wf_claim(const WfArgs2<T>& A, int 
 template <typename T, bool kLong>
 __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, uint32_t ring_base_s,
                                           uint32_t xbuf_s, uint32_t seg_s, uint32_t stg_s, int lane, int64_t s,
-                                          int nblk, int bin, bool trace = false) {
+                                          int nblk, int bin) {
   const int ncols = bin * A.bucket;
   int64_t* seg = reinterpret_cast<int64_t*>(__cvta_shared_to_generic(seg_s));
   __syncwarp();
@@ -627,9 +621,6 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   dnB = dnA;
   if (2 * lane < nblk) dnA = A.blk[phys(2 * lane)];
   if (2 * lane + 1 < nblk) dnB = A.blk[phys(2 * lane + 1)];
-#ifdef PHMM_DBG_TRACE
-  int tstep = 0;
-#endif
 
   // Ring rescale (FP32 pass, long rows only): when a pair continues from
   // virtual lane 63 of one pass into virtual lane 0 of the next, its ring row (the row
@@ -687,15 +678,6 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     upM = pk(__shfl_sync(0xffffffffu, sM, src), m3a);
     upI = pk(__shfl_sync(0xffffffffu, sI, src), i3a);
     upD = pk(__shfl_sync(0xffffffffu, sD, src), d3a);
-#endif
-#if defined(PHMM_DBG_TRACE) && defined(PHMM_DEFINE_WF)
-    if (sizeof(T) == 4 && trace && tstep < 4096) {
-      float* t = g_trace + ((size_t)tstep * 32 + lane) * 6;
-      t[0] = (float)m3a; t[1] = (float)i3a; t[2] = (float)d3a;
-      t[3] = (float)m3b; t[4] = (float)i3b; t[5] = (float)d3b;
-      if (lane == 0) g_trace_steps = tstep + 1;
-    }
-    ++tstep;
 #endif
     ++c0;
     ++c31B;
@@ -797,8 +779,7 @@ __global__ void __launch_bounds__(WF_WARPS * 32, WfT<T>::MINB) k_wavefront(WfArg
     int64_t s, e;
     wf_item(A, it, lane, bin, s, e);
     if (e <= s) continue;
-    wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, seg_s, stg_s, lane, s, (int)(e - s), bin,
-                        it == A.launch_items[0]);
+    wf_stream<T, kLong>(A, ptab_s, ring_s, xbuf_s, seg_s, stg_s, lane, s, (int)(e - s), bin);
     __syncwarp();
   }
 }
