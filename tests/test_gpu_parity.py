@@ -4,6 +4,7 @@ element on the same seeded inputs (BASELINE.json north_star tolerances):
   * FP32 + rescue path: |d log10| <= 1e-3 absolute
 Every pair the oracle computes is compared; -inf must match -inf.
 """
+import dataclasses
 import math
 
 import numpy as np
@@ -559,3 +560,58 @@ def test_device_call_argument_errors(ctx32):
     rc = ctx32._L.phmm_compute_batch(ctx32._h, ctypes.byref(st), out.ctypes.data_as(phmm._f64p), None)
     assert rc == -1 and np.all(out == 3.0)
     del keep
+
+
+def _shifted(t, k):
+    """The same bytes at an address k bytes past a 256-byte-aligned allocation."""
+    import torch
+
+    buf = torch.empty(t.numel() + 64, dtype=t.dtype, device=t.device)
+    v = buf[k:k + t.numel()]
+    v.copy_(t)
+    return v
+
+
+@pytest.mark.parametrize("shift", [(0, 0), (3, 3), (1, 5), (4, 4)])
+def test_validation_every_alignment_and_position(ctx32, shift):
+    """k_validate reads the five read arrays as 16-byte vectors when they share their
+    alignment mod 16, as 4-byte words when they share it mod 4, else bytes, and the
+    haplotype bases as 16-byte vectors after a scalar head: a bad byte in the head, inside a
+    vector or in the tail, at every alignment class, is reported (PHMM_E_INVALID_BASE /
+    PHMM_E_INVALID_QUAL) and the outputs stay untouched; the clean batch gives the oracle."""
+    import torch
+
+    base = synth.random_pairs_batch(11, 40)
+    nrb, nhb = int(base.read_offsets[-1]), int(base.hap_offsets[-1])
+    ref = oracle.batch_log10(base)
+    rs, qs = shift  # shift of read_bases and of the four quality arrays
+
+    def dev_batch(b):
+        db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+        db.read_bases = _shifted(db.read_bases, rs)
+        for k in ("base_quals", "ins_quals", "del_quals", "gcp_quals"):
+            setattr(db, k, _shifted(getattr(db, k), qs))
+        db.hap_bases = _shifted(db.hap_bases, rs + 1)
+        return db
+
+    got, _ = ctx32.compute_batch_dev(dev_batch(base))
+    _check(got.cpu().numpy(), ref, "fp32")
+    for pos in sorted({0, 1, 5, 15, 16, 17, 31, nrb // 2, nrb - 2, nrb - 1}):
+        for arr, bad, code in (("read_bases", ord("x"), -2), ("del_quals", 200, -3), ("ins_quals", 2, -3)):
+            b = dataclasses.replace(base, **{arr: getattr(base, arr).copy()})
+            getattr(b, arr)[pos] = bad
+            if arr == "ins_quals":  # Q2 insertion with a Q2 deletion: R16 (e(qi) + e(qd) > 1)
+                b.del_quals = b.del_quals.copy()
+                b.del_quals[pos] = 2
+            out = torch.full((b.n_pairs,), 12345.0, dtype=torch.float64, device="cuda:0")
+            st = torch.full((b.n_pairs,), 77, dtype=torch.uint8, device="cuda:0")
+            with pytest.raises(phmm.PhmmError) as ei:
+                ctx32.compute_batch_dev(dev_batch(b), out=out, status=st)
+            assert ei.value.code == code, (arr, pos)
+            assert bool(torch.all(out == 12345.0)) and bool(torch.all(st == 77))
+    for pos in sorted({0, 1, 15, 16, nhb // 2, nhb - 1}):
+        b = dataclasses.replace(base, hap_bases=base.hap_bases.copy())
+        b.hap_bases[pos] = ord("u")
+        with pytest.raises(phmm.PhmmError) as ei:
+            ctx32.compute_batch_dev(dev_batch(b))
+        assert ei.value.code == -2, pos

@@ -40,3 +40,23 @@ for r in rows[hi + 1:]:
 print(f"\n# per-instruction shared wavefronts (ncu source page): actual {tot}, ideal {ideal}, excess {tot - ideal}")
 for x, s in sorted(worst, reverse=True)[:10]:
     print(f"  excess {x:>10}  {s}")
+# by opcode
+from collections import defaultdict
+act, exc = defaultdict(int), defaultdict(int)
+isrc = h.index("Source")
+for r in rows[hi + 1:]:
+    if len(r) != len(h):
+        continue
+    try:
+        w, d = int(r[iw] or 0), int(r[ii] or 0)
+    except ValueError:
+        continue
+    if not w:
+        continue
+    t = r[isrc].strip().split()
+    op = (t[1] if t and t[0].startswith("@") and len(t) > 1 else (t[0] if t else "?")).split(".")[0]
+    act[op] += w
+    exc[op] += w - d
+print("\n# by opcode: actual / excess shared wavefronts")
+for op in sorted(act, key=lambda k: -act[k]):
+    print(f"  {op:8s} {act[op]:>12,} / {exc[op]:>10,}")
