@@ -633,7 +633,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
 #endif
   constexpr bool rescale = kLong && PHMM_RING_RESCALE && sizeof(T) == 4;  // long-row launch: ncols >= WF_RESCALE_COLS
 
-  auto step = [&](const int r) {
+  auto step = [&](const int r, const uint32_t wA, const uint32_t wB) {
     if (is31) rget<ring_packed<T, kLong>()>(ring_s + RS * (uint32_t)(c0 + 2), rvM, rvI, rvD);
     // code byte r (= code*WF_CB) placed in byte 1 -> the code's rows in the table
     // code stride of this pass's table relative to the code byte's (powers of 2)
@@ -688,7 +688,22 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
     wA_nx = wA_nx2; wB_nx = wB_nx2;
     wA_nx2 = __ldg(pA); wB_nx2 = __ldg(pB);
     ++pA; ++pB;
-    step(0); step(1); step(2); step(3);
+    step(0, wA, wB); step(1, wA, wB); step(2, wA, wB); step(3, wA, wB);
+  };
+  // groups g, g+1, g+2 with the code words in three fixed registers: each word is loaded two
+  // groups before the group that uses it and never moved (the rotation of group4 reads every
+  // load one group after issuing it, which waits on it when it misses in L1). Used for the
+  // long segment of a pass by the FP32 long-row kernel only: C4 kernel +5 %, while the
+  // FP32 short-row kernel (-O1) loses 3 % on C2 and the FP64 kernel 1 % with it
+  // (profiles/r02_ab_unroll3.txt).
+  constexpr bool kUnroll3 = kLong && sizeof(T) == 4;
+  auto group12 = [&](uint32_t& a0, uint32_t& a1, uint32_t& a2, uint32_t& b0, uint32_t& b1, uint32_t& b2) {
+    a2 = __ldg(pA); b2 = __ldg(pB); ++pA; ++pB;
+    step(0, a0, b0); step(1, a0, b0); step(2, a0, b0); step(3, a0, b0);
+    a0 = __ldg(pA); b0 = __ldg(pB); ++pA; ++pB;
+    step(0, a1, b1); step(1, a1, b1); step(2, a1, b1); step(3, a1, b1);
+    a1 = __ldg(pA); b1 = __ldg(pB); ++pA; ++pB;
+    step(0, a2, b2); step(1, a2, b2); step(2, a2, b2); step(3, a2, b2);
   };
 
   // Staged switch events: group e switches at pass step 8e (its lanes start column
@@ -728,16 +743,23 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
           wf_commit<1, T>(L, stgB_s, d0);
         }
       }
-      const int ngroups = (e2 < 2 * NGRP - 1) ? 1 : (q < npass ? (P - (2 * NGRP - 1) * 4) / 4 : 0);
+      int ngroups = (e2 < 2 * NGRP - 1) ? 1 : (q < npass ? (P - (2 * NGRP - 1) * 4) / 4 : 0);
+      if constexpr (kUnroll3) {
+        if (ngroups >= 3) {
+          uint32_t a0 = wA_nx, a1 = wA_nx2, a2, b0 = wB_nx, b1 = wB_nx2, b2;
+#pragma unroll 1
+          for (; ngroups >= 3; ngroups -= 3) group12(a0, a1, a2, b0, b1, b2);
+          wA_nx = a0; wA_nx2 = a1; wB_nx = b0; wB_nx2 = b1;
+        }
+      }
 #pragma unroll 1
       for (int k = 0; k < ngroups; ++k) group4();
     }
   }
 }
 
-// The kernels are defined in wf.cu (their own translation unit, compiled with
-// -Xptxas -O1: ptxas -O2/-O3 mis-schedules the FP32 kernel -- results silently differ
-// from the -O0/-O1 builds and from the CPU model of the schedule).
+// The kernels are defined in wf.cu (-Xptxas -O1) and wf_long32.cu (the FP32 long-row
+// kernel, -O3): the optimisation level each is fastest at.
 // phmm_lib.cu reaches them through these host functions.
 // shared memory of one warp: its prior tables and its ring
 template <typename T, bool kLong = false> __host__ __device__ size_t wf_warp_smem(int ring_len) {
