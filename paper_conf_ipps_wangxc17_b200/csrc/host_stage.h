@@ -12,6 +12,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <condition_variable>
 #include <cstdint>
 #include <cstring>
@@ -46,6 +47,7 @@ class CopyPool {
     }
     {
       std::lock_guard<std::mutex> g(m_);
+      fn_ = nullptr;
       dst_ = static_cast<char*>(dst);
       src_ = static_cast<const char*>(src);
       n_ = n;
@@ -57,9 +59,31 @@ class CopyPool {
     std::unique_lock<std::mutex> lk(m_);
     done_cv_.wait(lk, [this] { return pending_ == 0; });
   }
+  // fn(j) for j in [0, njobs), job j on participant j % size() (the caller is participant 0)
+  void for_each(int njobs, const std::function<void(int)>& fn) {
+    if (th_.empty() || njobs <= 1) {
+      for (int j = 0; j < njobs; ++j) fn(j);
+      return;
+    }
+    {
+      std::lock_guard<std::mutex> g(m_);
+      fn_ = &fn;
+      njobs_ = njobs;
+      pending_ = (int)th_.size();
+      ++gen_;
+    }
+    cv_.notify_all();
+    part(0, size());
+    std::unique_lock<std::mutex> lk(m_);
+    done_cv_.wait(lk, [this] { return pending_ == 0; });
+  }
 
  private:
   void part(int k, int parts) {
+    if (fn_) {
+      for (int j = k; j < njobs_; j += parts) (*fn_)(j);
+      return;
+    }
     const size_t per = ((n_ + parts - 1) / parts + 63) & ~(size_t)63;
     const size_t a = std::min(n_, per * (size_t)k), z = std::min(n_, a + per);
     if (z > a) std::memcpy(dst_ + a, src_ + a, z - a);
@@ -89,6 +113,8 @@ class CopyPool {
   char* dst_ = nullptr;
   const char* src_ = nullptr;
   size_t n_ = 0;
+  const std::function<void(int)>* fn_ = nullptr;  // for_each job, else a memcpy_par job
+  int njobs_ = 0;
 };
 
 constexpr int kStageSlots = 4;
@@ -204,6 +230,154 @@ struct Stager {
     }
     return cudaSuccess;
   }
+};
+
+// The host->device side of the pipelined host-buffer call (phmm_lib.cu): a
+// context-owned thread that runs one call's copy jobs in order on a copy stream (through the
+// Stager, so pageable buffers are staged while earlier pieces are in flight) and records an
+// event after each group of jobs. The compute thread waits (on the host) until group k's event
+// is recorded and then makes its stream wait on it, so chunk k computes while the copy engine
+// moves chunk k+1. One call at a time; the caller finishes every call with wait_all().
+struct CopyJob {
+  void* dst;
+  const void* src;
+  size_t n;
+};
+
+class Feeder {
+ public:
+  Feeder() = default;
+  Feeder(const Feeder&) = delete;
+  ~Feeder() { stop(); }
+
+  cudaError_t init(int device) {
+    device_ = device;
+    cudaError_t e = cudaStreamCreateWithFlags(&stream_, cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+      stream_ = nullptr;
+      return e;
+    }
+    th_ = std::thread([this] { run(); });
+    return cudaSuccess;
+  }
+  cudaStream_t stream() const { return stream_; }
+  bool trace = false;
+  std::vector<double> job_us;  // trace: host time of each job's issue
+
+  // Start a call: job groups[k] = jobs [group_end[k-1], group_end[k]), event ev[k] recorded
+  // on the copy stream after group k. The stager belongs to this thread until wait_all().
+  void start(Stager* st, const std::vector<CopyJob>* jobs, const std::vector<size_t>* group_end,
+             const std::vector<cudaEvent_t>* ev) {
+    std::lock_guard<std::mutex> g(m_);
+    st_ = st;
+    jobs_ = jobs;
+    group_end_ = group_end;
+    ev_ = ev;
+    recorded_ = 0;
+    err_ = cudaSuccess;
+    cancel_ = false;
+    busy_ = true;
+    ++gen_;
+    cv_.notify_all();
+  }
+  // Block until group k's event is recorded (or the feeder failed / was cancelled).
+  cudaError_t wait_group(int k) {
+    std::unique_lock<std::mutex> lk(m_);
+    done_cv_.wait(lk, [&] { return recorded_ > k || err_ != cudaSuccess || !busy_; });
+    if (err_ != cudaSuccess) return err_;
+    return recorded_ > k ? cudaSuccess : cudaErrorUnknown;
+  }
+  // Stop issuing further jobs (an error elsewhere in the call).
+  void cancel() {
+    std::lock_guard<std::mutex> g(m_);
+    cancel_ = true;
+  }
+  // Wait until the thread has issued (or dropped) every job of the call and the copy stream
+  // has drained: no copy reads the caller's buffers after this returns.
+  cudaError_t wait_all() {
+    std::unique_lock<std::mutex> lk(m_);
+    done_cv_.wait(lk, [&] { return !busy_; });
+    const cudaError_t e = err_;
+    lk.unlock();
+    const cudaError_t s = stream_ ? cudaStreamSynchronize(stream_) : cudaSuccess;
+    return e != cudaSuccess ? e : s;
+  }
+  void stop() {
+    if (th_.joinable()) {
+      {
+        std::lock_guard<std::mutex> g(m_);
+        quit_ = true;
+      }
+      cv_.notify_all();
+      th_.join();
+    }
+    if (stream_) {
+      cudaStreamSynchronize(stream_);
+      cudaStreamDestroy(stream_);
+      stream_ = nullptr;
+    }
+  }
+
+ private:
+  void run() {
+    uint64_t seen = 0;
+    bool dev_set = false;
+    while (true) {
+      {
+        std::unique_lock<std::mutex> lk(m_);
+        cv_.wait(lk, [&] { return quit_ || gen_ != seen; });
+        if (quit_) return;
+        seen = gen_;
+      }
+      if (!dev_set) {
+        cudaSetDevice(device_);
+        dev_set = true;
+      }
+      cudaError_t e = cudaSuccess;
+      size_t j = 0;
+      for (size_t k = 0; k < group_end_->size() && e == cudaSuccess; ++k) {
+        for (; j < (*group_end_)[k] && e == cudaSuccess; ++j) {
+          {
+            std::lock_guard<std::mutex> g(m_);
+            if (cancel_) break;
+          }
+          const CopyJob& c = (*jobs_)[j];
+          const auto t0 = std::chrono::steady_clock::now();
+          e = st_->h2d(c.dst, c.src, c.n, stream_);
+          if (trace) job_us.push_back(std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() - t0).count());
+        }
+        {
+          std::lock_guard<std::mutex> g(m_);
+          if (cancel_) break;
+        }
+        if (e == cudaSuccess) e = cudaEventRecord((*ev_)[k], stream_);
+        if (e == cudaSuccess) {
+          std::lock_guard<std::mutex> g(m_);
+          recorded_ = (int)k + 1;
+          done_cv_.notify_all();
+        }
+      }
+      if (e != cudaSuccess) cudaGetLastError();
+      std::lock_guard<std::mutex> g(m_);
+      err_ = e;
+      busy_ = false;
+      done_cv_.notify_all();
+    }
+  }
+
+  int device_ = 0;
+  cudaStream_t stream_ = nullptr;
+  std::thread th_;
+  std::mutex m_;
+  std::condition_variable cv_, done_cv_;
+  uint64_t gen_ = 0;
+  bool quit_ = false, cancel_ = false, busy_ = false;
+  int recorded_ = 0;
+  cudaError_t err_ = cudaSuccess;
+  Stager* st_ = nullptr;
+  const std::vector<CopyJob>* jobs_ = nullptr;
+  const std::vector<size_t>* group_end_ = nullptr;
+  const std::vector<cudaEvent_t>* ev_ = nullptr;
 };
 
 }  // namespace phmm

@@ -10,6 +10,7 @@
 #include <cub/device/device_scan.cuh>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -88,6 +89,20 @@ struct PhaseMs {
   float prep, wf, fin, resc;
 };
 
+struct PassInfo {
+  unsigned long long cells = 0, padded_cells = 0, total_blocks = 0;
+  int max_ncols = 0, min_ncols = 0;
+};
+
+
+// one chunk of a pipelined host call (compute_host_pipe)
+struct PipeChunk {
+  int64_t p0, p1;       // pairs [p0, p1)
+  int64_t rlo, rhi;     // read index range the chunk's pairs use
+  int64_t hlo, hhi;     // haplotype index range
+  int64_t rend, hend;   // reads [0, rend) and haplotypes [0, hend) are on the device before it runs
+};
+
 }  // namespace
 
 struct phmm_ctx {
@@ -98,7 +113,10 @@ struct phmm_ctx {
   uint32_t flags = 0;
   int bucket = 4;
   int nsm = 148;
-  Buf buf[B_COUNT];
+  Buf buf[2 * B_COUNT];                  // [set][id]: per-chunk buffers exist once per set (pipelined call)
+  int set = 0;                            // the buffer set the current chunk uses
+  uint32_t* gerr = nullptr;               // pipelined call: the call-wide device error word
+  cudaStream_t stream2 = nullptr;         // pipelined call: the second chunk stream (odd chunks)
   int smem_per_sm = 0, smem_reserved = 0, smem_optin = 0;  // bytes (device attributes)
   Scalars* host_scal = nullptr;  // pinned
   int64_t* host_sizes = nullptr;  // pinned, 2 values
@@ -117,7 +135,22 @@ struct phmm_ctx {
   unsigned long long* host_underflow = nullptr;  // pinned: the call's FP64 underflow count (read at its end)
   bool timing_deferred = false;           // one-chunk call: phase times read after the final sync
   int64_t host_ranges_n = 0;
+  Feeder* feeder = nullptr;               // pipelined host call: the copy thread + copy stream
+  std::vector<cudaEvent_t> pipe_ev;       // ... its per-group events
+  std::vector<CopyJob> pipe_jobs;
+  std::vector<size_t> pipe_groups;
+  std::vector<PipeChunk> pipe_chunks;
+  bool pipe = true;                       // PHMM_PIPE=0: no pipelined host calls
+  bool pipe_trace = false;                // PHMM_PIPE_TRACE=1: per-chunk device timeline on stderr
+  std::vector<cudaEvent_t> trace_ev;      // ... chunk start / end events
+  std::vector<std::pair<const char*, double>> trace_host;  // ... host timestamps (us)
+  std::chrono::steady_clock::time_point trace_t0;
 };
+static void trace_mark(phmm_ctx* c, const char* what) {
+  if (c->pipe_trace)
+    c->trace_host.emplace_back(what, std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now() -
+                                                                               c->trace_t0).count());
+}
 
 namespace {
 
@@ -156,7 +189,11 @@ template <class X>
 phmm_status ws(phmm_ctx* c, int id, size_t count, X** out) {
   size_t bytes = count * sizeof(X);
   if (bytes < 16) bytes = 16;
-  Buf& b = c->buf[id];
+  // inputs, outputs and the call-wide lists are one per context; every per-chunk buffer has
+  // one copy per set, so that two chunks can be in flight on two streams (compute_host_pipe)
+  const bool shared = id <= B_PAIRS || id == B_OUT_LOG10 || id == B_OUT_STATUS || id == B_RLIST ||
+                      id == B_UNDERFLOW || (id >= B_SW_REF && id <= B_SW_NOPOFF);
+  Buf& b = c->buf[id + (shared ? 0 : c->set * B_COUNT)];
   if (b.n < bytes) {
     if (b.p) cudaFree(b.p);
     b.p = nullptr;
@@ -217,10 +254,6 @@ struct DevBatch {
   int64_t n_reads, n_haps, n_pairs, n_rb, n_hb;
 };
 
-struct PassInfo {
-  unsigned long long cells = 0, padded_cells = 0, total_blocks = 0;
-  int max_ncols = 0, min_ncols = 0;
-};
 
 // Validation of the whole batch. Errors land in scal->err (read back by pass_prepare).
 phmm_status run_validate(phmm_ctx* c, const DevBatch& d) {
@@ -271,6 +304,7 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   int32_t *pair_bin, *pair_nb;
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
   ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
+  trace_mark(c, "prep start");
   CUDA_TRY(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * 3 * nb1, s));
   // per-pass scalars (err is kept: it accumulates validation errors)
   CUDA_TRY(cudaMemsetAsync(&scal->max_ncols, 0, offsetof(Scalars, n_rescue) - offsetof(Scalars, max_ncols), s));
@@ -280,7 +314,7 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   k_pair_bins<K><<<pb_grid, kThreads, 0, s>>>(
       d.pairs, list, nullptr, n, d.roff, d.n_reads, d.hoff, d.n_haps, c->bucket, pair_bin, pair_nb, bins,
       bins + nb1, &scal->max_ncols, &scal->min_ncols_c, &scal->cells, &scal->padded_cells, &scal->total_blocks,
-      &scal->err);
+      c->gerr ? c->gerr : &scal->err);
   LAUNCHED(c);
 
   // table items and their block offsets (exclusive scan over n_items + 1)
@@ -343,11 +377,14 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   }
   // one small D2H: sizes + error flag
   CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+  if (c->gerr) CUDA_TRY(cudaMemcpyAsync(&c->host_scal->err, c->gerr, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   int64_t* hsz = c->host_sizes;
   hsz[0] = hsz[1] = 0;
   CUDA_TRY(cudaMemcpyAsync(&hsz[0], item_off + n_items, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   if (hc_off) CUDA_TRY(cudaMemcpyAsync(&hsz[1], hc_off + d.n_haps, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  trace_mark(c, "prep sync");
   CUDA_TRY(cudaStreamSynchronize(s));
+  trace_mark(c, "prep synced");
   if (c->host_scal->err) return map_err(c->host_scal->err);
   if (total_hcodes_out) *total_hcodes_out = hsz[1];
   pi->cells = c->host_scal->cells;
@@ -893,6 +930,312 @@ void finish_stats(phmm_ctx* c) {
   }
 }
 
+// ---- pipelined host-buffer call (DESIGN.md §1 "Host buffers")
+// A host batch of kPipeMinPairs .. chunk_pairs pairs whose pairs use reads and haplotypes in
+// ascending index ranges (GATK order: region after region) runs as chunks of pairs of growing
+// size (n/F, n/F, 2n/F, 4n/F, ...; F = kPipeFirstDiv): the copy thread (Feeder) moves chunk
+// k's new input bytes to the device on a copy stream while chunk k-1 computes, so only the
+// first chunk's copy is exposed. Consecutive chunks alternate between two streams and two
+// buffer sets, so that chunk k's preparation kernels and wavefront start as soon as chunk
+// k-1's wavefront drains. Every chunk is an ordinary batch over the reads /
+// haplotypes it uses (the chunked device call's rebasing, R14: a pair's arithmetic does not
+// depend on its batch), validated as its bytes arrive; the FP32 chunks append their
+// underflowing pairs to one list and ONE FP64 rescue pass over the whole batch follows, so the
+// call has one host round trip per chunk plus two. Results are bitwise those of the one-pass call.
+constexpr int64_t kPipeMinPairs = 1ll << 17;
+constexpr int kPipeFirstDiv = 8;
+
+
+// Chunk plan from the host pair list (index ranges by a parallel scan). PHMM_E_INDEX for an
+// out-of-range index; *useful = false when the first chunk would need most of the inputs.
+phmm_status pipe_plan(phmm_ctx* c, const phmm_batch* b, std::vector<PipeChunk>& ch, bool* useful) {
+  const int64_t n = b->n_pairs;
+  int div = kPipeFirstDiv;
+  if (const char* e = std::getenv("PHMM_PIPE_FIRST")) div = std::max(2, std::min(1024, std::atoi(e)));
+  ch.clear();
+  const int64_t first = std::max<int64_t>(1, n / div);
+  for (int64_t p = 0, sz = first, k = 0; p < n; ++k) {
+    const int64_t e = (n - (p + sz) < first) ? n : p + sz;  // no runt chunk at the end
+    ch.push_back(PipeChunk{p, e, 0, 0, 0, 0, 0, 0});
+    p = e;
+    if (k >= 1) sz *= 2;
+  }
+  const int nch = (int)ch.size();
+  const int parts = c->stage.pool->size();
+  std::vector<int64_t> mm((size_t)nch * parts * 4);
+  std::vector<uint8_t> bad((size_t)nch * parts, 0);
+  const int32_t* pr = b->pairs;
+  const int64_t nr = b->n_reads, nh = b->n_haps;
+  c->stage.pool->for_each(nch * parts, [&](int j) {
+    const PipeChunk& k = ch[(size_t)(j / parts)];
+    const int64_t len = k.p1 - k.p0, per = (len + parts - 1) / parts;
+    const int64_t a = k.p0 + std::min(len, per * (j % parts)), z = std::min(k.p1, a + per);
+    int32_t rmin = INT32_MAX, rmax = -1, hmin = INT32_MAX, hmax = -1;
+    for (int64_t p = a; p < z; ++p) {
+      const int32_t r = pr[2 * p], h = pr[2 * p + 1];
+      rmin = std::min(rmin, r); rmax = std::max(rmax, r);
+      hmin = std::min(hmin, h); hmax = std::max(hmax, h);
+    }
+    if (z > a && (rmin < 0 || rmax >= nr || hmin < 0 || hmax >= nh)) bad[(size_t)j] = 1;
+    int64_t* o = &mm[(size_t)j * 4];
+    o[0] = rmin; o[1] = rmax; o[2] = hmin; o[3] = hmax;
+  });
+  for (size_t j = 0; j < bad.size(); ++j)
+    if (bad[j]) return PHMM_E_INDEX;
+  int64_t rend = 0, hend = 0;
+  for (int k = 0; k < nch; ++k) {
+    PipeChunk& x = ch[(size_t)k];
+    x.rlo = x.hlo = INT64_MAX;
+    x.rhi = x.hhi = -1;
+    for (int t = 0; t < parts; ++t) {
+      const int64_t* o = &mm[((size_t)k * parts + t) * 4];
+      if (o[1] < 0) continue;  // empty part
+      x.rlo = std::min(x.rlo, o[0]); x.rhi = std::max(x.rhi, o[1]);
+      x.hlo = std::min(x.hlo, o[2]); x.hhi = std::max(x.hhi, o[3]);
+    }
+    rend = std::max(rend, x.rhi + 1);
+    hend = std::max(hend, x.hhi + 1);
+    x.rend = (k == nch - 1) ? nr : rend;  // the last chunk brings every remaining byte (all validated)
+    x.hend = (k == nch - 1) ? nh : hend;
+  }
+  // the copies follow the host offsets: they must be in range and ascending over the chunks
+  // (else the one-pass call runs and its device validation reports the batch)
+  int64_t pr_ = 0, ph_ = 0;
+  for (const PipeChunk& x : ch) {
+    const int64_t r1 = b->read_offsets[x.rend], h1 = b->hap_offsets[x.hend];
+    if (r1 < pr_ || r1 > b->total_read_bases || h1 < ph_ || h1 > b->total_hap_bases) {
+      *useful = false;
+      return PHMM_OK;
+    }
+    pr_ = r1;
+    ph_ = h1;
+  }
+  const int64_t rb = b->read_offsets[ch[0].rend], hb = b->hap_offsets[ch[0].hend];
+  *useful = nch > 1 && 2 * (rb * 5 + hb) < b->total_read_bases * 5 + b->total_hap_bases;
+  return PHMM_OK;
+}
+
+phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vector<PipeChunk>& ch,
+                              double* out_log10, uint8_t* out_status) {
+  cudaStream_t s = c->stream;
+  const int nch = (int)ch.size();
+  if (!c->feeder) {
+    c->feeder = new (std::nothrow) Feeder();
+    if (!c->feeder) return PHMM_E_OOM;
+    if (c->feeder->init(c->device) != cudaSuccess) {
+      cudaGetLastError();
+      delete c->feeder;
+      c->feeder = nullptr;
+      return PHMM_E_CUDA;
+    }
+  }
+  while ((int)c->pipe_ev.size() < nch + 4) {
+    cudaEvent_t e;
+    CUDA_TRY(cudaEventCreate(&e));  // timed: PHMM_PIPE_TRACE reads the copy timeline
+    c->pipe_ev.push_back(e);
+  }
+  while (c->pipe_trace && (int)c->trace_ev.size() < 2 * nch) {
+    cudaEvent_t e;
+    CUDA_TRY(cudaEventCreate(&e));
+    c->trace_ev.push_back(e);
+  }
+  Feeder& F = *c->feeder;
+  const cudaStream_t cs = F.stream();
+  uint8_t *rb, *q, *qi, *qd, *qg, *hap;
+  int64_t *roff, *hoff;
+  int32_t* pairs;
+  double* out;
+  uint8_t* status = nullptr;
+  const size_t nr = (size_t)b->total_read_bases, nh = (size_t)b->total_hap_bases;
+  ST_TRY(ws(c, B_READ_BASES, nr, &rb));
+  ST_TRY(ws(c, B_BQ, nr, &q));
+  ST_TRY(ws(c, B_IQ, nr, &qi));
+  ST_TRY(ws(c, B_DQ, nr, &qd));
+  ST_TRY(ws(c, B_GQ, nr, &qg));
+  ST_TRY(ws(c, B_HAP, nh, &hap));
+  ST_TRY(ws(c, B_ROFF, (size_t)b->n_reads + 1, &roff));
+  ST_TRY(ws(c, B_HOFF, (size_t)b->n_haps + 1, &hoff));
+  ST_TRY(ws(c, B_PAIRS, (size_t)b->n_pairs * 2, &pairs));
+  ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
+  if (out_status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
+  int32_t* rlist = nullptr;
+  if (c->prec == PHMM_PREC_FP32_RESCUE) ST_TRY(ws(c, B_RLIST, (size_t)b->n_pairs, &rlist));
+  Scalars *scal, *scal1;
+  unsigned long long* uf;
+  ST_TRY(ws(c, B_SCAL, 1, &scal));
+  ST_TRY(ws(c, B_UNDERFLOW, 1, &uf));
+  c->set = 1;
+  const phmm_status s1 = ws(c, B_SCAL, 1, &scal1);
+  c->set = 0;
+  ST_TRY(s1);
+  // odd chunks run on a second stream with the second buffer set, so that chunk k + 1's
+  // preparation and wavefront start while chunk k's wavefront drains
+  if (!c->stream2) CUDA_TRY(cudaStreamCreateWithFlags(&c->stream2, cudaStreamNonBlocking));
+  const cudaStream_t sk[2] = {s, c->stream2};
+  // copy jobs: group 0 = the offsets, group k + 1 = chunk k's pairs and its new input bytes
+  std::vector<CopyJob>& J = c->pipe_jobs;
+  std::vector<size_t>& G = c->pipe_groups;
+  J.clear();
+  G.clear();
+  J.push_back(CopyJob{roff, b->read_offsets, sizeof(int64_t) * (size_t)(b->n_reads + 1)});
+  J.push_back(CopyJob{hoff, b->hap_offsets, sizeof(int64_t) * (size_t)(b->n_haps + 1)});
+  G.push_back(J.size());
+  int64_t r0 = 0, h0 = 0;
+  for (const PipeChunk& k : ch) {
+    J.push_back(CopyJob{pairs + 2 * k.p0, b->pairs + 2 * k.p0, sizeof(int32_t) * 2 * (size_t)(k.p1 - k.p0)});
+    const int64_t r1 = b->read_offsets[k.rend], h1 = b->hap_offsets[k.hend];
+    if (h1 > h0) J.push_back(CopyJob{hap + h0, b->hap_bases + h0, (size_t)(h1 - h0)});
+    if (r1 > r0) {
+      J.push_back(CopyJob{rb + r0, b->read_bases + r0, (size_t)(r1 - r0)});
+      J.push_back(CopyJob{q + r0, b->base_quals + r0, (size_t)(r1 - r0)});
+      J.push_back(CopyJob{qi + r0, b->ins_quals + r0, (size_t)(r1 - r0)});
+      J.push_back(CopyJob{qd + r0, b->del_quals + r0, (size_t)(r1 - r0)});
+      J.push_back(CopyJob{qg + r0, b->gcp_quals + r0, (size_t)(r1 - r0)});
+    }
+    G.push_back(J.size());
+    r0 = std::max(r0, r1);
+    h0 = std::max(h0, h1);
+  }
+  Stager& S = c->stage;
+  S.staged_bytes = 0;
+  c->st = phmm_stats{};
+  c->acc = PhaseMs{};
+  c->st.n_pairs = b->n_pairs;
+  c->timing_deferred = true;  // no per-chunk phase events (finish_stats overrides them)
+  ev_record(c, EV_START);
+  // the copies start after whatever the compute stream ran before the call
+  CUDA_TRY(cudaEventRecord(c->pipe_ev[nch + 1], s));
+  CUDA_TRY(cudaStreamWaitEvent(cs, c->pipe_ev[nch + 1], 0));
+  F.trace = c->pipe_trace;
+  F.job_us.clear();
+  c->trace_host.clear();
+  c->trace_t0 = std::chrono::steady_clock::now();
+  F.start(&S, &J, &G, &c->pipe_ev);
+  // every exit from here on stops the feeder and drains the copy stream first
+  auto run = [&]() -> phmm_status {
+    CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
+    CUDA_TRY(cudaMemsetAsync(scal1, 0, sizeof(Scalars), s));
+    CUDA_TRY(cudaMemsetAsync(uf, 0, sizeof(unsigned long long), s));
+    CUDA_TRY(cudaEventRecord(c->pipe_ev[nch + 2], s));
+    CUDA_TRY(cudaStreamWaitEvent(sk[1], c->pipe_ev[nch + 2], 0));
+    c->gerr = &scal->err;  // validation and binning errors of every chunk
+    CUDA_TRY(F.wait_group(0));
+    CUDA_TRY(cudaStreamWaitEvent(s, c->pipe_ev[0], 0));
+    k_validate_offsets<<<grid_for(c, b->n_reads + 1), kThreads, 0, s>>>(roff, b->n_reads, (int64_t)nr, c->gerr);
+    LAUNCHED(c);
+    k_validate_offsets<<<grid_for(c, b->n_haps + 1), kThreads, 0, s>>>(hoff, b->n_haps, (int64_t)nh, c->gerr);
+    LAUNCHED(c);
+    int64_t vr = 0, vh = 0;  // bytes validated so far
+    for (int i = 0; i < nch; ++i) {
+      const PipeChunk& k = ch[(size_t)i];
+      const cudaStream_t si = sk[i & 1];
+      c->set = i & 1;
+      c->stream = si;
+      trace_mark(c, "wait_group");
+      CUDA_TRY(F.wait_group(i + 1));
+      trace_mark(c, "group ready");
+      CUDA_TRY(cudaStreamWaitEvent(si, c->pipe_ev[i + 1], 0));
+      if (c->pipe_trace) CUDA_TRY(cudaEventRecord(c->trace_ev[2 * i], si));
+      const int64_t r1 = b->read_offsets[k.rend], h1 = b->hap_offsets[k.hend];
+      if (r1 > vr || h1 > vh) {
+        const int64_t nrb = std::max<int64_t>(0, r1 - vr), nhb = std::max<int64_t>(0, h1 - vh);
+        k_validate<<<grid_for(c, std::max(nhb, nrb / 4)), kThreads, 0, si>>>(
+            hap + vh, nhb, rb + vr, q + vr, qi + vr, qd + vr, qg + vr, nrb, nullptr, -1, nullptr, -1, c->gerr);
+        LAUNCHED(c);
+        vr = std::max(vr, r1);
+        vh = std::max(vh, h1);
+      }
+      const int64_t np = k.p1 - k.p0, nrk = k.rhi + 1 - k.rlo, nhk = k.hhi + 1 - k.hlo;
+      int64_t *roff_c, *hoff_c;
+      int32_t* pairs_c;
+      ST_TRY(ws(c, B_CH_ROFF, (size_t)nrk + 1, &roff_c));
+      ST_TRY(ws(c, B_CH_HOFF, (size_t)nhk + 1, &hoff_c));
+      ST_TRY(ws(c, B_CH_PAIRS, (size_t)2 * np, &pairs_c));
+      k_rebase_chunk<<<grid_for(c, std::max(std::max(nrk, nhk) + 1, np)), kThreads, 0, si>>>(
+          roff, k.rlo, nrk, roff_c, hoff, k.hlo, nhk, hoff_c, pairs, k.p0, np, pairs_c, 0);
+      LAUNCHED(c);
+      trace_mark(c, "rebased");
+      DevBatch dk{rb, q, qi, qd, qg, hap, roff_c, hoff_c, pairs_c, nrk, nhk, np, (int64_t)nr, (int64_t)nh};
+      double* o = out + k.p0;
+      uint8_t* st = status ? status + k.p0 : nullptr;
+      if (c->prec == PHMM_PREC_FP64) {
+        ST_TRY(compute_one(c, dk, o, st));
+      } else {
+        PassInfo pi;
+        uint8_t* hc = nullptr;
+        int64_t total_hc = 0;
+        ST_TRY(fp32_pass(c, dk, o, st, rlist, k.p0, &scal->n_rescue, &pi, &hc, &total_hc, false));
+        ++c->st.n_chunks;
+      }
+      if (c->pipe_trace) CUDA_TRY(cudaEventRecord(c->trace_ev[2 * i + 1], si));
+      trace_mark(c, "chunk issued");
+    }
+    c->set = 0;
+    c->stream = s;
+    c->gerr = nullptr;
+    CUDA_TRY(cudaEventRecord(c->pipe_ev[nch + 3], sk[1]));
+    CUDA_TRY(cudaStreamWaitEvent(s, c->pipe_ev[nch + 3], 0));
+    const DevBatch d{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs,
+                     (int64_t)nr, (int64_t)nh};
+    if (c->prec == PHMM_PREC_FP32_RESCUE) {
+      CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+      CUDA_TRY(cudaStreamSynchronize(s));
+      if (c->host_scal->err) return map_err(c->host_scal->err);
+      const int64_t n_resc = c->host_scal->n_rescue;
+      c->st.n_rescued += n_resc;
+      if (n_resc > 0) ST_TRY(rescue_pass(c, d, out, status, rlist, n_resc, nullptr, 0, false));
+    }
+    return PHMM_OK;
+  };
+  phmm_status st = run();
+  c->set = 0;
+  c->stream = s;
+  c->gerr = nullptr;
+  if (st != PHMM_OK) F.cancel();
+  const cudaError_t fe = F.wait_all();
+  if (st == PHMM_OK && fe != cudaSuccess) st = PHMM_E_CUDA;
+  if (st != PHMM_OK) {
+    cudaStreamSynchronize(sk[1]);
+    cudaStreamSynchronize(s);
+    cudaGetLastError();
+    return st;
+  }
+  ST_TRY(enqueue_underflow_readback(c));
+  ev_record(c, EV_D2H);
+  {
+    Nvtx nv("phmm:d2h");
+    CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s));
+    if (out_status) CUDA_TRY(S.d2h(out_status, status, b->n_pairs, s));
+  }
+  ev_record(c, EV_END);
+  CUDA_TRY(cudaStreamSynchronize(s));
+  finish_stats(c);
+  if (c->pipe_trace) {
+    auto t = [&](cudaEvent_t e) {
+      float ms = -1.f;
+      if (cudaEventElapsedTime(&ms, c->ev[EV_START], e) != cudaSuccess) cudaGetLastError();
+      return ms;
+    };
+    std::fprintf(stderr, "phmm pipe: %d chunks, offsets copied %.3f ms\n", nch, t(c->pipe_ev[0]));
+    for (int i = 0; i < nch; ++i)
+      std::fprintf(stderr, "  chunk %d pairs [%lld, %lld): copied %.3f, compute %.3f .. %.3f ms\n", i,
+                   (long long)ch[(size_t)i].p0, (long long)ch[(size_t)i].p1, t(c->pipe_ev[i + 1]),
+                   t(c->trace_ev[2 * i]), t(c->trace_ev[2 * i + 1]));
+    std::fprintf(stderr, "  rescue + d2h from %.3f, end %.3f ms\n", t(c->trace_ev[2 * nch - 1]), t(c->ev[EV_END]));
+    std::fprintf(stderr, "  host:");
+    for (auto& h : c->trace_host) std::fprintf(stderr, " %s %.0f,", h.first, h.second);
+    std::fprintf(stderr, "\n");
+    std::fprintf(stderr, "  copy issue (host us):");
+    for (size_t j = 0; j < F.job_us.size(); ++j) std::fprintf(stderr, " %zu:%.0f/%zuB", j, F.job_us[j], J[j].n);
+    std::fprintf(stderr, "\n");
+  }
+  // per-phase times are not split out in a pipelined call (chunks overlap the copies)
+  c->st.ms_h2d = c->st.ms_prep = c->st.ms_wavefront = c->st.ms_rescue = c->st.ms_finalize = -1.f;
+  c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
+  c->st.staged_bytes = S.staged_bytes;
+  return PHMM_OK;
+}
+
 phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status) {
   ST_TRY(check_batch_args(b));
   if (b->n_pairs > 0 && !out_log10) return PHMM_E_INVALID_ARG;
@@ -908,6 +1251,16 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
   // host-side size checks that need the host offsets
   if (b->read_offsets[b->n_reads] != b->total_read_bases || b->hap_offsets[b->n_haps] != b->total_hap_bases)
     return PHMM_E_INVALID_ARG;
+  if (b->n_pairs >= kPipeMinPairs && b->n_pairs <= c->chunk_pairs && c->pipe) {
+    std::vector<PipeChunk>& ch = c->pipe_chunks;
+    bool useful = false;
+    const auto t0 = std::chrono::steady_clock::now();
+    ST_TRY(pipe_plan(c, b, ch, &useful));
+    if (c->pipe_trace)
+      std::fprintf(stderr, "phmm pipe: plan %.3f ms (host)\n",
+                   std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    if (useful) return compute_host_pipe(c, b, ch, out_log10, out_status);
+  }
   cudaStream_t s = c->stream;
   uint8_t *rb, *q, *qi, *qd, *qg, *hap;
   int64_t *roff, *hoff;
@@ -1240,6 +1593,8 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
       return fail(PHMM_E_OOM);
     }
   }
+  if (const char* e = std::getenv("PHMM_PIPE")) c->pipe = std::atoi(e) != 0;
+  if (const char* e = std::getenv("PHMM_PIPE_TRACE")) c->pipe_trace = std::atoi(e) != 0;
   if (const char* e = std::getenv("PHMM_CHUNK_PAIRS")) c->chunk_pairs = std::max<int64_t>(64, std::atoll(e));
   *out = c;
   return PHMM_OK;
@@ -1252,8 +1607,20 @@ void phmm_destroy(phmm_ctx* c) {
   if (c->stream) cudaStreamSynchronize(c->stream);
   for (int i = 0; i < B_COUNT; ++i)
     if (c->buf[i].p) cudaFree(c->buf[i].p);
+  for (int i = 0; i < B_COUNT; ++i)
+    if (c->buf[B_COUNT + i].p) cudaFree(c->buf[B_COUNT + i].p);
+  if (c->stream2) {
+    cudaStreamSynchronize(c->stream2);
+    cudaStreamDestroy(c->stream2);
+  }
   for (int i = 0; i < kEvents; ++i)
     if (c->ev[i]) cudaEventDestroy(c->ev[i]);
+  delete c->feeder;  // joins the copy thread, drains its stream
+  c->feeder = nullptr;
+  for (cudaEvent_t e : c->pipe_ev) cudaEventDestroy(e);
+  c->pipe_ev.clear();
+  for (cudaEvent_t e : c->trace_ev) cudaEventDestroy(e);
+  c->trace_ev.clear();
   c->stage.release();
   if (c->host_scal) cudaFreeHost(c->host_scal);
   if (c->host_sizes) cudaFreeHost(c->host_sizes);

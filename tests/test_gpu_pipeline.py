@@ -134,3 +134,76 @@ def test_submit_queue_coalesces_regions_bitwise():
             tickets[0].wait()
     finally:
         ctx.close()
+
+
+@pytest.mark.parametrize("prec", ["fp32", "fp64"])
+def test_pipelined_host_call_is_bitwise_the_one_pass_call(prec):
+    """A host batch of 2^17 .. 2^23 pairs in region order runs pipelined (compute_host_pipe):
+    chunks of n/8, n/8, n/4, n/2 pairs, alternating between two streams and two buffer sets, whose input bytes reach the
+    device on a copy stream while the previous chunk computes; one FP64 rescue over the whole
+    batch at the end. Results and statuses must equal the device call and the unpipelined host
+    call (PHMM_PIPE=0) bit for bit, pageable and page-locked; staged_bytes counts every input
+    byte once; an invalid base or an out-of-range pair index in the LAST chunk fails the call
+    with the outputs untouched; a batch whose first chunk uses the last read is not pipelined."""
+    import torch
+
+    b = synth.concat_batches([synth.config_batch("C2", n_regions=1536), synth.config_batch("C3", n_regions=128)])
+    n = b.n_pairs
+    assert n >= 1 << 17
+    ctx = phmm.PairHMM(precision=prec)
+    os.environ["PHMM_PIPE"] = "0"
+    try:
+        flat = phmm.PairHMM(precision=prec)
+    finally:
+        del os.environ["PHMM_PIPE"]
+    try:
+        db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+        dev, dst = ctx.compute_batch_dev(db)
+        torch.cuda.synchronize()
+        dev, dst = dev.cpu().numpy(), dst.cpu().numpy()
+        got, st = ctx.compute_batch(b)
+        stats = ctx.stats()
+        assert stats["n_chunks"] == 4, stats
+        assert stats["staged_bytes"] == b.nbytes_inputs() + 9 * n
+        assert stats["cells"] == b.cells()
+        assert np.array_equal(got, dev) and np.array_equal(st, dst)
+        got0, st0 = flat.compute_batch(b)
+        assert flat.stats()["n_chunks"] == 1
+        assert np.array_equal(got0, dev) and np.array_equal(st0, dst)
+        if prec == "fp32":
+            assert stats["n_rescued"] == flat.stats()["n_rescued"] > 0
+        pin = {k: torch.from_numpy(np.ascontiguousarray(getattr(b, k))).pin_memory().numpy()
+               for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets",
+                         "hap_bases", "hap_offsets", "pairs")}
+        out = torch.empty(n, dtype=torch.float64).pin_memory().numpy()
+        sto = torch.empty(n, dtype=torch.uint8).pin_memory().numpy()
+        got2, st2 = ctx.compute_batch(synth.Batch(**pin), out=out, status=sto)
+        assert np.array_equal(got2, dev) and np.array_equal(st2, dst)
+        assert ctx.stats()["staged_bytes"] == 0 and ctx.stats()["n_chunks"] == 4
+        # errors in the last chunk's bytes / pairs: outputs untouched
+        bad = b.subset(np.arange(n))
+        bad.read_bases = bad.read_bases.copy()
+        bad.read_bases[-3] = ord("x")
+        o = np.full(n, 3.0)
+        with pytest.raises(phmm.PhmmError) as ei:
+            ctx.compute_batch(bad, out=o)
+        assert ei.value.code == -2 and np.all(o == 3.0)
+        bad = b.subset(np.arange(n))
+        bad.pairs[-1, 1] = b.n_haps
+        with pytest.raises(phmm.PhmmError) as ei:
+            ctx.compute_batch(bad, out=o)
+        assert ei.value.code == -5 and np.all(o == 3.0)
+        # the context is still usable after the errors
+        got3, _ = ctx.compute_batch(b)
+        assert np.array_equal(got3, dev)
+        # first chunk touching the last read: one pass
+        perm = np.arange(n)
+        last = int(np.nonzero(b.pairs[:, 0] == b.n_reads - 1)[0][0])
+        perm[[0, last]] = perm[[last, 0]]
+        sw = b.subset(perm)
+        got4, _ = ctx.compute_batch(sw)
+        assert ctx.stats()["n_chunks"] == 1
+        assert np.array_equal(got4, dev[perm])
+    finally:
+        ctx.close()
+        flat.close()

@@ -1,0 +1,5 @@
+python -m pytest tests -m gpu -q -x > gpurun_out/s8_gpu_tests.log 2>&1; tail -2 gpurun_out/s8_gpu_tests.log
+python bench.py --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/s8_bench.json 2>gpurun_out/s8_bench.err
+python -c "
+import json;d=json.loads(open('gpurun_out/s8_bench.json').read().strip().splitlines()[-1]);e=d['e2e'];print(round(d['value']),round(d['ms_per_step'],3),'e2e',round(e['value']),round(e['ms_per_step'],3),'pageable',round(e['pageable']['value']),round(e['pageable']['ms_per_step'],3), round(e['pageable_over_pinned'],3))"
+python tools/pipe_probe.py C2 > gpurun_out/s8_probe.txt 2>&1; grep '^{' gpurun_out/s8_probe.txt
