@@ -115,6 +115,19 @@ __global__ void k_validate(const uint8_t* __restrict__ hap, int64_t n_hb, const 
   if (e && (threadIdx.x & 31) == 0) atomicOr(err, e);
 }
 
+// Byte fill of device scratch as a kernel: a cudaMemsetAsync is queued behind the host->device
+// copies of the pipelined host call (measured: a 0.5 MB memset waited 150 us on another
+// stream's copy), a kernel is not. 16-byte stores from the first 16-byte boundary on.
+__global__ void k_fill_bytes(uint8_t* __restrict__ p, uint32_t v4, int64_t n) {
+  const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x, nthr = (int64_t)gridDim.x * blockDim.x;
+  const int64_t head = min(n, (int64_t)((16 - ((uintptr_t)p & 15)) & 15));
+  for (int64_t i = tid; i < head; i += nthr) p[i] = (uint8_t)v4;
+  const int64_t nv = (n - head) >> 4;
+  uint4* q = reinterpret_cast<uint4*>(p + head);
+  for (int64_t i = tid; i < nv; i += nthr) q[i] = make_uint4(v4, v4, v4, v4);
+  for (int64_t i = head + 16 * nv + tid; i < n; i += nthr) p[i] = (uint8_t)v4;
+}
+
 // Offsets (the Smith-Waterman batch): start at 0, non-decreasing, end at total.
 __global__ void k_validate_offsets(const int64_t* __restrict__ off, int64_t n, int64_t total, uint32_t* err) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= n; i += (int64_t)gridDim.x * blockDim.x)
@@ -327,6 +340,12 @@ __global__ void k_rebase_chunk(const int64_t* __restrict__ roff, int64_t rlo, in
       pairs_c[2 * i + 1] = pairs[2 * (p0 + i) + 1] - (int32_t)hlo;
     }
   }
+}
+
+// rng[4k .. 4k+3] = (UINT_MAX, 0, UINT_MAX, 0) for k < n: the identities of k_chunk_ranges
+__global__ void k_ranges_init(uint32_t* __restrict__ rng, int64_t n) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < 4 * n; i += (int64_t)gridDim.x * blockDim.x)
+    rng[i] = (i & 1) ? 0u : 0xffffffffu;
 }
 
 // Index ranges of the chunks of a chunked device call: chunk blockIdx.y = pairs

@@ -140,6 +140,7 @@ struct phmm_ctx {
   std::vector<CopyJob> pipe_jobs;
   std::vector<size_t> pipe_groups;
   std::vector<PipeChunk> pipe_chunks;
+  std::vector<cudaEvent_t> pipe_gev;      // ... the events of the copy groups of one call
   bool pipe = true;                       // PHMM_PIPE=0: no pipelined host calls
   bool pipe_trace = false;                // PHMM_PIPE_TRACE=1: per-chunk device timeline on stderr
   std::vector<cudaEvent_t> trace_ev;      // ... chunk start / end events
@@ -222,6 +223,18 @@ int grid_for(const phmm_ctx* c, int64_t n) {
   return (int)g;
 }
 
+// cudaMemsetAsync replacement (k_fill_bytes): value v in every byte of [p, p + n)
+cudaError_t fill_async(phmm_ctx* c, void* p, int v, size_t n, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  const uint32_t b = (uint32_t)(v & 0xff);
+  const int64_t work = (int64_t)(n / 16) + 1;
+  int g = (int)std::min<int64_t>((work + kThreads - 1) / kThreads, (int64_t)c->nsm * 4);
+  if (g < 1) g = 1;
+  k_fill_bytes<<<g, kThreads, 0, s>>>(static_cast<uint8_t*>(p), b * 0x01010101u, (int64_t)n);
+  ++c->launches;
+  return cudaGetLastError();
+}
+
 phmm_status map_err(uint32_t e) {
   if (e & ERR_INDEX) return PHMM_E_INDEX;
   if (e & ERR_ARG) return PHMM_E_INVALID_ARG;
@@ -261,7 +274,7 @@ phmm_status run_validate(phmm_ctx* c, const DevBatch& d) {
   cudaStream_t s = c->stream;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
-  CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
+  CUDA_TRY(fill_async(c, scal, 0, sizeof(Scalars), s));
   const int64_t work = std::max(std::max(d.n_hb, d.n_rb / 4), std::max(d.n_reads, d.n_haps) + 1);
   k_validate<<<grid_for(c, work), kThreads, 0, s>>>(d.hap, d.n_hb, d.rb, d.q, d.qi, d.qd, d.qg, d.n_rb, d.roff,
                                                     d.n_reads, d.hoff, d.n_haps, &scal->err);
@@ -305,9 +318,9 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   ST_TRY(ws(c, B_PAIR_BIN, (size_t)n, &pair_bin));
   ST_TRY(ws(c, B_PAIR_NB, (size_t)n, &pair_nb));
   trace_mark(c, "prep start");
-  CUDA_TRY(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * 3 * nb1, s));
+  CUDA_TRY(fill_async(c, bins, 0, sizeof(unsigned long long) * 3 * nb1, s));
   // per-pass scalars (err is kept: it accumulates validation errors)
-  CUDA_TRY(cudaMemsetAsync(&scal->max_ncols, 0, offsetof(Scalars, n_rescue) - offsetof(Scalars, max_ncols), s));
+  CUDA_TRY(fill_async(c, &scal->max_ncols, 0, offsetof(Scalars, n_rescue) - offsetof(Scalars, max_ncols), s));
 
   const int pb_grid = (int)std::max<int64_t>(grid_for(c, (n + kPairBinsU - 1) / kPairBinsU),
                                               (n + kPairBinsPerCta - 1) / kPairBinsPerCta);
@@ -408,7 +421,7 @@ phmm_status build_hap_codes(phmm_ctx* c, const DevBatch& d, int64_t total_hc, in
   uint8_t* hc;
   ST_TRY(ws(c, B_HC_OFF, (size_t)d.n_haps + 1, &hc_off));
   ST_TRY(ws(c, B_HCODES, (size_t)(total_hc + pad_len), &hc));
-  CUDA_TRY(cudaMemsetAsync(hc + total_hc, WF_PAD * WF_CB, (size_t)pad_len, s));
+  CUDA_TRY(fill_async(c, hc + total_hc, WF_PAD * WF_CB, (size_t)pad_len, s));
   k_hap_codes_wf<<<grid_for(c, d.n_haps * 32), kThreads, 0, s>>>(d.hap, d.hoff, d.n_haps, hc_off, c->bucket, hc);
   LAUNCHED(c);
   *hc_out = hc;
@@ -552,7 +565,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   A.lpt = WF_LPT;
   A.out = out;
   A.exp_out = exp_out;
-  CUDA_TRY(cudaMemsetAsync(scal->item_counter, 0, sizeof(scal->item_counter), s));
+  CUDA_TRY(fill_async(c, scal->item_counter, 0, sizeof(scal->item_counter), s));
   if (timed) ev_record(c, EV_WF0);
   for (int i = 0; i < nl; ++i) {
     A.bin_lo = L[i].bin_lo;
@@ -582,7 +595,7 @@ phmm_status fp32_pass(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t* 
   ST_TRY(ws(c, B_OUT32, (size_t)d.n_pairs, &out32));
   int32_t* exp32;  // powers of 2 applied by the ring rescale of long pairs
   ST_TRY(ws(c, B_EXP32, (size_t)d.n_pairs, &exp32));
-  CUDA_TRY(cudaMemsetAsync(exp32, 0, sizeof(int32_t) * (size_t)d.n_pairs, s));
+  CUDA_TRY(fill_async(c, exp32, 0, sizeof(int32_t) * (size_t)d.n_pairs, s));
   if (timed) ev_record(c, EV_PREP);
   ST_TRY(pass_run<float>(c, d, nullptr, d.n_pairs, *pi, total_tab, *hc, *total_hc, out32, timed, exp32));
   k_finalize_fp32<<<grid_for(c, d.n_pairs), kThreads, 0, s>>>(out32, exp32, d.n_pairs, d.pairs, d.hoff, c->bucket,
@@ -676,7 +689,7 @@ phmm_status compute_one(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   } else {
     int32_t* rlist;
     ST_TRY(ws(c, B_RLIST, (size_t)d.n_pairs, &rlist));
-    CUDA_TRY(cudaMemsetAsync(&scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
+    CUDA_TRY(fill_async(c, &scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
     ST_TRY(fp32_pass(c, d, dev_out, dev_status, rlist, 0, &scal->n_rescue, &pi, &hc, &total_hc, true));
     ev_record(c, EV_RESC0);
     CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
@@ -707,7 +720,7 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   ST_TRY(run_validate(c, d));
   unsigned long long* uf;
   ST_TRY(ws(c, B_UNDERFLOW, 1, &uf));
-  CUDA_TRY(cudaMemsetAsync(uf, 0, sizeof(unsigned long long), s));
+  CUDA_TRY(fill_async(c, uf, 0, sizeof(unsigned long long), s));
   const int64_t cp = c->chunk_pairs;
   // one chunk: the phase times and the underflow count are read after the call's final sync
   c->timing_deferred = d.n_pairs <= cp;
@@ -718,10 +731,10 @@ phmm_status compute_dev(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
   uint32_t* rng;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   ST_TRY(ws(c, B_CH_RANGES, (size_t)4 * nch, &rng));
-  CUDA_TRY(cudaMemsetAsync(rng, 0, sizeof(uint32_t) * 4 * nch, s));
+  CUDA_TRY(fill_async(c, rng, 0, sizeof(uint32_t) * 4 * nch, s));
   for (int64_t k = 0; k < nch; ++k) {  // minima start at UINT_MAX
-    CUDA_TRY(cudaMemsetAsync(rng + 4 * k, 0xff, sizeof(uint32_t), s));
-    CUDA_TRY(cudaMemsetAsync(rng + 4 * k + 2, 0xff, sizeof(uint32_t), s));
+    CUDA_TRY(fill_async(c, rng + 4 * k, 0xff, sizeof(uint32_t), s));
+    CUDA_TRY(fill_async(c, rng + 4 * k + 2, 0xff, sizeof(uint32_t), s));
   }
   {
     const int bpc = (int)std::max<int64_t>(1, std::min<int64_t>((cp + kThreads - 1) / kThreads, 4 * c->nsm));
@@ -800,7 +813,7 @@ phmm_status sw_compute_dev(phmm_ctx* c, const SwDev& d, const phmm_sw_params* pr
   if (d.n_tasks == 0) return PHMM_OK;
   Scalars* scal;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
-  CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
+  CUDA_TRY(fill_async(c, scal, 0, sizeof(Scalars), s));
   if (d.n_rb > 0) {
     k_validate_haps<<<grid_for(c, d.n_rb), kThreads, 0, s>>>(d.ref, d.n_rb, &scal->err);
     LAUNCHED(c);
@@ -865,7 +878,7 @@ phmm_status sw_compute_dev(phmm_ctx* c, const SwDev& d, const phmm_sw_params* pr
   int bps = 0;
   CUDA_TRY(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_sw_fill, SW_WARPS * 32, smem));
   if (bps < 1) return PHMM_E_INVALID_ARG;
-  CUDA_TRY(cudaMemsetAsync(A.counter, 0, sizeof(unsigned int), s));
+  CUDA_TRY(fill_async(c, A.counter, 0, sizeof(unsigned int), s));
   ev_record(c, EV_WF0);
   k_sw_fill<<<(unsigned)(c->nsm * bps), SW_WARPS * 32, smem, s>>>(A);
   LAUNCHED(c);
@@ -943,82 +956,98 @@ void finish_stats(phmm_ctx* c) {
 // underflowing pairs to one list and ONE FP64 rescue pass over the whole batch follows, so the
 // call has one host round trip per chunk plus two. Results are bitwise those of the one-pass call.
 constexpr int64_t kPipeMinPairs = 1ll << 17;
-constexpr int kPipeFirstDiv = 8;
+// chunk plans (measured on C2, profiles/r02_pipe_sweep.txt): page-locked inputs n/8 + 7n/8 (the
+// copy engine keeps up with the compute); pageable ones n/4, n/4, n/2 (the staging memcpy is the
+// slower side, so more and smaller chunks overlap it better)
+constexpr int kPipeFirstDivPinned = 8, kPipeMaxChPinned = 2;
+constexpr int kPipeFirstDivPageable = 4, kPipeMaxChPageable = 64;
 
 
-// Chunk plan from the host pair list (index ranges by a parallel scan). PHMM_E_INDEX for an
-// out-of-range index; *useful = false when the first chunk would need most of the inputs.
-phmm_status pipe_plan(phmm_ctx* c, const phmm_batch* b, std::vector<PipeChunk>& ch, bool* useful) {
-  const int64_t n = b->n_pairs;
-  int div = kPipeFirstDiv;
+// Chunk boundaries of a pipelined call: sub-chunks of n/F pairs, chunk k = 1, 1, 2, 4, ...
+// sub-chunks (the last one takes the rest, at most maxch chunks). Index ranges per sub-chunk:
+// a page-locked pair list is NOT read on the host -- a CPU pass over a page-locked buffer right
+// before its DMA slows that copy up to 10x on the GPU hosts (lines held in CPU caches,
+// tools/h2d_probe4.py) -- so the device computes them (k_chunk_ranges) after the pair list
+// arrived; a pageable pair list (which is staged through the context's slots anyway) is
+// scanned by the copy pool (pipe_scan), so the copies start at once.
+void pipe_chunks(int64_t n, bool pinned, std::vector<PipeChunk>& ch, int64_t* sub) {
+  int div = pinned ? kPipeFirstDivPinned : kPipeFirstDivPageable;
   if (const char* e = std::getenv("PHMM_PIPE_FIRST")) div = std::max(2, std::min(1024, std::atoi(e)));
+  int maxch = pinned ? kPipeMaxChPinned : kPipeMaxChPageable;
+  if (const char* e = std::getenv("PHMM_PIPE_MAXCH")) maxch = std::max(2, std::atoi(e));
+  *sub = std::max<int64_t>(1, n / div);
   ch.clear();
-  const int64_t first = std::max<int64_t>(1, n / div);
-  for (int64_t p = 0, sz = first, k = 0; p < n; ++k) {
-    const int64_t e = (n - (p + sz) < first) ? n : p + sz;  // no runt chunk at the end
+  for (int64_t p = 0, sz = *sub, k = 0; p < n; ++k) {
+    // no runt chunk at the end; at most maxch chunks
+    const int64_t e = (n - (p + sz) < *sub || k + 1 >= maxch) ? n : p + sz;
     ch.push_back(PipeChunk{p, e, 0, 0, 0, 0, 0, 0});
     p = e;
     if (k >= 1) sz *= 2;
   }
-  const int nch = (int)ch.size();
-  const int parts = c->stage.pool->size();
-  std::vector<int64_t> mm((size_t)nch * parts * 4);
-  std::vector<uint8_t> bad((size_t)nch * parts, 0);
+}
+
+// Host scan of a pageable pair list: rng[4t..4t+3] = min/max read index, min/max haplotype
+// index of sub-chunk t (k_chunk_ranges' layout). PHMM_E_INDEX for an index out of range.
+phmm_status pipe_scan(phmm_ctx* c, const phmm_batch* b, int64_t sub, int64_t nsub, uint32_t* rng) {
+  std::vector<uint8_t> bad((size_t)nsub, 0);
   const int32_t* pr = b->pairs;
   const int64_t nr = b->n_reads, nh = b->n_haps;
-  c->stage.pool->for_each(nch * parts, [&](int j) {
-    const PipeChunk& k = ch[(size_t)(j / parts)];
-    const int64_t len = k.p1 - k.p0, per = (len + parts - 1) / parts;
-    const int64_t a = k.p0 + std::min(len, per * (j % parts)), z = std::min(k.p1, a + per);
-    int32_t rmin = INT32_MAX, rmax = -1, hmin = INT32_MAX, hmax = -1;
+  c->stage.pool->for_each((int)nsub, [&](int t) {
+    const int64_t a = (int64_t)t * sub, z = std::min(b->n_pairs, a + sub);
+    int64_t rmin = INT64_MAX, rmax = -1, hmin = INT64_MAX, hmax = -1;
     for (int64_t p = a; p < z; ++p) {
-      const int32_t r = pr[2 * p], h = pr[2 * p + 1];
+      const int64_t r = pr[2 * p], h = pr[2 * p + 1];
       rmin = std::min(rmin, r); rmax = std::max(rmax, r);
       hmin = std::min(hmin, h); hmax = std::max(hmax, h);
     }
-    if (z > a && (rmin < 0 || rmax >= nr || hmin < 0 || hmax >= nh)) bad[(size_t)j] = 1;
-    int64_t* o = &mm[(size_t)j * 4];
-    o[0] = rmin; o[1] = rmax; o[2] = hmin; o[3] = hmax;
+    if (z > a && (rmin < 0 || rmax >= nr || hmin < 0 || hmax >= nh)) bad[(size_t)t] = 1;
+    uint32_t* g = rng + 4 * t;
+    g[0] = z > a ? (uint32_t)rmin : 0xffffffffu; g[1] = z > a ? (uint32_t)rmax : 0u;
+    g[2] = z > a ? (uint32_t)hmin : 0xffffffffu; g[3] = z > a ? (uint32_t)hmax : 0u;
   });
-  for (size_t j = 0; j < bad.size(); ++j)
-    if (bad[j]) return PHMM_E_INDEX;
+  for (uint8_t x : bad)
+    if (x) return PHMM_E_INDEX;
+  return PHMM_OK;
+}
+
+// Index ranges of the chunks from the sub-chunk ranges rng (k_chunk_ranges, validated
+// indices) and the byte ranges each chunk brings. *useful = false (run as one chunk) when the
+// first chunk would need more than half of the input bytes or the host offsets are not
+// ascending over the chunks (the device validation then reports the batch).
+void pipe_ranges(const phmm_batch* b, std::vector<PipeChunk>& ch, int64_t sub, const uint32_t* rng, bool* useful) {
+  const int nch = (int)ch.size();
   int64_t rend = 0, hend = 0;
   for (int k = 0; k < nch; ++k) {
     PipeChunk& x = ch[(size_t)k];
     x.rlo = x.hlo = INT64_MAX;
     x.rhi = x.hhi = -1;
-    for (int t = 0; t < parts; ++t) {
-      const int64_t* o = &mm[((size_t)k * parts + t) * 4];
-      if (o[1] < 0) continue;  // empty part
-      x.rlo = std::min(x.rlo, o[0]); x.rhi = std::max(x.rhi, o[1]);
-      x.hlo = std::min(x.hlo, o[2]); x.hhi = std::max(x.hhi, o[3]);
+    for (int64_t t = x.p0 / sub; t * sub < x.p1; ++t) {
+      const uint32_t* g = rng + 4 * t;
+      if (g[0] == 0xffffffffu) continue;  // empty sub-chunk
+      x.rlo = std::min<int64_t>(x.rlo, g[0]); x.rhi = std::max<int64_t>(x.rhi, g[1]);
+      x.hlo = std::min<int64_t>(x.hlo, g[2]); x.hhi = std::max<int64_t>(x.hhi, g[3]);
     }
     rend = std::max(rend, x.rhi + 1);
     hend = std::max(hend, x.hhi + 1);
-    x.rend = (k == nch - 1) ? nr : rend;  // the last chunk brings every remaining byte (all validated)
-    x.hend = (k == nch - 1) ? nh : hend;
+    x.rend = (k == nch - 1) ? b->n_reads : rend;  // the last chunk brings every remaining byte (all validated)
+    x.hend = (k == nch - 1) ? b->n_haps : hend;
   }
-  // the copies follow the host offsets: they must be in range and ascending over the chunks
-  // (else the one-pass call runs and its device validation reports the batch)
   int64_t pr_ = 0, ph_ = 0;
   for (const PipeChunk& x : ch) {
     const int64_t r1 = b->read_offsets[x.rend], h1 = b->hap_offsets[x.hend];
     if (r1 < pr_ || r1 > b->total_read_bases || h1 < ph_ || h1 > b->total_hap_bases) {
       *useful = false;
-      return PHMM_OK;
+      return;
     }
     pr_ = r1;
     ph_ = h1;
   }
   const int64_t rb = b->read_offsets[ch[0].rend], hb = b->hap_offsets[ch[0].hend];
   *useful = nch > 1 && 2 * (rb * 5 + hb) < b->total_read_bases * 5 + b->total_hap_bases;
-  return PHMM_OK;
 }
 
-phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vector<PipeChunk>& ch,
-                              double* out_log10, uint8_t* out_status) {
+phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status) {
   cudaStream_t s = c->stream;
-  const int nch = (int)ch.size();
   if (!c->feeder) {
     c->feeder = new (std::nothrow) Feeder();
     if (!c->feeder) return PHMM_E_OOM;
@@ -1029,15 +1058,32 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
       return PHMM_E_CUDA;
     }
   }
-  while ((int)c->pipe_ev.size() < nch + 4) {
+  std::vector<PipeChunk>& ch = c->pipe_chunks;
+  int64_t sub = 0;
+  const bool pinned = Stager::is_pinned(b->read_bases) && Stager::is_pinned(b->pairs);
+  pipe_chunks(b->n_pairs, pinned, ch, &sub);
+  const int64_t nsub = (b->n_pairs + sub - 1) / sub;
+  const int nmax = (int)ch.size();
+  while ((int)c->pipe_ev.size() < nmax + 4) {
     cudaEvent_t e;
     CUDA_TRY(cudaEventCreate(&e));  // timed: PHMM_PIPE_TRACE reads the copy timeline
     c->pipe_ev.push_back(e);
   }
-  while (c->pipe_trace && (int)c->trace_ev.size() < 2 * nch) {
+  while (c->pipe_trace && (int)c->trace_ev.size() < 2 * nmax) {
     cudaEvent_t e;
     CUDA_TRY(cudaEventCreate(&e));
     c->trace_ev.push_back(e);
+  }
+  if (c->host_ranges_n < nsub) {
+    if (c->host_ranges) cudaFreeHost(c->host_ranges);
+    c->host_ranges = nullptr;
+    c->host_ranges_n = 0;
+    if (cudaMallocHost(&c->host_ranges, sizeof(uint32_t) * 4 * nsub) != cudaSuccess) {
+      cudaGetLastError();
+      c->host_ranges = nullptr;
+      return PHMM_E_OOM;
+    }
+    c->host_ranges_n = nsub;
   }
   Feeder& F = *c->feeder;
   const cudaStream_t cs = F.stream();
@@ -1062,8 +1108,10 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
   if (c->prec == PHMM_PREC_FP32_RESCUE) ST_TRY(ws(c, B_RLIST, (size_t)b->n_pairs, &rlist));
   Scalars *scal, *scal1;
   unsigned long long* uf;
+  uint32_t* rng;
   ST_TRY(ws(c, B_SCAL, 1, &scal));
   ST_TRY(ws(c, B_UNDERFLOW, 1, &uf));
+  ST_TRY(ws(c, B_CH_RANGES, (size_t)4 * nsub, &rng));
   c->set = 1;
   const phmm_status s1 = ws(c, B_SCAL, 1, &scal1);
   c->set = 0;
@@ -1072,59 +1120,104 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
   // preparation and wavefront start while chunk k's wavefront drains
   if (!c->stream2) CUDA_TRY(cudaStreamCreateWithFlags(&c->stream2, cudaStreamNonBlocking));
   const cudaStream_t sk[2] = {s, c->stream2};
-  // copy jobs: group 0 = the offsets, group k + 1 = chunk k's pairs and its new input bytes
-  std::vector<CopyJob>& J = c->pipe_jobs;
-  std::vector<size_t>& G = c->pipe_groups;
-  J.clear();
-  G.clear();
-  J.push_back(CopyJob{roff, b->read_offsets, sizeof(int64_t) * (size_t)(b->n_reads + 1)});
-  J.push_back(CopyJob{hoff, b->hap_offsets, sizeof(int64_t) * (size_t)(b->n_haps + 1)});
-  G.push_back(J.size());
-  int64_t r0 = 0, h0 = 0;
-  for (const PipeChunk& k : ch) {
-    J.push_back(CopyJob{pairs + 2 * k.p0, b->pairs + 2 * k.p0, sizeof(int32_t) * 2 * (size_t)(k.p1 - k.p0)});
-    const int64_t r1 = b->read_offsets[k.rend], h1 = b->hap_offsets[k.hend];
-    if (h1 > h0) J.push_back(CopyJob{hap + h0, b->hap_bases + h0, (size_t)(h1 - h0)});
-    if (r1 > r0) {
-      J.push_back(CopyJob{rb + r0, b->read_bases + r0, (size_t)(r1 - r0)});
-      J.push_back(CopyJob{q + r0, b->base_quals + r0, (size_t)(r1 - r0)});
-      J.push_back(CopyJob{qi + r0, b->ins_quals + r0, (size_t)(r1 - r0)});
-      J.push_back(CopyJob{qd + r0, b->del_quals + r0, (size_t)(r1 - r0)});
-      J.push_back(CopyJob{qg + r0, b->gcp_quals + r0, (size_t)(r1 - r0)});
-    }
-    G.push_back(J.size());
-    r0 = std::max(r0, r1);
-    h0 = std::max(h0, h1);
-  }
   Stager& S = c->stage;
   S.staged_bytes = 0;
   c->st = phmm_stats{};
   c->acc = PhaseMs{};
   c->st.n_pairs = b->n_pairs;
   c->timing_deferred = true;  // no per-chunk phase events (finish_stats overrides them)
-  ev_record(c, EV_START);
-  // the copies start after whatever the compute stream ran before the call
-  CUDA_TRY(cudaEventRecord(c->pipe_ev[nch + 1], s));
-  CUDA_TRY(cudaStreamWaitEvent(cs, c->pipe_ev[nch + 1], 0));
-  F.trace = c->pipe_trace;
-  F.job_us.clear();
   c->trace_host.clear();
   c->trace_t0 = std::chrono::steady_clock::now();
-  F.start(&S, &J, &G, &c->pipe_ev);
-  // every exit from here on stops the feeder and drains the copy stream first
+  ev_record(c, EV_START);
+  cudaEvent_t ev_start = c->pipe_ev[nmax + 1], ev_s1 = c->pipe_ev[nmax + 2], ev_s1_end = c->pipe_ev[nmax + 3];
+  cudaEvent_t ev_pre = c->pipe_ev[0];
+  int nch = nmax;
+  bool fed = false;
+  // every exit from here on drains the copy stream (and stops the feeder) first
   auto run = [&]() -> phmm_status {
-    CUDA_TRY(cudaMemsetAsync(scal, 0, sizeof(Scalars), s));
-    CUDA_TRY(cudaMemsetAsync(scal1, 0, sizeof(Scalars), s));
-    CUDA_TRY(cudaMemsetAsync(uf, 0, sizeof(unsigned long long), s));
-    CUDA_TRY(cudaEventRecord(c->pipe_ev[nch + 2], s));
-    CUDA_TRY(cudaStreamWaitEvent(sk[1], c->pipe_ev[nch + 2], 0));
+    // the copies start after whatever the compute stream ran before the call
+    CUDA_TRY(cudaEventRecord(ev_start, s));
+    CUDA_TRY(cudaStreamWaitEvent(cs, ev_start, 0));
+    CUDA_TRY(fill_async(c, scal, 0, sizeof(Scalars), s));
+    CUDA_TRY(fill_async(c, scal1, 0, sizeof(Scalars), s));
+    CUDA_TRY(fill_async(c, uf, 0, sizeof(unsigned long long), s));
     c->gerr = &scal->err;  // validation and binning errors of every chunk
-    CUDA_TRY(F.wait_group(0));
-    CUDA_TRY(cudaStreamWaitEvent(s, c->pipe_ev[0], 0));
+    if (pinned) {
+      // step 1: offsets and pair list (this thread), the sub-chunks' index ranges on the device
+      CUDA_TRY(S.h2d(roff, b->read_offsets, sizeof(int64_t) * (size_t)(b->n_reads + 1), cs));
+      CUDA_TRY(S.h2d(hoff, b->hap_offsets, sizeof(int64_t) * (size_t)(b->n_haps + 1), cs));
+      CUDA_TRY(S.h2d(pairs, b->pairs, sizeof(int32_t) * 2 * (size_t)b->n_pairs, cs));
+      CUDA_TRY(cudaEventRecord(ev_pre, cs));
+      k_ranges_init<<<grid_for(c, 4 * nsub), kThreads, 0, s>>>(rng, nsub);
+      LAUNCHED(c);
+      CUDA_TRY(cudaStreamWaitEvent(s, ev_pre, 0));
+      const int bpc = (int)std::max<int64_t>(1, std::min<int64_t>((sub + kThreads - 1) / kThreads, 2 * c->nsm / nsub + 1));
+      k_chunk_ranges<<<dim3((unsigned)bpc, (unsigned)nsub), kThreads, 0, s>>>(pairs, b->n_pairs, sub, b->n_reads,
+                                                                                 b->n_haps, rng, c->gerr);
+      LAUNCHED(c);
+      CUDA_TRY(cudaMemcpyAsync(c->host_ranges, rng, sizeof(uint32_t) * 4 * (size_t)nsub, cudaMemcpyDeviceToHost, s));
+      CUDA_TRY(cudaMemcpyAsync(&c->host_scal->err, c->gerr, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+      CUDA_TRY(cudaStreamSynchronize(s));
+      trace_mark(c, "ranges");
+      if (c->host_scal->err) return map_err(c->host_scal->err);  // index errors: nothing computed
+    } else {
+      ST_TRY(pipe_scan(c, b, sub, nsub, c->host_ranges));
+      trace_mark(c, "ranges");
+    }
+    bool useful = false;
+    pipe_ranges(b, ch, sub, c->host_ranges, &useful);
+    if (!useful) {  // one chunk over the whole batch
+      ch.assign(1, PipeChunk{0, b->n_pairs, 0, b->n_reads - 1, 0, b->n_haps - 1, b->n_reads, b->n_haps});
+      if (b->n_reads == 0 || b->n_haps == 0) return PHMM_E_INDEX;  // cannot happen: ranges validated
+    }
+    nch = (int)ch.size();
+    // step 2: chunk k's new input bytes, one event per chunk, by the copy thread
+    std::vector<CopyJob>& J = c->pipe_jobs;
+    std::vector<size_t>& G = c->pipe_groups;
+    std::vector<cudaEvent_t>& E = c->pipe_gev;
+    J.clear();
+    G.clear();
+    E.clear();
+    const int g0 = pinned ? 0 : 1;  // pageable: the copy thread also stages offsets + pair list first
+    if (!pinned) {
+      J.push_back(CopyJob{roff, b->read_offsets, sizeof(int64_t) * (size_t)(b->n_reads + 1)});
+      J.push_back(CopyJob{hoff, b->hap_offsets, sizeof(int64_t) * (size_t)(b->n_haps + 1)});
+      J.push_back(CopyJob{pairs, b->pairs, sizeof(int32_t) * 2 * (size_t)b->n_pairs});
+      G.push_back(J.size());
+      E.push_back(ev_pre);
+    }
+    int64_t r0 = 0, h0 = 0;
+    for (int i = 0; i < nch; ++i) {
+      const PipeChunk& k = ch[(size_t)i];
+      const int64_t r1 = b->read_offsets[k.rend], h1 = b->hap_offsets[k.hend];
+      if (h1 > h0) J.push_back(CopyJob{hap + h0, b->hap_bases + h0, (size_t)(h1 - h0)});
+      if (r1 > r0) {
+        J.push_back(CopyJob{rb + r0, b->read_bases + r0, (size_t)(r1 - r0)});
+        J.push_back(CopyJob{q + r0, b->base_quals + r0, (size_t)(r1 - r0)});
+        J.push_back(CopyJob{qi + r0, b->ins_quals + r0, (size_t)(r1 - r0)});
+        J.push_back(CopyJob{qd + r0, b->del_quals + r0, (size_t)(r1 - r0)});
+        J.push_back(CopyJob{qg + r0, b->gcp_quals + r0, (size_t)(r1 - r0)});
+      }
+      G.push_back(J.size());
+      E.push_back(c->pipe_ev[i + 1]);
+      r0 = std::max(r0, r1);
+      h0 = std::max(h0, h1);
+    }
+    F.trace = c->pipe_trace;
+    F.job_us.clear();
+    F.start(&S, &J, &G, &E);
+    fed = true;
+    // the offsets' validation (once they are on the device)
+    if (!pinned) {
+      CUDA_TRY(F.wait_group(0));
+      CUDA_TRY(cudaStreamWaitEvent(s, ev_pre, 0));
+    }
     k_validate_offsets<<<grid_for(c, b->n_reads + 1), kThreads, 0, s>>>(roff, b->n_reads, (int64_t)nr, c->gerr);
     LAUNCHED(c);
     k_validate_offsets<<<grid_for(c, b->n_haps + 1), kThreads, 0, s>>>(hoff, b->n_haps, (int64_t)nh, c->gerr);
     LAUNCHED(c);
+    CUDA_TRY(cudaEventRecord(ev_s1, s));
+    CUDA_TRY(cudaStreamWaitEvent(sk[1], ev_s1, 0));
     int64_t vr = 0, vh = 0;  // bytes validated so far
     for (int i = 0; i < nch; ++i) {
       const PipeChunk& k = ch[(size_t)i];
@@ -1132,7 +1225,7 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
       c->set = i & 1;
       c->stream = si;
       trace_mark(c, "wait_group");
-      CUDA_TRY(F.wait_group(i + 1));
+      CUDA_TRY(F.wait_group(i + g0));
       trace_mark(c, "group ready");
       CUDA_TRY(cudaStreamWaitEvent(si, c->pipe_ev[i + 1], 0));
       if (c->pipe_trace) CUDA_TRY(cudaEventRecord(c->trace_ev[2 * i], si));
@@ -1173,14 +1266,15 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
     c->set = 0;
     c->stream = s;
     c->gerr = nullptr;
-    CUDA_TRY(cudaEventRecord(c->pipe_ev[nch + 3], sk[1]));
-    CUDA_TRY(cudaStreamWaitEvent(s, c->pipe_ev[nch + 3], 0));
+    CUDA_TRY(cudaEventRecord(ev_s1_end, sk[1]));
+    CUDA_TRY(cudaStreamWaitEvent(s, ev_s1_end, 0));
     const DevBatch d{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs,
                      (int64_t)nr, (int64_t)nh};
+    // the call's errors (validation of every chunk's bytes, binning), then the FP64 rescue
+    CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    if (c->host_scal->err) return map_err(c->host_scal->err);
     if (c->prec == PHMM_PREC_FP32_RESCUE) {
-      CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
-      CUDA_TRY(cudaStreamSynchronize(s));
-      if (c->host_scal->err) return map_err(c->host_scal->err);
       const int64_t n_resc = c->host_scal->n_rescue;
       c->st.n_rescued += n_resc;
       if (n_resc > 0) ST_TRY(rescue_pass(c, d, out, status, rlist, n_resc, nullptr, 0, false));
@@ -1191,8 +1285,8 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
   c->set = 0;
   c->stream = s;
   c->gerr = nullptr;
-  if (st != PHMM_OK) F.cancel();
-  const cudaError_t fe = F.wait_all();
+  if (st != PHMM_OK && fed) F.cancel();
+  const cudaError_t fe = fed ? F.wait_all() : cudaStreamSynchronize(cs);
   if (st == PHMM_OK && fe != cudaSuccess) st = PHMM_E_CUDA;
   if (st != PHMM_OK) {
     cudaStreamSynchronize(sk[1]);
@@ -1216,7 +1310,7 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
       if (cudaEventElapsedTime(&ms, c->ev[EV_START], e) != cudaSuccess) cudaGetLastError();
       return ms;
     };
-    std::fprintf(stderr, "phmm pipe: %d chunks, offsets copied %.3f ms\n", nch, t(c->pipe_ev[0]));
+    std::fprintf(stderr, "phmm pipe: %d chunks, offsets + pairs copied %.3f ms\n", nch, t(ev_pre));
     for (int i = 0; i < nch; ++i)
       std::fprintf(stderr, "  chunk %d pairs [%lld, %lld): copied %.3f, compute %.3f .. %.3f ms\n", i,
                    (long long)ch[(size_t)i].p0, (long long)ch[(size_t)i].p1, t(c->pipe_ev[i + 1]),
@@ -1224,9 +1318,6 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, const std::vecto
     std::fprintf(stderr, "  rescue + d2h from %.3f, end %.3f ms\n", t(c->trace_ev[2 * nch - 1]), t(c->ev[EV_END]));
     std::fprintf(stderr, "  host:");
     for (auto& h : c->trace_host) std::fprintf(stderr, " %s %.0f,", h.first, h.second);
-    std::fprintf(stderr, "\n");
-    std::fprintf(stderr, "  copy issue (host us):");
-    for (size_t j = 0; j < F.job_us.size(); ++j) std::fprintf(stderr, " %zu:%.0f/%zuB", j, F.job_us[j], J[j].n);
     std::fprintf(stderr, "\n");
   }
   // per-phase times are not split out in a pipelined call (chunks overlap the copies)
@@ -1251,16 +1342,8 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
   // host-side size checks that need the host offsets
   if (b->read_offsets[b->n_reads] != b->total_read_bases || b->hap_offsets[b->n_haps] != b->total_hap_bases)
     return PHMM_E_INVALID_ARG;
-  if (b->n_pairs >= kPipeMinPairs && b->n_pairs <= c->chunk_pairs && c->pipe) {
-    std::vector<PipeChunk>& ch = c->pipe_chunks;
-    bool useful = false;
-    const auto t0 = std::chrono::steady_clock::now();
-    ST_TRY(pipe_plan(c, b, ch, &useful));
-    if (c->pipe_trace)
-      std::fprintf(stderr, "phmm pipe: plan %.3f ms (host)\n",
-                   std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
-    if (useful) return compute_host_pipe(c, b, ch, out_log10, out_status);
-  }
+  if (b->n_pairs >= kPipeMinPairs && b->n_pairs <= c->chunk_pairs && c->pipe)
+    return compute_host_pipe(c, b, out_log10, out_status);
   cudaStream_t s = c->stream;
   uint8_t *rb, *q, *qi, *qd, *qg, *hap;
   int64_t *roff, *hoff;
