@@ -15,13 +15,35 @@
 #include <chrono>
 #include <condition_variable>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
 #include <mutex>
 #include <thread>
 #include <vector>
 
+#include <emmintrin.h>  // SSE2 streaming stores (x86-64 baseline)
+
 namespace phmm {
+
+// memcpy into a page-locked staging slot with non-temporal (streaming) stores, so that the
+// slot's lines are not left in CPU caches: the GPU's DMA read of lines a CPU core holds runs at
+// 5-20 GB/s instead of ~50 on the GPU hosts (tools/h2d_probe4.py). dst must be 16-byte aligned.
+inline void memcpy_stream(char* dst, const char* src, size_t n) {
+  size_t i = 0;
+  for (; i + 64 <= n; i += 64) {
+    const __m128i a = _mm_loadu_si128(reinterpret_cast<const __m128i*>(src + i));
+    const __m128i b = _mm_loadu_si128(reinterpret_cast<const __m128i*>(src + i + 16));
+    const __m128i c = _mm_loadu_si128(reinterpret_cast<const __m128i*>(src + i + 32));
+    const __m128i d = _mm_loadu_si128(reinterpret_cast<const __m128i*>(src + i + 48));
+    _mm_stream_si128(reinterpret_cast<__m128i*>(dst + i), a);
+    _mm_stream_si128(reinterpret_cast<__m128i*>(dst + i + 16), b);
+    _mm_stream_si128(reinterpret_cast<__m128i*>(dst + i + 32), c);
+    _mm_stream_si128(reinterpret_cast<__m128i*>(dst + i + 48), d);
+  }
+  if (i < n) std::memcpy(dst + i, src + i, n - i);
+  _mm_sfence();
+}
 
 // A fixed pool of host threads for parallel memcpy (one job at a time, split evenly).
 class CopyPool {
@@ -38,11 +60,12 @@ class CopyPool {
     for (auto& t : th_) t.join();
   }
   int size() const { return (int)th_.size() + 1; }
-  // dst[0..n) = src[0..n), split over the pool's threads and the caller's
+  bool stream_stores = true;  // PHMM_STAGE_NT=0: plain memcpy into the staging slots
+  // dst[0..n) = src[0..n), split over the pool's threads and the caller's (64-byte aligned parts)
   void memcpy_par(void* dst, const void* src, size_t n) {
     const int parts = size();
     if (n < (size_t)1 << 20 || parts == 1) {
-      std::memcpy(dst, src, n);
+      cpy(static_cast<char*>(dst), static_cast<const char*>(src), n);
       return;
     }
     {
@@ -86,7 +109,11 @@ class CopyPool {
     }
     const size_t per = ((n_ + parts - 1) / parts + 63) & ~(size_t)63;
     const size_t a = std::min(n_, per * (size_t)k), z = std::min(n_, a + per);
-    if (z > a) std::memcpy(dst_ + a, src_ + a, z - a);
+    if (z > a) cpy(dst_ + a, src_ + a, z - a);
+  }
+  void cpy(char* d, const char* s, size_t n) const {
+    if (stream_stores && ((uintptr_t)d & 15) == 0) memcpy_stream(d, s, n);
+    else std::memcpy(d, s, n);
   }
   void run(int i) {
     uint64_t seen = 0;
@@ -142,6 +169,7 @@ struct Stager {
       }
     }
     pool = new CopyPool(std::max(0, threads - 1));
+    if (const char* e = std::getenv("PHMM_STAGE_NT")) pool->stream_stores = std::atoi(e) != 0;
     return cudaSuccess;
   }
   void release() {
