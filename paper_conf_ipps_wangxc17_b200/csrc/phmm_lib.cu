@@ -142,6 +142,7 @@ struct phmm_ctx {
   std::vector<PipeChunk> pipe_chunks;
   std::vector<cudaEvent_t> pipe_gev;      // ... the events of the copy groups of one call
   bool pipe = true;                       // PHMM_PIPE=0: no pipelined host calls
+  int64_t pipe_min = 1ll << 17;           // smallest pipelined batch (kPipeMinPairs; PHMM_PIPE_MIN: tests, sanitizer)
   bool pipe_trace = false;                // PHMM_PIPE_TRACE=1: per-chunk device timeline on stderr
   std::vector<cudaEvent_t> trace_ev;      // ... chunk start / end events
   std::vector<std::pair<const char*, double>> trace_host;  // ... host timestamps (us)
@@ -1342,7 +1343,7 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
   // host-side size checks that need the host offsets
   if (b->read_offsets[b->n_reads] != b->total_read_bases || b->hap_offsets[b->n_haps] != b->total_hap_bases)
     return PHMM_E_INVALID_ARG;
-  if (b->n_pairs >= kPipeMinPairs && b->n_pairs <= c->chunk_pairs && c->pipe)
+  if (b->n_pairs >= c->pipe_min && b->n_pairs <= c->chunk_pairs && c->pipe)
     return compute_host_pipe(c, b, out_log10, out_status);
   cudaStream_t s = c->stream;
   uint8_t *rb, *q, *qi, *qd, *qg, *hap;
@@ -1677,6 +1678,7 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg) {
     }
   }
   if (const char* e = std::getenv("PHMM_PIPE")) c->pipe = std::atoi(e) != 0;
+  if (const char* e = std::getenv("PHMM_PIPE_MIN")) c->pipe_min = std::max<int64_t>(16, std::atoll(e));
   if (const char* e = std::getenv("PHMM_PIPE_TRACE")) c->pipe_trace = std::atoi(e) != 0;
   if (const char* e = std::getenv("PHMM_CHUNK_PAIRS")) c->chunk_pairs = std::max<int64_t>(64, std::atoll(e));
   *out = c;

@@ -207,3 +207,43 @@ def test_pipelined_host_call_is_bitwise_the_one_pass_call(prec):
     finally:
         ctx.close()
         flat.close()
+
+
+@pytest.mark.parametrize("prec", ["fp32", "fp64"])
+def test_pipelined_small_ragged_batches_are_bitwise(prec):
+    """The pipelined host call on small, ragged batches (PHMM_PIPE_MIN lowers its threshold):
+    multi-bin C3 regions, long C4 rows, random pairs of 1..60 x 1..80 bases (some below the
+    40-column minimum) and decoys, with chunks of a few pairs each; pageable and page-locked
+    inputs give the one-pass results bit for bit, statuses included; also for 16..100 pairs,
+    where a chunk may hold a single pair."""
+    import torch
+
+    big = synth.concat_batches([synth.config_batch("C2", n_regions=4),
+                                synth.random_pairs_batch(3, 100, m_range=(1, 60), n_range=(1, 80)),
+                                synth.config_batch("C3", n_regions=2), synth.config_batch("C4", n_regions=1).subset(range(6))])
+    flat_env = {"PHMM_PIPE": "0"}
+    os.environ.update(flat_env)
+    try:
+        flat = phmm.PairHMM(precision=prec)
+    finally:
+        del os.environ["PHMM_PIPE"]
+    os.environ["PHMM_PIPE_MIN"] = "16"
+    try:
+        pipe = phmm.PairHMM(precision=prec)
+    finally:
+        del os.environ["PHMM_PIPE_MIN"]
+    try:
+        for n in (16, 17, 31, 100, big.n_pairs):
+            b = big.subset(np.arange(n)) if n < big.n_pairs else big
+            ref, rst = flat.compute_batch(b)
+            got, gst = pipe.compute_batch(b)
+            assert np.array_equal(got, ref) and np.array_equal(gst, rst), n
+            assert pipe.stats()["n_chunks"] >= 2, (n, pipe.stats()["n_chunks"])
+            pin = synth.Batch(**{k: torch.from_numpy(np.ascontiguousarray(getattr(b, k))).pin_memory().numpy()
+                                 for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals",
+                                           "read_offsets", "hap_bases", "hap_offsets", "pairs")})
+            got2, gst2 = pipe.compute_batch(pin)
+            assert np.array_equal(got2, ref) and np.array_equal(gst2, rst), n
+    finally:
+        flat.close()
+        pipe.close()
