@@ -71,7 +71,7 @@
 extern "C" {
 #endif
 
-#define PHMM_ABI_VERSION 3
+#define PHMM_ABI_VERSION 4
 
 typedef struct phmm_ctx phmm_ctx; /* opaque */
 
@@ -204,6 +204,23 @@ phmm_status phmm_set_stream(phmm_ctx* ctx, void* cuda_stream);
 phmm_status phmm_submit(phmm_ctx* ctx, const phmm_batch* b, double* out_log10, uint8_t* out_status,
                         uint64_t* ticket);
 phmm_status phmm_wait(phmm_ctx* ctx, uint64_t ticket);
+
+/*
+ * Asynchronous host-buffer call WITHOUT an input copy (for large batches streamed one after
+ * another): returns at once with a ticket; the library reads the caller's input arrays and
+ * writes out_log10 / out_status until phmm_wait(ctx, ticket) returns, so the caller keeps all
+ * of them valid and the inputs unchanged until then. Batches of this call run one at a time in
+ * their submission order on the context's worker thread (the phmm_submit queue's); while one
+ * batch computes, the worker already copies the NEXT submitted batch's inputs to the device
+ * (two device input regions, used alternately), when all of that batch's arrays are page-locked
+ * -- so a caller that keeps two batches in flight overlaps one batch's host->device copy with
+ * the other's compute. A batch that was not prefetched runs as phmm_compute_batch. Results are
+ * bitwise those of phmm_compute_batch; phmm_wait returns the batch's status (input errors as
+ * for phmm_compute_batch, outputs then untouched). Returns PHMM_E_INVALID_ARG (NULL
+ * arguments, bad sizes) or PHMM_E_OOM at submission.
+ */
+phmm_status phmm_compute_batch_async(phmm_ctx* ctx, const phmm_batch* b, double* out_log10, uint8_t* out_status,
+                                     uint64_t* ticket);
 
 /* Release the context and its device workspace. NULL-safe, idempotent per pointer. */
 void phmm_destroy(phmm_ctx* ctx);

@@ -224,12 +224,13 @@ struct Stager {
     return cudaSuccess;
   }
 
-  // device -> host on stream s; returns when dst holds the data
-  cudaError_t d2h(void* dst, const void* src, size_t n, cudaStream_t s) {
+  // device -> host on stream s; returns when dst holds the data (a page-locked dst with
+  // sync = false: when the copy is queued; the caller synchronises s)
+  cudaError_t d2h(void* dst, const void* src, size_t n, cudaStream_t s, bool sync = true) {
     if (n == 0) return cudaSuccess;
     if (is_pinned(dst)) {
       cudaError_t e = cudaMemcpyAsync(dst, src, n, cudaMemcpyDeviceToHost, s);
-      return e != cudaSuccess ? e : cudaStreamSynchronize(s);
+      return e != cudaSuccess || !sync ? e : cudaStreamSynchronize(s);
     }
     // keep up to kStageSlots pieces in flight; copy each out as soon as it arrived
     const size_t npieces = (n + kStagePiece - 1) / kStagePiece;

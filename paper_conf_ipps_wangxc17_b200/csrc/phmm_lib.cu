@@ -16,6 +16,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <condition_variable>
+#include <deque>
 #include <map>
 #include <set>
 #include <mutex>
@@ -113,8 +114,12 @@ struct phmm_ctx {
   uint32_t flags = 0;
   int bucket = 4;
   int nsm = 148;
-  Buf buf[2 * B_COUNT];                  // [set][id]: per-chunk buffers exist once per set (pipelined call)
+  Buf buf[4 * B_COUNT];                  // [region][id]: 0 shared + chunk set 0, 1 chunk set 1, 2-3 async inputs
   int set = 0;                            // the buffer set the current chunk uses
+  int iset = 0;                           // input buffers: 0 = the synchronous calls', 1 / 2 = async batches'
+  cudaStream_t pf_stream = nullptr;       // async calls: the next batch's input prefetch
+  cudaEvent_t pf_ev = nullptr;
+  bool in_xjob = false;                   // the worker is running a no-copy batch (maybe_prefetch)
   uint32_t* gerr = nullptr;               // pipelined call: the call-wide device error word
   cudaStream_t stream2 = nullptr;         // pipelined call: the second chunk stream (odd chunks)
   int smem_per_sm = 0, smem_reserved = 0, smem_optin = 0;  // bytes (device attributes)
@@ -193,9 +198,12 @@ phmm_status ws(phmm_ctx* c, int id, size_t count, X** out) {
   if (bytes < 16) bytes = 16;
   // inputs, outputs and the call-wide lists are one per context; every per-chunk buffer has
   // one copy per set, so that two chunks can be in flight on two streams (compute_host_pipe)
-  const bool shared = id <= B_PAIRS || id == B_OUT_LOG10 || id == B_OUT_STATUS || id == B_RLIST ||
+  // (the async calls keep their inputs in regions 2 and 3, so that one batch's inputs can be
+  // prefetched while another computes)
+  const bool input = id <= B_PAIRS;
+  const bool shared = input || id == B_OUT_LOG10 || id == B_OUT_STATUS || id == B_RLIST ||
                       id == B_UNDERFLOW || (id >= B_SW_REF && id <= B_SW_NOPOFF);
-  Buf& b = c->buf[id + (shared ? 0 : c->set * B_COUNT)];
+  Buf& b = c->buf[id + (input ? (c->iset ? (1 + c->iset) * B_COUNT : 0) : (shared ? 0 : c->set * B_COUNT))];
   if (b.n < bytes) {
     if (b.p) cudaFree(b.p);
     b.p = nullptr;
@@ -282,6 +290,10 @@ phmm_status run_validate(phmm_ctx* c, const DevBatch& d) {
   LAUNCHED(c);
   return PHMM_OK;
 }
+
+// While the worker runs a no-copy batch: copy the NEXT queued no-copy batch's inputs to the
+// device now (called at the host round trips of the path, so the copy overlaps this batch).
+void maybe_prefetch(phmm_ctx* c);
 
 // Blocks per SM of a wavefront kernel configuration, cached per context (the occupancy
 // calculator costs microseconds per query, a small batch asks a few times per call).
@@ -397,6 +409,7 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   CUDA_TRY(cudaMemcpyAsync(&hsz[0], item_off + n_items, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   if (hc_off) CUDA_TRY(cudaMemcpyAsync(&hsz[1], hc_off + d.n_haps, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   trace_mark(c, "prep sync");
+  maybe_prefetch(c);
   CUDA_TRY(cudaStreamSynchronize(s));
   trace_mark(c, "prep synced");
   if (c->host_scal->err) return map_err(c->host_scal->err);
@@ -578,6 +591,7 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
     CUDA_TRY(wf_launch<T>(i == 1, (unsigned)(c->nsm * L[i].bps), L[i].warps, smem, s, A));
     ++c->launches;
   }
+  maybe_prefetch(c);
   if (timed) ev_record(c, EV_WF1);
   return PHMM_OK;
 }
@@ -694,6 +708,7 @@ phmm_status compute_one(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     ST_TRY(fp32_pass(c, d, dev_out, dev_status, rlist, 0, &scal->n_rescue, &pi, &hc, &total_hc, true));
     ev_record(c, EV_RESC0);
     CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
+    maybe_prefetch(c);
     CUDA_TRY(cudaStreamSynchronize(s));
     const int64_t nr = c->host_scal->n_rescue;
     c->st.n_rescued += nr;
@@ -1299,7 +1314,7 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, double* out_log1
   ev_record(c, EV_D2H);
   {
     Nvtx nv("phmm:d2h");
-    CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s));
+    CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s, false));  // synchronised below
     if (out_status) CUDA_TRY(S.d2h(out_status, status, b->n_pairs, s));
   }
   ev_record(c, EV_END);
@@ -1392,7 +1407,7 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
   ev_record(c, EV_D2H);
   {
     Nvtx nv("phmm:d2h");
-    CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s));
+    CUDA_TRY(S.d2h(out_log10, out, sizeof(double) * b->n_pairs, s, false));  // synchronised below
     if (out_status) CUDA_TRY(S.d2h(out_status, status, b->n_pairs, s));
   }
   ev_record(c, EV_END);
@@ -1460,6 +1475,17 @@ struct Arena {
   }
 };
 
+// A no-copy batch (phmm_compute_batch_async): the caller's pointers, valid until phmm_wait.
+struct XJob {
+  uint64_t ticket;
+  phmm_batch b;
+  double* out;
+  uint8_t* status;
+  int iset;        // its async input region
+  bool prefetched; // its inputs were copied to that region while the previous batch computed
+  bool tried;      // a prefetch was attempted
+};
+
 struct AsyncQueue {
   std::mutex mu;
   std::condition_variable cv, done_cv;
@@ -1470,6 +1496,8 @@ struct AsyncQueue {
   std::map<uint64_t, phmm_status> done;  // finished tickets not yet waited for
   std::set<uint64_t> outstanding;        // submitted tickets not yet waited for
   std::thread worker;
+  std::deque<XJob> xjobs;                // phmm_compute_batch_async: no-copy batches, in order
+  int xset = 1;                          // the async input region (1 / 2) of the next no-copy batch
 };
 
 void run_arena(phmm_ctx* c, Arena& A) {
@@ -1531,14 +1559,159 @@ void run_arena(phmm_ctx* c, Arena& A) {
   q->done_cv.notify_all();
 }
 
+// Copy every input array of an all-page-locked no-copy batch into its async input region on the
+// prefetch stream (ends with pf_ev). false: not prefetchable (a pageable array) or a copy failed.
+bool prefetch_inputs(phmm_ctx* c, XJob& j) {
+  const phmm_batch& b = j.b;
+  const void* arrs[9] = {b.read_bases, b.base_quals, b.ins_quals, b.del_quals, b.gcp_quals, b.hap_bases,
+                         b.read_offsets, b.hap_offsets, b.pairs};
+  for (const void* a : arrs)
+    if (a && !Stager::is_pinned(a)) return false;
+  if (!c->pf_stream && cudaStreamCreateWithFlags(&c->pf_stream, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaGetLastError();
+    c->pf_stream = nullptr;
+    return false;
+  }
+  if (!c->pf_ev && cudaEventCreateWithFlags(&c->pf_ev, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    c->pf_ev = nullptr;
+    return false;
+  }
+  const int keep = c->iset;
+  c->iset = j.iset;
+  const size_t nr = (size_t)b.total_read_bases, nh = (size_t)b.total_hap_bases;
+  uint8_t* d[6];
+  int64_t *roff, *hoff;
+  int32_t* pairs;
+  bool ok = ws(c, B_READ_BASES, nr, &d[0]) == PHMM_OK && ws(c, B_BQ, nr, &d[1]) == PHMM_OK &&
+            ws(c, B_IQ, nr, &d[2]) == PHMM_OK && ws(c, B_DQ, nr, &d[3]) == PHMM_OK &&
+            ws(c, B_GQ, nr, &d[4]) == PHMM_OK && ws(c, B_HAP, nh, &d[5]) == PHMM_OK &&
+            ws(c, B_ROFF, (size_t)b.n_reads + 1, &roff) == PHMM_OK &&
+            ws(c, B_HOFF, (size_t)b.n_haps + 1, &hoff) == PHMM_OK &&
+            ws(c, B_PAIRS, (size_t)b.n_pairs * 2, &pairs) == PHMM_OK;
+  c->iset = keep;
+  if (!ok) return false;
+  cudaStream_t s = c->pf_stream;
+  const size_t sz[6] = {nr, nr, nr, nr, nr, nh};
+  for (int i = 0; i < 6 && ok; ++i)
+    ok = sz[i] == 0 || cudaMemcpyAsync(d[i], arrs[i], sz[i], cudaMemcpyHostToDevice, s) == cudaSuccess;
+  ok = ok && cudaMemcpyAsync(roff, b.read_offsets, 8 * (size_t)(b.n_reads + 1), cudaMemcpyHostToDevice, s) == cudaSuccess;
+  ok = ok && cudaMemcpyAsync(hoff, b.hap_offsets, 8 * (size_t)(b.n_haps + 1), cudaMemcpyHostToDevice, s) == cudaSuccess;
+  ok = ok && cudaMemcpyAsync(pairs, b.pairs, 8 * (size_t)b.n_pairs, cudaMemcpyHostToDevice, s) == cudaSuccess;
+  ok = ok && cudaEventRecord(c->pf_ev, s) == cudaSuccess;
+  if (!ok) {
+    cudaGetLastError();
+    cudaStreamSynchronize(s);
+  }
+  return ok;
+}
+
+void maybe_prefetch(phmm_ctx* c) {
+  if (!c->in_xjob || !c->aq) return;
+  AsyncQueue* q = c->aq;
+  std::lock_guard<std::mutex> g(q->mu);
+  if (q->xjobs.size() > 1 && !q->xjobs[1].prefetched && !q->xjobs[1].tried) {
+    q->xjobs[1].tried = true;
+    q->xjobs[1].prefetched = prefetch_inputs(c, q->xjobs[1]);
+  }
+}
+
+// One no-copy batch. Prefetched: its inputs are in its async region (after pf_ev): the device
+// path on them, then the results to the caller's buffers; otherwise the host-buffer call with
+// that region as its input buffers. Bitwise phmm_compute_batch (R14).
+phmm_status run_xjob(phmm_ctx* c, XJob& j) {
+  Nvtx nvtx_("phmm:async_batch");
+  const phmm_batch* b = &j.b;
+  c->iset = j.iset;
+  phmm_status st = PHMM_OK;
+  if (!j.prefetched) {
+    st = compute_host(c, b, j.out, j.status);
+    c->iset = 0;
+    return st;
+  }
+  auto run = [&]() -> phmm_status {
+    c->launches = 0;
+    if (b->n_pairs == 0) {
+      c->st = phmm_stats{};
+      return PHMM_OK;
+    }
+    uint8_t *rb, *q, *qi, *qd, *qg, *hap;
+    int64_t *roff, *hoff;
+    int32_t* pairs;
+    double* out;
+    uint8_t* status = nullptr;
+    const size_t nr = (size_t)b->total_read_bases, nh = (size_t)b->total_hap_bases;
+    ST_TRY(ws(c, B_READ_BASES, nr, &rb));
+    ST_TRY(ws(c, B_BQ, nr, &q));
+    ST_TRY(ws(c, B_IQ, nr, &qi));
+    ST_TRY(ws(c, B_DQ, nr, &qd));
+    ST_TRY(ws(c, B_GQ, nr, &qg));
+    ST_TRY(ws(c, B_HAP, nh, &hap));
+    ST_TRY(ws(c, B_ROFF, (size_t)b->n_reads + 1, &roff));
+    ST_TRY(ws(c, B_HOFF, (size_t)b->n_haps + 1, &hoff));
+    ST_TRY(ws(c, B_PAIRS, (size_t)b->n_pairs * 2, &pairs));
+    ST_TRY(ws(c, B_OUT_LOG10, (size_t)b->n_pairs, &out));
+    if (j.status) ST_TRY(ws(c, B_OUT_STATUS, (size_t)b->n_pairs, &status));
+    cudaStream_t s = c->stream;
+    ev_record(c, EV_START);
+    CUDA_TRY(cudaStreamWaitEvent(s, c->pf_ev, 0));
+    ev_record(c, EV_H2D);
+    DevBatch d{rb, q, qi, qd, qg, hap, roff, hoff, pairs, b->n_reads, b->n_haps, b->n_pairs, (int64_t)nr, (int64_t)nh};
+    phmm_status e = compute_dev(c, d, out, status);
+    if (e != PHMM_OK) {
+      cudaStreamSynchronize(s);
+      cudaGetLastError();
+      return e;
+    }
+    ST_TRY(enqueue_underflow_readback(c));
+    ev_record(c, EV_D2H);
+    CUDA_TRY(c->stage.d2h(j.out, out, sizeof(double) * b->n_pairs, s, false));  // synchronised below
+    if (j.status) CUDA_TRY(c->stage.d2h(j.status, status, b->n_pairs, s));
+    ev_record(c, EV_END);
+    CUDA_TRY(cudaStreamSynchronize(s));
+    finish_stats(c);
+    c->st.ms_h2d = -1.f;  // the prefetch overlapped the previous batch
+    c->st.ms_d2h = ev_ms(c, EV_D2H, EV_END);
+    c->st.staged_bytes = c->stage.staged_bytes;
+    return PHMM_OK;
+  };
+  c->stage.staged_bytes = 0;
+  st = run();
+  c->iset = 0;
+  return st;
+}
+
 void async_worker(phmm_ctx* c) {
   AsyncQueue* q = c->aq;
   cudaSetDevice(c->device);
   while (true) {
     int k;
+    // no-copy batches first (in their submission order); the next one's inputs are prefetched
+    // while this one computes
     {
       std::unique_lock<std::mutex> lk(q->mu);
-      q->cv.wait(lk, [&] { return q->stop || !q->arena[q->fill].jobs.empty(); });
+      q->cv.wait(lk, [&] { return q->stop || !q->arena[q->fill].jobs.empty() || !q->xjobs.empty(); });
+      if (!q->xjobs.empty()) {
+        XJob j = q->xjobs.front();
+        q->busy = true;
+        lk.unlock();
+        phmm_status st;
+        {
+          std::lock_guard<std::mutex> g(c->run_mu);
+          // the next batch (its region differs from this one's: regions alternate) is prefetched
+          // at this batch's first host round trip (maybe_prefetch), after its first kernels are
+          // queued, not before them
+          c->in_xjob = true;
+          st = run_xjob(c, j);
+          c->in_xjob = false;
+        }
+        lk.lock();
+        q->xjobs.pop_front();
+        q->done[j.ticket] = st;
+        q->busy = false;
+        q->done_cv.notify_all();
+        continue;
+      }
       if (q->arena[q->fill].jobs.empty()) return;  // stop, nothing left
       k = q->fill;
       q->fill ^= 1;  // submissions go to the other arena while this one runs
@@ -1692,8 +1865,13 @@ void phmm_destroy(phmm_ctx* c) {
   if (c->stream) cudaStreamSynchronize(c->stream);
   for (int i = 0; i < B_COUNT; ++i)
     if (c->buf[i].p) cudaFree(c->buf[i].p);
-  for (int i = 0; i < B_COUNT; ++i)
-    if (c->buf[B_COUNT + i].p) cudaFree(c->buf[B_COUNT + i].p);
+  for (int i = B_COUNT; i < 4 * B_COUNT; ++i)
+    if (c->buf[i].p) cudaFree(c->buf[i].p);
+  if (c->pf_stream) {
+    cudaStreamSynchronize(c->pf_stream);
+    cudaStreamDestroy(c->pf_stream);
+  }
+  if (c->pf_ev) cudaEventDestroy(c->pf_ev);
   if (c->stream2) {
     cudaStreamSynchronize(c->stream2);
     cudaStreamDestroy(c->stream2);
@@ -1801,6 +1979,31 @@ phmm_status phmm_submit(phmm_ctx* c, const phmm_batch* b, double* out_log10, uin
   A.n_haps += nh;
   A.any_status |= out_status != nullptr;
   A.jobs.push_back(j);
+  q->outstanding.insert(j.ticket);
+  *ticket = q->next_ticket++;
+  q->cv.notify_one();
+  return PHMM_OK;
+}
+
+phmm_status phmm_compute_batch_async(phmm_ctx* c, const phmm_batch* b, double* out_log10, uint8_t* out_status,
+                                     uint64_t* ticket) {
+  if (!c || !ticket) return PHMM_E_INVALID_ARG;
+  ST_TRY(check_batch_args(b));
+  if (b->n_pairs > 0 && !out_log10) return PHMM_E_INVALID_ARG;
+  if (b->n_pairs > 0 &&
+      (b->read_offsets[b->n_reads] != b->total_read_bases || b->hap_offsets[b->n_haps] != b->total_hap_bases))
+    return PHMM_E_INVALID_ARG;
+  if (!c->aq) {
+    c->aq = new (std::nothrow) AsyncQueue();
+    if (!c->aq) return PHMM_E_OOM;
+    c->aq->worker = std::thread(async_worker, c);
+  }
+  AsyncQueue* q = c->aq;
+  std::lock_guard<std::mutex> g(q->mu);
+  if (q->stop) return PHMM_E_INVALID_ARG;
+  XJob j{q->next_ticket, *b, out_log10, out_status, q->xset, false, false};
+  q->xset = 3 - q->xset;  // regions alternate 1, 2
+  q->xjobs.push_back(j);
   q->outstanding.insert(j.ticket);
   *ticket = q->next_ticket++;
   q->cv.notify_one();

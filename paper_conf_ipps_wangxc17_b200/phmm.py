@@ -85,7 +85,7 @@ SW_OPS = "MID"
 # every symbol include/phmm.h declares (checked by tests/test_abi.py)
 EXPORTED_SYMBOLS = ("phmm_create", "phmm_compute_batch", "phmm_compute_batch_dev", "phmm_destroy",
                     "phmm_status_string", "phmm_get_stats", "phmm_abi_version", "phmm_set_stream", "phmm_submit", "phmm_wait",
-                    "phmm_sw_align_batch", "phmm_sw_align_batch_dev")
+                    "phmm_compute_batch_async", "phmm_sw_align_batch", "phmm_sw_align_batch_dev")
 
 _lib = None
 
@@ -119,6 +119,9 @@ def load_library(path: str = LIB_PATH):
     L.phmm_submit.restype = ctypes.c_int
     L.phmm_wait.argtypes = [ctypes.c_void_p, ctypes.c_uint64]
     L.phmm_wait.restype = ctypes.c_int
+    L.phmm_compute_batch_async.argtypes = [ctypes.c_void_p, ctypes.POINTER(_Batch), _f64p, _u8p,
+                                           ctypes.POINTER(ctypes.c_uint64)]
+    L.phmm_compute_batch_async.restype = ctypes.c_int
     for f in (L.phmm_sw_align_batch, L.phmm_sw_align_batch_dev):
         f.argtypes = [ctypes.c_void_p, ctypes.POINTER(_SwBatch), ctypes.POINTER(_SwParams), ctypes.c_void_p,
                       ctypes.c_void_p]
@@ -241,13 +244,15 @@ def _check_out(t, dtype, n: int, dev, name: str) -> None:
 
 
 class Ticket:
-    """A submitted batch (``phmm_submit``); ``wait()`` blocks in ``phmm_wait``."""
+    """A submitted batch (``phmm_submit`` / ``phmm_compute_batch_async``); ``wait()`` blocks in
+    ``phmm_wait``. For a no-copy batch the ticket also keeps the input arrays alive."""
 
-    def __init__(self, ctx, ticket: int, out, status):
-        self.ctx, self.ticket, self.out, self.status = ctx, ticket, out, status
+    def __init__(self, ctx, ticket: int, out, status, keep=None):
+        self.ctx, self.ticket, self.out, self.status, self._keep = ctx, ticket, out, status, keep
 
     def wait(self):
         rc = self.ctx._L.phmm_wait(self.ctx._h, self.ticket)
+        self._keep = None
         if rc != PHMM_OK:
             raise PhmmError(rc, "phmm_wait")
         return self.out, self.status
@@ -295,6 +300,39 @@ class PairHMM:
         if rc != PHMM_OK:
             raise PhmmError(rc, "phmm_compute_batch")
         return out, status
+
+    def compute_batch_async(self, batch, out: Optional[np.ndarray] = None, status: Optional[np.ndarray] = None,
+                            want_status: bool = True) -> "Ticket":
+        """``phmm_compute_batch_async``: enqueue a host batch WITHOUT copying it (the ticket keeps
+        the arrays alive; do not modify them before ``wait()``); the next submitted batch's inputs
+        are copied to the device while this one computes when they are page-locked."""
+        s, keep = _host_struct(batch)
+        n = int(s.n_pairs)
+        if out is None:
+            out = np.empty(n, dtype=np.float64)
+        if status is None and want_status:
+            status = np.empty(n, dtype=np.uint8)
+        t = ctypes.c_uint64()
+        rc = self._L.phmm_compute_batch_async(self._h, ctypes.byref(s), out.ctypes.data_as(_f64p),
+                                              status.ctypes.data_as(_u8p) if status is not None else None,
+                                              ctypes.byref(t))
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_compute_batch_async")
+        return Ticket(self, int(t.value), out, status, keep=(keep, s))
+
+    def compute_batch_async_raw(self, s: _Batch, out_ptr: int, status_ptr: int = 0) -> int:
+        """Direct ``phmm_compute_batch_async`` with prepared pointers (bench e2e leg); returns the
+        ticket (raises on a submission error)."""
+        t = ctypes.c_uint64()
+        rc = int(self._L.phmm_compute_batch_async(self._h, ctypes.byref(s), ctypes.cast(out_ptr, _f64p),
+                                                  ctypes.cast(status_ptr, _u8p) if status_ptr else None,
+                                                  ctypes.byref(t)))
+        if rc != PHMM_OK:
+            raise PhmmError(rc, "phmm_compute_batch_async")
+        return int(t.value)
+
+    def wait_raw(self, ticket: int) -> int:
+        return int(self._L.phmm_wait(self._h, ctypes.c_uint64(ticket)))
 
     def compute_batch_raw(self, s: _Batch, out_ptr: int, status_ptr: int = 0) -> int:
         """Direct ``phmm_compute_batch`` with prepared pointers (bench e2e leg)."""

@@ -247,3 +247,57 @@ def test_pipelined_small_ragged_batches_are_bitwise(prec):
     finally:
         flat.close()
         pipe.close()
+
+
+def test_async_no_copy_batches_are_bitwise_and_prefetched():
+    """phmm_compute_batch_async: batches streamed with two in flight (page-locked: the next
+    batch's inputs are prefetched into the other device input region while one computes;
+    pageable: each runs as phmm_compute_batch) give phmm_compute_batch's results bit for bit,
+    in any mix with synchronous calls; a batch with an invalid base fails alone (outputs
+    untouched) and the following ones still succeed."""
+    import torch
+
+    ctx = phmm.PairHMM(precision="fp32")
+    try:
+        batches = [synth.config_batch("C2", n_regions=256, region_start=256 * k) for k in range(3)]
+        batches.append(synth.config_batch("C3", n_regions=16))
+        batches.append(synth.random_pairs_batch(5, 500))
+        keys = ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets", "hap_bases",
+                "hap_offsets", "pairs")
+        pinned = [synth.Batch(**{k: torch.from_numpy(np.ascontiguousarray(getattr(b, k))).pin_memory().numpy()
+                                 for k in keys}) for b in batches]
+        refs = [ctx.compute_batch(b) for b in batches]
+        bad = batches[1].subset(np.arange(batches[1].n_pairs))
+        bad.read_bases = bad.read_bases.copy()
+        bad.read_bases[7] = ord("Q")
+        badp = synth.Batch(**{k: torch.from_numpy(np.ascontiguousarray(getattr(bad, k))).pin_memory().numpy()
+                              for k in keys})
+        for rnd in range(2):
+            srcs = pinned if rnd == 0 else batches  # page-locked (prefetched), then pageable
+            ts = []
+            for k, b in enumerate(srcs):
+                if k == 2:
+                    o = torch.empty(bad.n_pairs, dtype=torch.float64).pin_memory().numpy()
+                    o[:] = 9.0
+                    ts.append(("bad", ctx.compute_batch_async(badp if rnd == 0 else bad, out=o)))
+                ts.append((k, ctx.compute_batch_async(b)))
+                if len(ts) >= 3:  # keep two or three in flight
+                    k0, t0 = ts.pop(0)
+                    _check(k0, t0, refs)
+            # a synchronous call in between must not disturb the queued batches
+            mid, _ = ctx.compute_batch(batches[0])
+            assert np.array_equal(mid, refs[0][0])
+            for k0, t0 in ts:
+                _check(k0, t0, refs)
+    finally:
+        ctx.close()
+
+
+def _check(k, t, refs):
+    if k == "bad":
+        with pytest.raises(phmm.PhmmError) as ei:
+            t.wait()
+        assert ei.value.code == -2 and np.all(t.out == 9.0)
+        return
+    got, st = t.wait()
+    assert np.array_equal(got, refs[k][0]) and np.array_equal(st, refs[k][1]), k
