@@ -278,6 +278,12 @@ def _e2e_leg(args, ctx, batch, ws, flush, stream, gloo, n_slot, pair_start, pinn
         # last result
         outs = [(hout, hst)] + [(torch.empty(n, dtype=torch.float64).pin_memory(),
                                  torch.empty(n, dtype=torch.uint8).pin_memory()) for _ in range(inflight - 1)]
+        # warm-up of the async path itself (its device input regions are allocated on first use)
+        wq = [ctx.compute_batch_async_raw(s, o.data_ptr(), st_.data_ptr()) for o, st_ in outs]
+        for t in wq:
+            assert ctx.wait_raw(t) == 0
+        if ws > 1:
+            dist.barrier()
         t0 = time.perf_counter()
         q = []
         for i in range(args.steps):
