@@ -50,6 +50,7 @@ enum BufId {
   B_DEDUP,                                       // rescue pass: head flags + their scan (one table per read)
   B_CH_RANGES,                                   // chunked device call: read / haplotype index range per chunk
   B_UNDERFLOW,                                   // pairs of the call whose FP64 sum underflowed
+  B_RLIST_CH,                                    // a chunk's own rescue list (per set: compute_one in a pipelined call)
   B_COUNT
 };
 
@@ -702,8 +703,8 @@ phmm_status compute_one(phmm_ctx* c, const DevBatch& d, double* dev_out, uint8_t
     c->st.cells += (int64_t)pi.cells;
     c->st.padded_cells += (int64_t)pi.padded_cells;
   } else {
-    int32_t* rlist;
-    ST_TRY(ws(c, B_RLIST, (size_t)d.n_pairs, &rlist));
+    int32_t* rlist;  // per set: two chunks of a pipelined call may be in flight
+    ST_TRY(ws(c, B_RLIST_CH, (size_t)d.n_pairs, &rlist));
     CUDA_TRY(fill_async(c, &scal->n_rescue, 0, sizeof(int64_t) + sizeof(unsigned long long), s));
     ST_TRY(fp32_pass(c, d, dev_out, dev_status, rlist, 0, &scal->n_rescue, &pi, &hc, &total_hc, true));
     ev_record(c, EV_RESC0);
@@ -986,17 +987,23 @@ constexpr int kPipeFirstDivPageable = 4, kPipeMaxChPageable = 64;
 // tools/h2d_probe4.py) -- so the device computes them (k_chunk_ranges) after the pair list
 // arrived; a pageable pair list (which is staged through the context's slots anyway) is
 // scanned by the copy pool (pipe_scan), so the copies start at once.
-void pipe_chunks(int64_t n, bool pinned, std::vector<PipeChunk>& ch, int64_t* sub) {
+void pipe_chunks(int64_t n, bool pinned, int64_t cap, std::vector<PipeChunk>& ch, int64_t* sub) {
   int div = pinned ? kPipeFirstDivPinned : kPipeFirstDivPageable;
   if (const char* e = std::getenv("PHMM_PIPE_FIRST")) div = std::max(2, std::min(1024, std::atoi(e)));
   int maxch = pinned ? kPipeMaxChPinned : kPipeMaxChPageable;
   if (const char* e = std::getenv("PHMM_PIPE_MAXCH")) maxch = std::max(2, std::atoi(e));
-  *sub = std::max<int64_t>(1, n / div);
+  *sub = std::min<int64_t>(std::max<int64_t>(1, n / div), cap);
   ch.clear();
   for (int64_t p = 0, sz = *sub, k = 0; p < n; ++k) {
     // no runt chunk at the end; at most maxch chunks
     const int64_t e = (n - (p + sz) < *sub || k + 1 >= maxch) ? n : p + sz;
-    ch.push_back(PipeChunk{p, e, 0, 0, 0, 0, 0, 0});
+    // chunks of at most cap pairs (the device-call chunk size: per-chunk tables and descriptors
+    // stay a few GB), as whole sub-chunks
+    for (int64_t a = p; a < e;) {
+      const int64_t z = (e - a > cap) ? a + std::max<int64_t>(*sub, cap / *sub * *sub) : e;
+      ch.push_back(PipeChunk{a, z, 0, 0, 0, 0, 0, 0});
+      a = z;
+    }
     p = e;
     if (k >= 1) sz *= 2;
   }
@@ -1077,7 +1084,11 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, double* out_log1
   std::vector<PipeChunk>& ch = c->pipe_chunks;
   int64_t sub = 0;
   const bool pinned = Stager::is_pinned(b->read_bases) && Stager::is_pinned(b->pairs);
-  pipe_chunks(b->n_pairs, pinned, ch, &sub);
+  pipe_chunks(b->n_pairs, pinned, c->chunk_pairs, ch, &sub);
+  // batches larger than one device chunk: every chunk runs its own FP64 rescue (compute_one), as
+  // in the chunked device call (one rescue over all of them would outgrow the 32-bit code-region
+  // offsets); otherwise one rescue pass over the whole batch at the end
+  const bool chunk_rescue = b->n_pairs > c->chunk_pairs;
   const int64_t nsub = (b->n_pairs + sub - 1) / sub;
   const int nmax = (int)ch.size();
   while ((int)c->pipe_ev.size() < nmax + 4) {
@@ -1267,7 +1278,7 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, double* out_log1
       DevBatch dk{rb, q, qi, qd, qg, hap, roff_c, hoff_c, pairs_c, nrk, nhk, np, (int64_t)nr, (int64_t)nh};
       double* o = out + k.p0;
       uint8_t* st = status ? status + k.p0 : nullptr;
-      if (c->prec == PHMM_PREC_FP64) {
+      if (c->prec == PHMM_PREC_FP64 || chunk_rescue) {
         ST_TRY(compute_one(c, dk, o, st));
       } else {
         PassInfo pi;
@@ -1290,7 +1301,7 @@ phmm_status compute_host_pipe(phmm_ctx* c, const phmm_batch* b, double* out_log1
     CUDA_TRY(cudaMemcpyAsync(c->host_scal, scal, sizeof(Scalars), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
     if (c->host_scal->err) return map_err(c->host_scal->err);
-    if (c->prec == PHMM_PREC_FP32_RESCUE) {
+    if (c->prec == PHMM_PREC_FP32_RESCUE && !chunk_rescue) {
       const int64_t n_resc = c->host_scal->n_rescue;
       c->st.n_rescued += n_resc;
       if (n_resc > 0) ST_TRY(rescue_pass(c, d, out, status, rlist, n_resc, nullptr, 0, false));
@@ -1358,7 +1369,7 @@ phmm_status compute_host(phmm_ctx* c, const phmm_batch* b, double* out_log10, ui
   // host-side size checks that need the host offsets
   if (b->read_offsets[b->n_reads] != b->total_read_bases || b->hap_offsets[b->n_haps] != b->total_hap_bases)
     return PHMM_E_INVALID_ARG;
-  if (b->n_pairs >= c->pipe_min && b->n_pairs <= c->chunk_pairs && c->pipe)
+  if (b->n_pairs >= c->pipe_min && c->pipe)
     return compute_host_pipe(c, b, out_log10, out_status);
   cudaStream_t s = c->stream;
   uint8_t *rb, *q, *qi, *qd, *qg, *hap;

@@ -301,3 +301,38 @@ def _check(k, t, refs):
         return
     got, st = t.wait()
     assert np.array_equal(got, refs[k][0]) and np.array_equal(st, refs[k][1]), k
+
+
+def test_pipelined_call_above_the_device_chunk_is_bitwise():
+    """A host batch larger than one device chunk (PHMM_CHUNK_PAIRS lowers it to 5,000 pairs
+    here) runs pipelined in chunks of at most that many pairs, each with its own FP64 rescue
+    (as the chunked device call): bitwise the one-pass call, pageable and page-locked."""
+    import torch
+
+    b = synth.concat_batches([synth.config_batch("C2", n_regions=160), synth.config_batch("C3", n_regions=24)])
+    os.environ["PHMM_PIPE"] = "0"
+    try:
+        flat = phmm.PairHMM(precision="fp32")
+    finally:
+        del os.environ["PHMM_PIPE"]
+    os.environ["PHMM_CHUNK_PAIRS"] = "5000"
+    os.environ["PHMM_PIPE_MIN"] = "64"
+    try:
+        pipe = phmm.PairHMM(precision="fp32")
+    finally:
+        del os.environ["PHMM_CHUNK_PAIRS"]
+        del os.environ["PHMM_PIPE_MIN"]
+    try:
+        ref, rst = flat.compute_batch(b)
+        got, gst = pipe.compute_batch(b)
+        st = pipe.stats()
+        assert st["n_chunks"] >= (b.n_pairs + 4999) // 5000 and st["n_rescued"] == flat.stats()["n_rescued"]
+        assert np.array_equal(got, ref) and np.array_equal(gst, rst)
+        pin = synth.Batch(**{k: torch.from_numpy(np.ascontiguousarray(getattr(b, k))).pin_memory().numpy()
+                             for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals",
+                                       "read_offsets", "hap_bases", "hap_offsets", "pairs")})
+        got2, gst2 = pipe.compute_batch(pin)
+        assert np.array_equal(got2, ref) and np.array_equal(gst2, rst)
+    finally:
+        flat.close()
+        pipe.close()
