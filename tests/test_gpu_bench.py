@@ -88,7 +88,7 @@ def test_bench_multi_rank_path_is_bitwise_across_rank_counts():
         assert d["n_gpus"] == n and d["scaling"] == "strong"
         assert d["config"]["job_cells"] == one["config"]["job_cells"]
         assert d["result_sha256"] == one["result_sha256"], n
-        assert d["e2e"]["value"] > 0
+        assert d["e2e"]["value"] > 0 and d["e2e"]["streamed"]["value"] > 0
     w = _bench_line(["--workload", "C2", "--regions", "8", "--steps", "2", "--warmup", "3", "--no-cpu-baseline",
                      "--no-e2e", "--no-extra"], nproc=2, env_extra={"PHMM_BENCH_BACKEND": "gloo"})
     assert w["scaling"] == "weak" and w["config"]["job_pairs"] == 2 * 8 * 16 * 8
