@@ -148,8 +148,8 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg);
  * previous piece is in flight; phmm_stats.staged_bytes counts these bytes). The
  * number of host threads is min(8, cores / 2), or PHMM_STAGE_THREADS when the
  * context is created.
- * Pipelining: a batch of >= 2^17 pairs runs as chunks of pairs (page-locked inputs: n/8 and
- * 7n/8; pageable: n/4, n/4, n/2; at most 2^23 pairs each): a context-owned copy thread
+ * Pipelining: a batch of >= 2^17 pairs runs as chunks of pairs (n/8 and 7n/8, at most 2^23
+ * pairs each): a context-owned copy thread
  * moves chunk k+1's new input bytes to the device on a copy stream while chunk k computes,
  * chunks alternate between two compute streams, and one FP64 rescue pass over the whole
  * batch follows (batches above 2^23 pairs: a rescue per chunk). Results are bitwise those

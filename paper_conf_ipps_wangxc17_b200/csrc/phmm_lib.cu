@@ -973,11 +973,11 @@ void finish_stats(phmm_ctx* c) {
 // underflowing pairs to one list and ONE FP64 rescue pass over the whole batch follows, so the
 // call has one host round trip per chunk plus two. Results are bitwise those of the one-pass call.
 constexpr int64_t kPipeMinPairs = 1ll << 17;
-// chunk plans (measured on C2, profiles/r02_pipe_sweep.txt): page-locked inputs n/8 + 7n/8 (the
-// copy engine keeps up with the compute); pageable ones n/4, n/4, n/2 (the staging memcpy is the
-// slower side, so more and smaller chunks overlap it better)
+// chunk plans (measured on C2, profiles/r02_pipe_sweep.txt): n/8 + 7n/8 for page-locked and
+// pageable inputs alike (with streaming-store staging the staging memcpy keeps up as well; more,
+// smaller chunks cost more in chunk boundaries than they hide)
 constexpr int kPipeFirstDivPinned = 8, kPipeMaxChPinned = 2;
-constexpr int kPipeFirstDivPageable = 4, kPipeMaxChPageable = 64;
+constexpr int kPipeFirstDivPageable = 8, kPipeMaxChPageable = 2;
 
 
 // Chunk boundaries of a pipelined call: sub-chunks of n/F pairs, chunk k = 1, 1, 2, 4, ...

@@ -139,7 +139,7 @@ def test_submit_queue_coalesces_regions_bitwise():
 @pytest.mark.parametrize("prec", ["fp32", "fp64"])
 def test_pipelined_host_call_is_bitwise_the_one_pass_call(prec):
     """A host batch of 2^17 .. 2^23 pairs in region order runs pipelined (compute_host_pipe):
-    chunks of n/8 + 7n/8 pairs (page-locked inputs) or n/4, n/4, n/2 (pageable), alternating between two streams and two buffer sets, whose input bytes reach the
+    chunks of n/8 + 7n/8 pairs, alternating between two streams and two buffer sets, whose input bytes reach the
     device on a copy stream while the previous chunk computes; one FP64 rescue over the whole
     batch at the end. Results and statuses must equal the device call and the unpipelined host
     call (PHMM_PIPE=0) bit for bit, pageable and page-locked; staged_bytes counts every input
@@ -163,7 +163,7 @@ def test_pipelined_host_call_is_bitwise_the_one_pass_call(prec):
         dev, dst = dev.cpu().numpy(), dst.cpu().numpy()
         got, st = ctx.compute_batch(b)
         stats = ctx.stats()
-        assert stats["n_chunks"] == 3, stats
+        assert stats["n_chunks"] == 2, stats
         assert stats["staged_bytes"] == b.nbytes_inputs() + 9 * n
         assert stats["cells"] == b.cells()
         assert np.array_equal(got, dev) and np.array_equal(st, dst)
