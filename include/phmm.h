@@ -149,10 +149,11 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg);
  * number of host threads is min(8, cores / 2), or PHMM_STAGE_THREADS when the
  * context is created.
  * Pipelining: a batch of >= 2^17 pairs runs as chunks of pairs (n/8 and 7n/8, at most 2^23
- * pairs each): a context-owned copy thread
- * moves chunk k+1's new input bytes to the device on a copy stream while chunk k computes,
- * chunks alternate between two compute streams, and one FP64 rescue pass over the whole
- * batch follows (batches above 2^23 pairs: a rescue per chunk). Results are bitwise those
+ * pairs each): a context-owned copy thread moves chunk k+1's new input bytes to the device
+ * on a copy stream while chunk k computes, chunks alternate between two compute streams,
+ * and one FP64 rescue pass over the whole batch follows (batches above 2^23 pairs: a rescue
+ * per chunk). Fills of device scratch are kernels, not cudaMemsetAsync (which would queue
+ * behind the copy stream's transfers). Results are bitwise those
  * of the unpipelined call (PHMM_PIPE=0 at context creation disables it). Pairs that use
  * reads and haplotypes in ascending index ranges (region after region, as GATK emits them)
  * overlap best; a batch whose first chunk would need more than half of the input bytes
