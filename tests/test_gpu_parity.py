@@ -505,6 +505,11 @@ def test_full_c5_one_gpu_sampled(ctx32):
     sample = np.unique(np.concatenate([rng.choice(b.n_pairs, 4000, replace=False),
                                        rng.permutation(np.nonzero(st != 0)[0])[:1000]]))
     _check(out[sample], oracle.batch_log10(b, pair_idx=sample), "fp32")
+    # the host-buffer call on the same job (pipelined: 2^23-pair chunks whose inputs a copy thread
+    # moves while the previous chunk computes, a rescue per chunk): bitwise the device call
+    hout, hst = ctx32.compute_batch(b)
+    assert ctx32.stats()["n_chunks"] >= 8
+    assert np.array_equal(hout, out) and np.array_equal(hst, st)
 
 
 @pytest.mark.parametrize("seed", [71, 72, 73, 74])
