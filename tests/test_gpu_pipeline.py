@@ -336,3 +336,40 @@ def test_pipelined_call_above_the_device_chunk_is_bitwise():
     finally:
         flat.close()
         pipe.close()
+
+
+@pytest.mark.parametrize("window", [1000, 30000, 0])
+def test_pipelined_call_with_overlapping_chunk_ranges(window):
+    """Pairs shuffled inside windows of `window` pairs (0: the whole batch) so that consecutive
+    chunks use overlapping read / haplotype index ranges (a chunk's reads partly brought by the
+    previous chunk's bytes; with a full shuffle the first chunk needs everything and the call runs
+    as one chunk): bitwise the one-pass call, page-locked and pageable."""
+    import torch
+
+    b = synth.concat_batches([synth.config_batch("C2", n_regions=1200), synth.config_batch("C3", n_regions=40)])
+    n = b.n_pairs
+    rng = np.random.default_rng(window + 5)
+    if window:
+        perm = np.concatenate([s + rng.permutation(min(window, n - s)) for s in range(0, n, window)])
+    else:
+        perm = rng.permutation(n)
+    bs = b.subset(perm)
+    os.environ["PHMM_PIPE"] = "0"
+    try:
+        flat = phmm.PairHMM(precision="fp32")
+    finally:
+        del os.environ["PHMM_PIPE"]
+    pipe = phmm.PairHMM(precision="fp32")
+    try:
+        ref, rst = flat.compute_batch(bs)
+        got, gst = pipe.compute_batch(bs)
+        assert np.array_equal(got, ref) and np.array_equal(gst, rst)
+        assert pipe.stats()["n_chunks"] == (1 if window == 0 else 2), pipe.stats()["n_chunks"]
+        pin = synth.Batch(**{k: torch.from_numpy(np.ascontiguousarray(getattr(bs, k))).pin_memory().numpy()
+                             for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals",
+                                       "read_offsets", "hap_bases", "hap_offsets", "pairs")})
+        got2, gst2 = pipe.compute_batch(pin)
+        assert np.array_equal(got2, ref) and np.array_equal(gst2, rst)
+    finally:
+        flat.close()
+        pipe.close()
