@@ -10,7 +10,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libphmm.so")
-SOURCES = [os.path.join(CSRC, "phmm_lib.cu"), os.path.join(CSRC, "wf.cu"), os.path.join(CSRC, "wf_long32.cu")]
+SOURCES = [os.path.join(CSRC, "phmm_lib.cu"), os.path.join(CSRC, "wf.cu"), os.path.join(CSRC, "wf_long32.cu"),
+           os.path.join(CSRC, "wf_f64.cu")]
 # per-source extra flags: the FP32 short-row and the FP64 wavefront kernels are faster with
 # ptxas -O1, the FP32 long-row kernel with the default -O3
 SOURCE_FLAGS = {"wf.cu": ["-Xptxas", "-O1"]}

@@ -696,7 +696,10 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   // long segment of a pass by the FP32 long-row kernel only: C4 kernel +5 %, while the
   // FP32 short-row kernel (-O1) loses 3 % on C2 and the FP64 kernel 1 % with it
   // (profiles/r02_ab_unroll3.txt).
-  constexpr bool kUnroll3 = kLong && sizeof(T) == 4;
+#ifndef PHMM_UNROLL3_F64
+#define PHMM_UNROLL3_F64 0
+#endif
+  constexpr bool kUnroll3 = (kLong && sizeof(T) == 4) || (PHMM_UNROLL3_F64 && sizeof(T) == 8);
   auto group12 = [&](uint32_t& a0, uint32_t& a1, uint32_t& a2, uint32_t& b0, uint32_t& b1, uint32_t& b2) {
     a2 = __ldg(pA); b2 = __ldg(pB); ++pA; ++pB;
     step(0, a0, b0); step(1, a0, b0); step(2, a0, b0); step(3, a0, b0);
