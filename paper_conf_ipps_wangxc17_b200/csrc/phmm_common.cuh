@@ -72,6 +72,11 @@ struct BlkDesc {
 };
 static_assert(sizeof(BlkDesc) == 16, "BlkDesc must be 16 bytes");
 constexpr uint16_t BLK_LAST = 1, BLK_FIRST = 2;
+// block of a pair of more than 64 blocks (FP32: reads of more than 509 bases), the only pairs the
+// ring rescale of the long-row kernel may rescale: a pair that fits in one pass
+// is never rescaled, so its result cannot depend on where the pass boundaries fall in it
+constexpr uint16_t BLK_RESC = 4;
+constexpr int kRescaleMinBlocks = 65;
 
 __host__ __device__ constexpr int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 

@@ -278,7 +278,8 @@ __global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32
         d.out_idx = (int32_t)slote;
         d.pad = 0;
         const int rrow = (fe / K == j) ? (fe % K) : WF_RROW_NONE;
-        d.flags = (uint16_t)((j == nbe - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) | (rrow << WF_RROW_SHIFT));
+        d.flags = (uint16_t)((j == nbe - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) |
+                             (nbe >= kRescaleMinBlocks ? BLK_RESC : 0) | (rrow << WF_RROW_SHIFT));
         blk[pos] = d;
       }
     }

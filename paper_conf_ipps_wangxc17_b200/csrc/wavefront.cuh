@@ -88,7 +88,7 @@ constexpr int WF_KC64 = PHMM_F64_K / 2;  // ... of the FP64 pass (K doubles)
 // (the FP64 pass, which reads the same code arrays, scales it by WF_KC64 / WF_KC32)
 constexpr int WF_CB = 2 * WF_KC32;
 
-// BlkDesc.flags: bit0 last, bit1 first, bits 8-11 R row (15 = none)
+// BlkDesc.flags: bit0 last, bit1 first, bit2 BLK_RESC (pair of >= 65 blocks), bits 8-11 R row (15 = none)
 constexpr uint16_t WF_RROW_SHIFT = 8;
 constexpr uint16_t WF_RROW_NONE = 15;
 
@@ -443,8 +443,10 @@ __device__ __forceinline__ void wf_commit(Lane<T>& L, uint32_t stg_s, T d0) {
 #endif
 // Ring rescale helpers, used once per rescaled pass by the non-inlined
 // wf_ring_rescale, so they do not perturb the register allocation of the hot loop.
-// Max of the ring row (slots [0, ncols], every value incl. the FP32 slot padding, which is
-// 0 or a scaled copy of real values), reduced over the warp.
+// Max of the ring row (slots [0, ncols]: M, I, D of every slot; NOT the 4th word of a 16-byte
+// FP32 slot, which no store writes and which therefore holds whatever an earlier stream left
+// there -- reading it made the rescale, and so a pair's rounding and rescue decision, depend on
+// the warp's history, i.e. on the batch the pair ran in), reduced over the warp.
 // (the ring addresses travel as 64-bit values: that is the code generation measured, §4.8)
 template <typename T>
 __device__ __forceinline__ T ring_ld1(uint64_t a) {
@@ -462,10 +464,20 @@ __device__ __forceinline__ void ring_st1(uint64_t a, T x) {
 template <typename T, bool kPacked>
 __device__ __forceinline__ T wf_ring_max(uint64_t ring_a, int ncols, int lane) {
   constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
-  const int nw = (ncols + 1) * (int)(RS / sizeof(T));
   T m = 0;
   __syncwarp();
-  for (int k = lane; k < nw; k += 32) m = fmax(m, ring_ld1<T>(ring_a + (uint64_t)(k * (int)sizeof(T))));
+  if constexpr (sizeof(T) == 4 && RS == 16) {
+    // one 16-byte load per slot (consecutive lanes on consecutive slots: 4 wavefronts per warp
+    // load, no conflicts), the three values of the slot
+    for (int j = lane; j <= ncols; j += 32) {
+      float x, y, z;
+      ring_get3((uint32_t)ring_a + 16u * (uint32_t)j, x, y, z);
+      m = fmax(m, fmax(x, fmax(y, z)));
+    }
+  } else {
+    const int nw = (ncols + 1) * (int)(RS / sizeof(T));
+    for (int k = lane; k < nw; k += 32) m = fmax(m, ring_ld1<T>(ring_a + (uint64_t)(k * (int)sizeof(T))));
+  }
   for (int o = 16; o > 0; o >>= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
   return m;
 }
@@ -474,21 +486,36 @@ __device__ __forceinline__ T wf_ring_max(uint64_t ring_a, int ncols, int lane) {
 // (cannot happen with the exact row max; such a pair would go to the FP64 rescue).
 template <typename T, bool kPacked>
 __device__ __forceinline__ bool wf_ring_scale(uint64_t ring_a, int ncols, int lane, int sh) {
-  // the slots as a flat array of T (FP32: the 4th word of a 16-byte slot is padding and is
-  // scaled too): consecutive lanes on consecutive words, no bank conflicts
   constexpr uint32_t RS = kPacked ? 3u * (uint32_t)sizeof(T) : ring_slot_bytes<T, false>();
-  const int nw = (ncols + 1) * (int)(RS / sizeof(T));
   const T f = (T)__int_as_float((127 + sh) << 23);
   const T cap = (T)__int_as_float((127 + PHMM_RS_CAP) << 23);
   bool sat = false;
   __syncwarp();
-  for (int k = lane; k < nw; k += 32) {
-    const uint64_t a = ring_a + (uint64_t)(k * (int)sizeof(T));
-    T x = ring_ld1<T>(a);
-    x *= f;
-    sat |= x > cap;
-    x = fmin(x, cap);
-    ring_st1<T>(a, x);
+  if constexpr (sizeof(T) == 4 && RS == 16) {
+    // slot-wise 16-byte loads and stores (the 4th word, padding, is written back unchanged)
+    for (int j = lane; j <= ncols; j += 32) {
+      const uint32_t a = (uint32_t)ring_a + 16u * (uint32_t)j;
+      float v[4];
+      lds16(a, v);
+#pragma unroll
+      for (int t = 0; t < 3; ++t) {
+        v[t] *= f;
+        sat |= v[t] > cap;
+        v[t] = fmin(v[t], cap);
+      }
+      sts16(a, make_uint4(__float_as_uint(v[0]), __float_as_uint(v[1]), __float_as_uint(v[2]), __float_as_uint(v[3])));
+    }
+  } else {
+    // the slots as a flat array of T: consecutive lanes on consecutive words, no bank conflicts
+    const int nw = (ncols + 1) * (int)(RS / sizeof(T));
+    for (int k = lane; k < nw; k += 32) {
+      const uint64_t a = ring_a + (uint64_t)(k * (int)sizeof(T));
+      T x = ring_ld1<T>(a);
+      x *= f;
+      sat |= x > cap;
+      x = fmin(x, cap);
+      ring_st1<T>(a, x);
+    }
   }
   __syncwarp();
   return __any_sync(0xffffffffu, sat);
@@ -721,7 +748,8 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
       if (e2 == 0) {
         c0 = -1 - SH;  // virtual lane 0 starts its pass
         if constexpr (rescale) {
-          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && ncols >= WF_RESCALE_COLS;
+          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && (dnA.flags & BLK_RESC) &&
+                            ncols >= WF_RESCALE_COLS;
           wf_ring_rescale<T, ring_packed<T, kLong>()>((uint64_t)ring_s, ncols, lane, cont,
                                                       A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
         }

@@ -1,0 +1,96 @@
+"""Stress of the multi-stream host paths: random batch shapes (sizes, region mixes, local pair
+shuffles, page-locked or pageable, FP32 or FP64) through the pipelined host call and the
+streamed async call, each compared bit for bit with the one-pass call. Prints one line per
+round and a final summary; exits non-zero on the first mismatch."""
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+KEYS = ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals", "read_offsets", "hap_bases",
+        "hap_offsets", "pairs")
+
+
+def main():
+    import torch
+
+    from paper_conf_ipps_wangxc17_b200 import phmm, synth
+    rounds = int(sys.argv[1]) if len(sys.argv) > 1 else 12
+    rng = np.random.default_rng(2024)
+    os.environ["PHMM_PIPE"] = "0"
+    flat = {p: phmm.PairHMM(precision=p) for p in ("fp32", "fp64")}
+    del os.environ["PHMM_PIPE"]
+    os.environ["PHMM_PIPE_MIN"] = "512"
+    pipe = {p: phmm.PairHMM(precision=p) for p in ("fp32", "fp64")}
+    del os.environ["PHMM_PIPE_MIN"]
+    n_checked = 0
+    for r in range(rounds):
+        parts = []
+        for _ in range(int(rng.integers(1, 4))):
+            w = ["C2", "C3", "C4"][int(rng.integers(0, 3))]
+            nreg = {"C2": int(rng.integers(4, 400)), "C3": int(rng.integers(2, 40)), "C4": 1}[w]
+            b = synth.config_batch(w, n_regions=nreg, region_start=int(rng.integers(0, 1000)))
+            if w == "C4":
+                b = b.subset(np.arange(min(b.n_pairs, int(rng.integers(16, 200)))))
+            parts.append(b)
+        if rng.random() < 0.3:
+            parts.append(synth.random_pairs_batch(int(rng.integers(0, 1 << 30)), int(rng.integers(50, 3000))))
+        b = synth.concat_batches(parts)
+        win = int(rng.choice([0, 64, 5000]))
+        if win:
+            n = b.n_pairs
+            perm = np.concatenate([s + rng.permutation(min(win, n - s)) for s in range(0, n, win)])
+            b = b.subset(perm)
+        prec = "fp32" if rng.random() < 0.75 else "fp64"
+        ref, rst = flat[prec].compute_batch(b)
+        src = b
+        if rng.random() < 0.5:
+            src = synth.Batch(**{k: torch.from_numpy(np.ascontiguousarray(getattr(b, k))).pin_memory().numpy()
+                                 for k in KEYS})
+        got, gst = pipe[prec].compute_batch(src)
+        nch = pipe[prec].stats()["n_chunks"]
+        t1 = pipe[prec].compute_batch_async(src)
+        t2 = pipe[prec].compute_batch_async(src)
+        a1, s1 = t1.wait()
+        a2, s2 = t2.wait()
+        # bitwise except the layout-dependent pairs (reads > 509 bases against haplotypes >= 766
+        # bases: the ring rescale at pass boundaries, R14), which agree within 1e-4
+        m = b.read_lengths()[b.pairs[:, 0]]
+        nh = b.hap_lengths()[b.pairs[:, 1]]
+        dep = (m > 509) & (nh >= 766)
+
+        def same(x, y):
+            if not (np.array_equal(x[~dep], ref[~dep]) and np.array_equal(y[~dep], rst[~dep])):
+                return False
+            fin = np.isfinite(ref[dep])
+            return (np.all(np.isfinite(x[dep]) == fin) and
+                    np.max(np.abs(x[dep][fin] - ref[dep][fin]), initial=0.0) <= 1e-4 and
+                    np.all((y[dep] <= 1) == (rst[dep] <= 1)))
+
+        ok = same(got, gst) and same(a1, s1) and same(a2, s2)
+        print(f"round {r}: {b.n_pairs} pairs, {prec}, window {win}, chunks {nch}, "
+              f"{'pinned' if src is not b else 'pageable'}: {'ok' if ok else 'MISMATCH'}", flush=True)
+        if not ok:
+            for name, (x, y) in {"pipelined": (got, gst), "async1": (a1, s1), "async2": (a2, s2)}.items():
+                bad = np.nonzero((x != ref) & ~(np.isnan(x) & np.isnan(ref)) & ~dep)[0]
+                sbad = np.nonzero(y != rst)[0]
+                print(f"  {name}: {bad.size} values differ, {sbad.size} statuses differ; first {bad[:10].tolist()}",
+                      flush=True)
+                if bad.size:
+                    k = bad[:5]
+                    print("    ref", ref[k].tolist(), "got", x[k].tolist(), "st ref", rst[k].tolist(),
+                          "st got", y[k].tolist(), "pairs", b.pairs[k].tolist())
+            again, ast = pipe[prec].compute_batch(src)
+            print("  pipelined again equal to ref:", np.array_equal(again, ref), "to first:", np.array_equal(again, got))
+            ref2, _ = flat[prec].compute_batch(b)
+            print("  flat again equal to ref:", np.array_equal(ref2, ref))
+            print("  parts:", [(p.n_pairs, p.n_reads, p.n_haps) for p in parts], "stats:", pipe[prec].stats())
+            sys.exit(1)
+        n_checked += 1
+    print(f"all {n_checked} rounds bitwise equal")
+
+
+if __name__ == "__main__":
+    main()
