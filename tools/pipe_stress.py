@@ -1,6 +1,7 @@
 """Stress of the multi-stream host paths: random batch shapes (sizes, region mixes, local pair
-shuffles, page-locked or pageable, FP32 or FP64) through the pipelined host call and the
-streamed async call, each compared bit for bit with the one-pass call. Prints one line per
+shuffles, page-locked or pageable, FP32 or FP64) through the pipelined host call, the streamed
+async call and the device call split into 3,000-pair chunks, each compared bit for bit with the
+one-pass call (pairs of reads > 509 bases against haplotypes >= 766 bases within 1e-4, R14). Prints one line per
 round and a final summary; exits non-zero on the first mismatch."""
 import os
 import sys
@@ -25,6 +26,9 @@ def main():
     os.environ["PHMM_PIPE_MIN"] = "512"
     pipe = {p: phmm.PairHMM(precision=p) for p in ("fp32", "fp64")}
     del os.environ["PHMM_PIPE_MIN"]
+    os.environ["PHMM_CHUNK_PAIRS"] = "3000"
+    chunked = {p: phmm.PairHMM(precision=p) for p in ("fp32", "fp64")}
+    del os.environ["PHMM_CHUNK_PAIRS"]
     n_checked = 0
     for r in range(rounds):
         parts = []
@@ -69,11 +73,18 @@ def main():
                     np.max(np.abs(x[dep][fin] - ref[dep][fin]), initial=0.0) <= 1e-4 and
                     np.all((y[dep] <= 1) == (rst[dep] <= 1)))
 
-        ok = same(got, gst) and same(a1, s1) and same(a2, s2)
+        # the device call split into chunks of 3,000 pairs (compute_dev chunking)
+        db = phmm.DeviceBatch.from_host(b, device="cuda:0")
+        c1, cs1 = chunked[prec].compute_batch_dev(db)
+        torch.cuda.synchronize()
+        c1, cs1 = c1.cpu().numpy(), cs1.cpu().numpy()
+        del db
+        ok = same(got, gst) and same(a1, s1) and same(a2, s2) and same(c1, cs1)
         print(f"round {r}: {b.n_pairs} pairs, {prec}, window {win}, chunks {nch}, "
               f"{'pinned' if src is not b else 'pageable'}: {'ok' if ok else 'MISMATCH'}", flush=True)
         if not ok:
-            for name, (x, y) in {"pipelined": (got, gst), "async1": (a1, s1), "async2": (a2, s2)}.items():
+            for name, (x, y) in {"pipelined": (got, gst), "async1": (a1, s1), "async2": (a2, s2),
+                                 "device-chunked": (c1, cs1)}.items():
                 bad = np.nonzero((x != ref) & ~(np.isnan(x) & np.isnan(ref)) & ~dep)[0]
                 sbad = np.nonzero(y != rst)[0]
                 print(f"  {name}: {bad.size} values differ, {sbad.size} statuses differ; first {bad[:10].tolist()}",
