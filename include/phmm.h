@@ -154,10 +154,8 @@ phmm_status phmm_create(phmm_ctx** out, const phmm_config* cfg);
  * and one FP64 rescue pass over the whole batch follows (batches above 2^23 pairs: a rescue
  * per chunk). Fills of device scratch are kernels, not cudaMemsetAsync (which would queue
  * behind the copy stream's transfers). Results are bitwise those of the unpipelined call
- * (PHMM_PIPE=0 at context creation disables it) -- as for any change of batch composition,
- * except pairs of a read longer than 509 bases against a haplotype of >= 766 bases, whose
- * FP32 ring rescale depends on their position in the block stream: those agree within 1e-4
- * in log10 (reading R14). Pairs that use
+ * (PHMM_PIPE=0 at context creation disables it), as for any change of batch composition
+ * (reading R14). Pairs that use
  * reads and haplotypes in ascending index ranges (region after region, as GATK emits them)
  * overlap best; a batch whose first chunk would need more than half of the input bytes
  * runs as one chunk.

@@ -77,6 +77,15 @@ constexpr uint16_t BLK_LAST = 1, BLK_FIRST = 2;
 // is never rescaled, so its result cannot depend on where the pass boundaries fall in it
 constexpr uint16_t BLK_RESC = 4;
 constexpr int kRescaleMinBlocks = 65;
+// filler block after such a pair: the FP32 pass pads every rescalable pair of a long-row bin to a
+// whole number of 64-block passes and sorts them to the front of their bin, so each starts a pass
+// (virtual lane 0) in any stream and its pass boundaries fall at the same rows in every batch
+// (R14); a filler is an idle lane (no table, PAD codes)
+constexpr uint16_t BLK_FILLER = 8;
+constexpr int kRescaleCols = 768;  // long-row kernel (ring rescale) from this many columns on
+__host__ __device__ inline int padded_nb(int nb, int ncols, int align) {
+  return (align && ncols >= kRescaleCols && nb >= kRescaleMinBlocks) ? ((nb + 63) & ~63) : nb;
+}
 
 __host__ __device__ constexpr int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 

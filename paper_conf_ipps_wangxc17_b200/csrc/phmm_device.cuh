@@ -148,7 +148,7 @@ template <int K>
 __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __restrict__ pair_list,
                             const int64_t* __restrict__ n_list_dev, int64_t n_pairs,
                             const int64_t* __restrict__ roff, int64_t n_reads,
-                            const int64_t* __restrict__ hoff, int64_t n_haps, int bucket,
+                            const int64_t* __restrict__ hoff, int64_t n_haps, int bucket, int align,
                             int32_t* __restrict__ pair_bin, int32_t* __restrict__ pair_nb,
                             unsigned long long* __restrict__ bin_blocks, unsigned long long* __restrict__ bin_pairs,
                             int* __restrict__ max_ncols, int* __restrict__ min_ncols_c,
@@ -204,7 +204,7 @@ __global__ void k_pair_bins(const int32_t* __restrict__ pairs, const int32_t* __
           } else {
             const int nc = ncols_of((int)nh, bucket);
             bin = bin_of_ncols(nc, bucket);
-            nb = nblocks_of<K>((int)m);
+            nb = padded_nb(nblocks_of<K>((int)m), nc, align);
             my_max = max(my_max, nc);
             my_minc = max(my_minc, kNcolsComplement - nc);
             my_cells += (unsigned long long)(m * nh);

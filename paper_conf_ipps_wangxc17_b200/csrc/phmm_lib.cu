@@ -339,7 +339,8 @@ phmm_status pass_prepare(phmm_ctx* c, const DevBatch& d, const int32_t* list, in
   const int pb_grid = (int)std::max<int64_t>(grid_for(c, (n + kPairBinsU - 1) / kPairBinsU),
                                               (n + kPairBinsPerCta - 1) / kPairBinsPerCta);
   k_pair_bins<K><<<pb_grid, kThreads, 0, s>>>(
-      d.pairs, list, nullptr, n, d.roff, d.n_reads, d.hoff, d.n_haps, c->bucket, pair_bin, pair_nb, bins,
+      d.pairs, list, nullptr, n, d.roff, d.n_reads, d.hoff, d.n_haps, c->bucket, sizeof(T) == 4 ? 1 : 0, pair_bin,
+      pair_nb, bins,
       bins + nb1, &scal->max_ncols, &scal->min_ncols_c, &scal->cells, &scal->padded_cells, &scal->total_blocks,
       c->gerr ? c->gerr : &scal->err);
   LAUNCHED(c);
@@ -541,13 +542,14 @@ phmm_status pass_run(phmm_ctx* c, const DevBatch& d, const int32_t* list, int64_
   ST_TRY(ws(c, B_SVALS, (size_t)2 * n, &vals));
   ST_TRY(ws(c, B_NBS, (size_t)n + 1, &nbs));
   ST_TRY(ws(c, B_BLKOFF, (size_t)n + 1, &blk_off));
-  k_iota_keys<<<grid_for(c, n), kThreads, 0, s>>>(pair_bin, n, keys, vals);
+  k_iota_keys<<<grid_for(c, n), kThreads, 0, s>>>(pair_bin, pair_nb, n, keys, vals);
   LAUNCHED(c);
   int end_bit = 1;
-  while ((1 << end_bit) <= kMaxBins + 1) ++end_bit;
+  while ((1 << end_bit) <= 2 * (kMaxBins + 1)) ++end_bit;  // keys 2 * bin + class (k_iota_keys)
   size_t sort_bytes = 0, scan_bytes = 0;
   // one length bin (every pair the same column count, e.g. C2): the stable sort is the identity
-  const bool one_bin = pi.min_ncols == pi.max_ncols;
+  // (not for a long-row bin, whose pass-padded pairs must come first)
+  const bool one_bin = pi.min_ncols == pi.max_ncols && pi.max_ncols < kRescaleCols;
   const int32_t* sorted = one_bin ? vals : vals + n;
   if (!one_bin)
     CUDA_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, keys + n, vals, vals + n, n, 0, end_bit, s));

@@ -205,10 +205,12 @@ __global__ void __launch_bounds__(kTabThreads) k_build_table_wf(
 // Pairs are radix-sorted by bin (stable: read-major input order survives inside a bin,
 // the pairs of one read stay adjacent and its table is reused from L2), then each
 // sorted pair gets a contiguous block range from an exclusive scan. Deterministic.
-__global__ void k_iota_keys(const int32_t* __restrict__ pair_bin, int64_t n, uint32_t* __restrict__ keys,
-                            int32_t* __restrict__ vals) {
+// sort keys: 2 * bin + (pair of <= 64 blocks): inside a bin the pass-padded pairs come first
+// (padded_nb), so every one of them starts at a multiple of 64 blocks from any stream start
+__global__ void k_iota_keys(const int32_t* __restrict__ pair_bin, const int32_t* __restrict__ pair_nb, int64_t n,
+                            uint32_t* __restrict__ keys, int32_t* __restrict__ vals) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    keys[i] = (uint32_t)pair_bin[i];
+    keys[i] = 2u * (uint32_t)pair_bin[i] + (pair_nb[i] < kRescaleMinBlocks ? 1u : 0u);
     vals[i] = (int32_t)i;
   }
 }
@@ -237,16 +239,17 @@ __global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t base = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) & ~31ll; base < n; base += stride) {
     const int64_t i = base + lane;
-    int nb = 0, f = 0;
+    int nb = 0, nbr = 0, f = 0;
     int64_t g0 = INT64_MAX, slot = 0;
     uint32_t tab0 = 0, hap = 0;
     if (i < n) {
       const int64_t k = sorted_idx[i];
       const int64_t p = list ? list[k] : k;
-      nb = pair_nb[k];
+      nb = pair_nb[k];  // blocks of the pair incl. fillers (padded_nb)
       const int32_t r = pairs[2 * p], h = pairs[2 * p + 1];
       const int m = (int)(roff[r + 1] - roff[r]);
-      f = nb * K - (m + 2);  // R row index within the pair's rows (f >= 1 Z rows before it)
+      nbr = nblocks_of<K>(m);  // blocks with rows
+      f = nbr * K - (m + 2);   // R row index within the pair's rows (f >= 1 Z rows before it)
       g0 = blk_off[i];
       tab0 = (uint32_t)item_tab_off[pair_item ? pair_item[k] : r];
       hap = (uint32_t)(hc_off[h] + WF_HC_FRONT);
@@ -265,7 +268,7 @@ __global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32
         if (cand < cnt && gc <= pos) e = cand;
       }
       const int64_t g0e = __shfl_sync(0xffffffffu, g0, e);
-      const int nbe = __shfl_sync(0xffffffffu, nb, e);
+      const int nbe = __shfl_sync(0xffffffffu, nbr, e);
       const int fe = __shfl_sync(0xffffffffu, f, e);
       const int64_t slote = __shfl_sync(0xffffffffu, slot, e);
       const uint32_t tabe = __shfl_sync(0xffffffffu, tab0, e);
@@ -279,7 +282,9 @@ __global__ void k_alloc_blocks_wf(const int32_t* __restrict__ pairs, const int32
         d.pad = 0;
         const int rrow = (fe / K == j) ? (fe % K) : WF_RROW_NONE;
         d.flags = (uint16_t)((j == nbe - 1 ? BLK_LAST : 0) | (j == 0 ? BLK_FIRST : 0) |
-                             (nbe >= kRescaleMinBlocks ? BLK_RESC : 0) | (rrow << WF_RROW_SHIFT));
+                             (nbe >= kRescaleMinBlocks ? BLK_RESC : 0) | (j >= nbe ? BLK_FILLER : 0) |
+                             (rrow << WF_RROW_SHIFT));
+        if (j >= nbe) d.out_idx = -1;
         blk[pos] = d;
       }
     }

@@ -88,7 +88,8 @@ constexpr int WF_KC64 = PHMM_F64_K / 2;  // ... of the FP64 pass (K doubles)
 // (the FP64 pass, which reads the same code arrays, scales it by WF_KC64 / WF_KC32)
 constexpr int WF_CB = 2 * WF_KC32;
 
-// BlkDesc.flags: bit0 last, bit1 first, bit2 BLK_RESC (pair of >= 65 blocks), bits 8-11 R row (15 = none)
+// BlkDesc.flags: bit0 last, bit1 first, bit2 BLK_RESC (pair of >= 65 blocks), bit3 BLK_FILLER,
+// bits 8-11 R row (15 = none)
 constexpr uint16_t WF_RROW_SHIFT = 8;
 constexpr uint16_t WF_RROW_NONE = 15;
 
@@ -311,7 +312,7 @@ __device__ __forceinline__ void sts16(uint32_t a, const uint4 v) {
 // before it is read (virtual lane 0 of the next pass). Long rows (ncols >= WF_RESCALE_COLS)
 // get 64 more steps, so that virtual lane 63 has finished its whole row when virtual lane
 // 0 of the next pass starts: the ring rescale then sees the full ring row.
-constexpr int WF_RESCALE_COLS = 768;
+constexpr int WF_RESCALE_COLS = kRescaleCols;
 template <typename T = float>
 __host__ __device__ inline int wf_pass_len(int ncols) {
   constexpr int SH = wf_sh<T>();
@@ -602,7 +603,12 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   __syncwarp();
   if (lane == 0) seg[0] = s;
   __syncwarp();
-  auto phys = [&](int b) -> int64_t { return seg[0] + b; };
+  // FP32 long-row streams start LEAD idle virtual lanes late: the pass-padded (rescalable) pairs,
+  // which sit at multiples of 64 blocks from every stream start (padded_nb, k_iota_keys), then
+  // start half a pass into a pass, so a 1,000-row read crosses two pass boundaries (rows ~250 and
+  // ~760) for its ring rescale, at the same rows in every batch (R14)
+  constexpr int LEAD = (kLong && sizeof(T) == 4) ? 32 : 0;
+  auto phys = [&](int b) -> int64_t { return seg[0] + b - LEAD; };  // b: virtual block index
   using V = typename WfT<T>::V;
   constexpr int K = WfT<T>::K;
   constexpr int PER = 16 / sizeof(T);
@@ -618,7 +624,7 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   const int giA = 2 * (lane % LPG), giB = giA + 1;  // position of each half inside its group
   const T d0 = (T)ldexp(1.0, WfT<T>::kScaleExp) / (T)ncols;  // virtual row 0
   const int P = wf_pass_len<T>(ncols);                        // multiple of 4 (ncols is)
-  int npass = (nblk + 63) >> 6;
+  int npass = (nblk + LEAD + 63) >> 6;
   const int copy_len = wf_hc_copy_len(ncols);
   Lane<T> L;
 #pragma unroll
@@ -646,8 +652,8 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
   BlkDesc dnA, dnB;  // descriptors of the lane's next blocks (loaded one pass ahead)
   dnA.tab_blk = 0; dnA.hap_off = 0; dnA.out_idx = -1; dnA.pad = 0; dnA.flags = 0;
   dnB = dnA;
-  if (2 * lane < nblk) dnA = A.blk[phys(2 * lane)];
-  if (2 * lane + 1 < nblk) dnB = A.blk[phys(2 * lane + 1)];
+  if (2 * lane >= LEAD && 2 * lane < nblk + LEAD) dnA = A.blk[phys(2 * lane)];
+  if (2 * lane + 1 >= LEAD && 2 * lane + 1 < nblk + LEAD) dnB = A.blk[phys(2 * lane + 1)];
 
   // Ring rescale (FP32 pass, long rows only): when a pair continues from
   // virtual lane 63 of one pass into virtual lane 0 of the next, its ring row (the row
@@ -748,8 +754,8 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
       if (e2 == 0) {
         c0 = -1 - SH;  // virtual lane 0 starts its pass
         if constexpr (rescale) {
-          const bool cont = (q < npass) && (q * 64 < nblk) && !(dnA.flags & BLK_FIRST) && (dnA.flags & BLK_RESC) &&
-                            ncols >= WF_RESCALE_COLS;
+          const bool cont = (q < npass) && (q * 64 >= LEAD) && (q * 64 < nblk + LEAD) && !(dnA.flags & BLK_FIRST) &&
+                            (dnA.flags & BLK_RESC) && ncols >= WF_RESCALE_COLS;
           wf_ring_rescale<T, ring_packed<T, kLong>()>((uint64_t)ring_s, ncols, lane, cont,
                                                       A.exp_out ? A.exp_out + dnA.out_idx : nullptr);
         }
@@ -758,8 +764,10 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
       if (grp == e) {
         if (!(e2 & 1)) {  // switch event of virtual lanes 8e..8e+7 = lanes 4e..4e+3
           const int bA = q * 64 + 2 * lane, bB = bA + 1;
-          const bool hA = (q < npass) && (bA < nblk), hB = (q < npass) && (bB < nblk);
           const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
+          // (a filler block after a pass-aligned pair is an idle lane)
+          const bool hA = (q < npass) && (bA >= LEAD) && (bA < nblk + LEAD) && !(dA.flags & BLK_FILLER);
+          const bool hB = (q < npass) && (bB >= LEAD) && (bB < nblk + LEAD) && !(dB.flags & BLK_FILLER);
           if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S row: the last-row M+I sum (L20@2262)
           if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
           pA = wf_stage<0, T>(A, tabA_s, stgA_s, hA, dA, outA, giA, copy_len);
@@ -767,8 +775,8 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
           // the first code word of a block (columns -1-gi-4 .. -2-gi) is PAD
           wA_nx = kPadW; wA_nx2 = __ldg(pA + 1); pA += 2;
           wB_nx = kPadW; wB_nx2 = __ldg(pB + 1); pB += 2;
-          if (bA + 64 < nblk) dnA = A.blk[phys(bA + 64)];
-          if (bB + 64 < nblk) dnB = A.blk[phys(bB + 64)];
+          if (bA + 64 >= LEAD && bA + 64 < nblk + LEAD) dnA = A.blk[phys(bA + 64)];
+          if (bB + 64 >= LEAD && bB + 64 < nblk + LEAD) dnB = A.blk[phys(bB + 64)];
         } else {  // commit of the group that switched 4 steps ago
           wf_commit<0, T>(L, stgA_s, d0);
           wf_commit<1, T>(L, stgB_s, d0);

@@ -17,28 +17,6 @@ from paper_conf_ipps_wangxc17_b200 import phmm, synth
 pytestmark = pytest.mark.gpu
 
 
-def _layout_dependent(b):
-    """Pairs whose FP32 result may depend on their position in the wavefront's block stream:
-    reads of more than 509 bases (more than 64 blocks of 8 rows) against haplotypes of 766 or
-    more bases (the long-row kernel's ring rescale happens at pass boundaries, DESIGN.md §4.5 /
-    reading R14). Every other pair is bitwise batch-independent."""
-    m = b.read_lengths()[b.pairs[:, 0]]
-    n = b.hap_lengths()[b.pairs[:, 1]]
-    return (m > 509) & (n >= 766)
-
-
-def _assert_same(got, gst, ref, rst, b):
-    """Bitwise for batch-independent pairs; within 1e-4 in log10 (the FP32 + rescue tolerance is
-    1e-3) and statuses 0/1 interchangeable for the layout-dependent ones."""
-    dep = _layout_dependent(b)
-    assert np.array_equal(got[~dep], ref[~dep]) and np.array_equal(gst[~dep], rst[~dep])
-    if dep.any():
-        fin = np.isfinite(ref[dep])
-        assert np.all(np.isfinite(got[dep]) == fin)
-        assert np.max(np.abs(got[dep][fin] - ref[dep][fin]), initial=0.0) <= 1e-4
-        assert np.all((gst[dep] <= 1) == (rst[dep] <= 1))
-
-
 @pytest.fixture(scope="module")
 def batch():
     b = synth.config_batch("C2", n_regions=2048)  # 2^18 pairs, 26 MB per read array: several 8 MiB pieces
@@ -236,9 +214,9 @@ def test_pipelined_small_ragged_batches_are_bitwise(prec):
     """The pipelined host call on small, ragged batches (PHMM_PIPE_MIN lowers its threshold):
     multi-bin C3 regions, long C4 rows, random pairs of 1..60 x 1..80 bases (some below the
     40-column minimum) and decoys, with chunks of a few pairs each; pageable and page-locked
-    inputs give the one-pass results bit for bit, statuses included (the C4 pairs -- reads > 509
-    bases against haplotypes >= 766 bases -- within 1e-4: _layout_dependent); also for 16..100
-    pairs, where a chunk may hold a single pair."""
+    inputs give the one-pass results bit for bit, statuses included (the C4 pairs too: their ring
+    rescale happens at the same rows in any batch, R14); also for 16..100 pairs, where a chunk
+    may hold a single pair."""
     import torch
 
     big = synth.concat_batches([synth.config_batch("C2", n_regions=4),
@@ -260,13 +238,13 @@ def test_pipelined_small_ragged_batches_are_bitwise(prec):
             b = big.subset(np.arange(n)) if n < big.n_pairs else big
             ref, rst = flat.compute_batch(b)
             got, gst = pipe.compute_batch(b)
-            _assert_same(got, gst, ref, rst, b)
+            assert np.array_equal(got, ref) and np.array_equal(gst, rst), n
             assert pipe.stats()["n_chunks"] >= 2, (n, pipe.stats()["n_chunks"])
             pin = synth.Batch(**{k: torch.from_numpy(np.ascontiguousarray(getattr(b, k))).pin_memory().numpy()
                                  for k in ("read_bases", "base_quals", "ins_quals", "del_quals", "gcp_quals",
                                            "read_offsets", "hap_bases", "hap_offsets", "pairs")})
             got2, gst2 = pipe.compute_batch(pin)
-            _assert_same(got2, gst2, ref, rst, b)
+            assert np.array_equal(got2, ref) and np.array_equal(gst2, rst), n
     finally:
         flat.close()
         pipe.close()

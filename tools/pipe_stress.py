@@ -1,7 +1,7 @@
 """Stress of the multi-stream host paths: random batch shapes (sizes, region mixes, local pair
 shuffles, page-locked or pageable, FP32 or FP64) through the pipelined host call, the streamed
 async call and the device call split into 3,000-pair chunks, each compared bit for bit with the
-one-pass call (pairs of reads > 509 bases against haplotypes >= 766 bases within 1e-4, R14). Prints one line per
+one-pass call. Prints one line per
 round and a final summary; exits non-zero on the first mismatch."""
 import os
 import sys
@@ -59,11 +59,11 @@ def main():
         t2 = pipe[prec].compute_batch_async(src)
         a1, s1 = t1.wait()
         a2, s2 = t2.wait()
-        # bitwise except the layout-dependent pairs (reads > 509 bases against haplotypes >= 766
-        # bases: the ring rescale at pass boundaries, R14), which agree within 1e-4
+        # bit for bit (PHMM_STRESS_TOL=1: pairs of reads > 509 bases against haplotypes >= 766 bases
+        # only within 1e-4 -- how the library behaved before their pass alignment, R14)
         m = b.read_lengths()[b.pairs[:, 0]]
         nh = b.hap_lengths()[b.pairs[:, 1]]
-        dep = (m > 509) & (nh >= 766)
+        dep = ((m > 509) & (nh >= 766)) if os.environ.get("PHMM_STRESS_TOL") else np.zeros(b.n_pairs, bool)
 
         def same(x, y):
             if not (np.array_equal(x[~dep], ref[~dep]) and np.array_equal(y[~dep], rst[~dep])):
