@@ -766,8 +766,11 @@ __device__ __forceinline__ void wf_stream(const WfArgs2<T>& A, uint32_t ptab_s, 
           const int bA = q * 64 + 2 * lane, bB = bA + 1;
           const BlkDesc dA = dnA, dB = dnB;  // loaded one pass ago (pass 0: before the loop)
           // (a filler block after a pass-aligned pair is an idle lane)
-          const bool hA = (q < npass) && (bA >= LEAD) && (bA < nblk + LEAD) && !(dA.flags & BLK_FILLER);
-          const bool hB = (q < npass) && (bB >= LEAD) && (bB < nblk + LEAD) && !(dB.flags & BLK_FILLER);
+          // (fillers only occur in long-row FP32 streams: the short-row kernel's code stays as it was,
+          // its register allocation is sensitive even to switch-path changes)
+          constexpr bool kFill = LEAD > 0;
+          const bool hA = (q < npass) && (bA >= LEAD) && (bA < nblk + LEAD) && !(kFill && (dA.flags & BLK_FILLER));
+          const bool hB = (q < npass) && (bB >= LEAD) && (bB < nblk + LEAD) && !(kFill && (dB.flags & BLK_FILLER));
           if (outA >= 0) A.out[outA] = lo(L.D[K - 1]);  // S row: the last-row M+I sum (L20@2262)
           if (outB >= 0) A.out[outB] = hi(L.D[K - 1]);
           pA = wf_stage<0, T>(A, tabA_s, stgA_s, hA, dA, outA, giA, copy_len);
