@@ -374,3 +374,17 @@ def test_pipelined_call_with_overlapping_chunk_ranges(window):
     finally:
         flat.close()
         pipe.close()
+
+
+def test_random_shapes_stress_bitwise():
+    """tools/pipe_stress.py for 15 rounds: random batch shapes (C2/C3/C4 region mixes incl. long
+    reads against long haplotypes, local pair shuffles, page-locked or pageable, FP32 or FP64)
+    through the pipelined host call, the streamed async call and the device call in 3,000-pair
+    chunks, each bit for bit the one-pass call (R14)."""
+    import subprocess
+    import sys
+
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "tools", "pipe_stress.py"), "15"], capture_output=True,
+                       text=True, timeout=900, cwd=root)
+    assert r.returncode == 0 and "all 15 rounds bitwise equal" in r.stdout, r.stdout[-3000:] + r.stderr[-2000:]
