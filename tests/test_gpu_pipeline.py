@@ -379,8 +379,9 @@ def test_pipelined_call_with_overlapping_chunk_ranges(window):
 def test_random_shapes_stress_bitwise():
     """tools/pipe_stress.py for 15 rounds: random batch shapes (C2/C3/C4 region mixes incl. long
     reads against long haplotypes, local pair shuffles, page-locked or pageable, FP32 or FP64)
-    through the pipelined host call, the streamed async call and the device call in 3,000-pair
-    chunks, each bit for bit the one-pass call (R14)."""
+    through the pipelined host call, the streamed async call, the device call in 3,000-pair
+    chunks and the submission queue (three slices coalesced by the worker), each bit for bit the
+    one-pass call (R14)."""
     import subprocess
     import sys
 

@@ -1,6 +1,7 @@
 """Stress of the multi-stream host paths: random batch shapes (sizes, region mixes, local pair
 shuffles, page-locked or pageable, FP32 or FP64) through the pipelined host call, the streamed
-async call and the device call split into 3,000-pair chunks, each compared bit for bit with the
+async call, the device call split into 3,000-pair chunks and the submission queue (three slices
+submitted separately, coalesced by the worker), each compared bit for bit with the
 one-pass call. Prints one line per
 round and a final summary; exits non-zero on the first mismatch."""
 import os
@@ -79,12 +80,22 @@ def main():
         torch.cuda.synchronize()
         c1, cs1 = c1.cpu().numpy(), cs1.cpu().numpy()
         del db
-        ok = same(got, gst) and same(a1, s1) and same(a2, s2) and same(c1, cs1)
+        # the submission queue: three slices submitted separately (coalesced into one run on the
+        # worker) must give the slices of the one-pass results
+        cuts = np.sort(rng.choice(np.arange(1, b.n_pairs), size=min(2, b.n_pairs - 1), replace=False))
+        sl = np.split(np.arange(b.n_pairs), cuts)
+        tks = [pipe[prec].submit(b.subset(ix)) for ix in sl]
+        sub = np.empty(b.n_pairs)
+        subst = np.empty(b.n_pairs, np.uint8)
+        for ix, t in zip(sl, tks):
+            o_, st_ = t.wait()
+            sub[ix], subst[ix] = o_, st_
+        ok = same(got, gst) and same(a1, s1) and same(a2, s2) and same(c1, cs1) and same(sub, subst)
         print(f"round {r}: {b.n_pairs} pairs, {prec}, window {win}, chunks {nch}, "
               f"{'pinned' if src is not b else 'pageable'}: {'ok' if ok else 'MISMATCH'}", flush=True)
         if not ok:
             for name, (x, y) in {"pipelined": (got, gst), "async1": (a1, s1), "async2": (a2, s2),
-                                 "device-chunked": (c1, cs1)}.items():
+                                 "device-chunked": (c1, cs1), "submit": (sub, subst)}.items():
                 bad = np.nonzero((x != ref) & ~(np.isnan(x) & np.isnan(ref)) & ~dep)[0]
                 sbad = np.nonzero(y != rst)[0]
                 print(f"  {name}: {bad.size} values differ, {sbad.size} statuses differ; first {bad[:10].tolist()}",
