@@ -42,6 +42,9 @@ def main():
             parts.append(b)
         if rng.random() < 0.3:
             parts.append(synth.random_pairs_batch(int(rng.integers(0, 1 << 30)), int(rng.integers(50, 3000))))
+        if rng.random() < 0.25:  # long random pairs: several passes per pair, several long-row bins
+            parts.append(synth.random_pairs_batch(int(rng.integers(0, 1 << 30)), int(rng.integers(8, 60)),
+                                                  m_range=(300, 2000), n_range=(600, 4094)))
         b = synth.concat_batches(parts)
         win = int(rng.choice([0, 64, 5000]))
         if win:
